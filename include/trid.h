@@ -1,0 +1,124 @@
+/* include/trid.h — C-ABI of libtrid.so: two-stage FP64 symmetric tridiagonalization on B200 (sm_100a).
+ *
+ * Method: Wang et al., "Improving Tridiagonalization Performance on GPU Architectures", PPoPP'25.
+ * Citations P:<line> are lines of that paper's text; R<k> are the readings listed in
+ * DESIGN.md (where the paper is silent, ambiguous or garbled).
+ *
+ * Problem: A in R^{n x n} symmetric  ->  A = Q T Q^T, T tridiagonal, Q orthogonal
+ * (the paper writes A = Q^{-1} T Q; its Q is our Q^T, reading R2).
+ *   stage 1 (Alg. 1, DBBR): full -> band of bandwidth b, Q1 = prod_c (I - tau1[c] v_c v_c^T)
+ *   stage 2 (Alg. 2, BC):   band -> tridiagonal,       Q2 = prod_{s,m} (I - tau2 v v^T)
+ *   Q = Q1 Q2.
+ *
+ * Conventions for every entry point:
+ *   - All array pointers are DEVICE pointers (cudaMalloc / torch CUDA tensors) unless stated otherwise.
+ *   - Column-major (Fortran) storage: element (i, j) of A is A[i + j*lda].  Symmetric matrices are
+ *     referenced through their LOWER triangle only; the strict upper triangle is never read or written
+ *     (reading R6).  A row-major torch (n, n) tensor passed with lda = n is therefore seen transposed:
+ *     for symmetric input that is the same matrix, and our lower triangle is torch's upper triangle.
+ *   - Sizes are 64-bit.  Every call is asynchronous and stream-ordered on `stream`; the library never
+ *     allocates device memory and never synchronizes the host.  The caller owns every buffer.
+ *   - Workspaces come from the matching *_bufsize query (host-only).  Calls are reentrant across
+ *     streams when each call has its own workspace.
+ *   - Errors: argument checks happen on the host before any launch and return -i for the i-th invalid
+ *     argument (LAPACK `info` convention).  CUDA launch errors return TRID_ERR_CUDA.  Faults inside
+ *     kernels surface at the caller's next synchronization (as in cuBLAS).  NaN/Inf inputs are not
+ *     checked and propagate.  No exceptions cross the ABI.
+ */
+#ifndef TRID_H
+#define TRID_H
+
+#include <stddef.h>
+#include <stdint.h>
+#include <cuda_runtime.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  TRID_SUCCESS = 0,
+  TRID_ERR_CUDA = 1,        /* a CUDA runtime call or launch failed */
+  TRID_ERR_NCCL = 2,        /* reserved for the multi-GPU stage-1 path */
+  TRID_ERR_WORKSPACE = 3,   /* dwork_bytes smaller than the *_bufsize result */
+  TRID_ERR_UNSUPPORTED = 4  /* a valid but unsupported configuration (e.g. b > TRID_MAX_B) */
+};
+
+#define TRID_MAX_B 256      /* largest band width / panel width supported */
+
+/* Human-readable status ("success", "invalid argument 3", ...).  Static storage, never NULL. */
+const char* trid_status_string(int status);
+
+/* Library version string, e.g. "trid-b200 0.1 sm_100a". */
+const char* trid_version(void);
+
+/* Default outer block k for DBBR: the largest multiple of b that is <= max(b, 1024) (P:442 uses
+ * b = 32, k = 1024; reading R5). */
+int trid_default_k(int64_t n, int b);
+
+/* Number of bulge-chasing steps of the whole chase (reading R7): sum_{s=0}^{n-3} (floor((n-3-s)/b)+1)
+ * for b >= 2, else 0.  V2 holds b doubles per step, tau2 one. */
+int64_t trid_bc_total_steps(int64_t n, int b);
+
+/* ---- workspace queries (host only; no allocation; no CUDA call) -------------------------------- */
+int trid_sbr_dbbr_bufsize(int64_t n, int b, int nb, int k, size_t* dwork_bytes);
+int trid_bulge_chase_bufsize(int64_t n, int b, size_t* dwork_bytes, int64_t* v2_len, int64_t* tau2_len);
+int trid_sytrd_2stage_bufsize(int64_t n, int b, int nb, int k, size_t* dwork_bytes, int64_t* v2_len,
+                              int64_t* tau2_len);
+
+/* ---- stage 1: double-blocking band reduction (Alg. 1; readings R4a-f) ----------------
+ * In : A (n x n, lda >= max(1,n)), lower triangle = the symmetric input.
+ * Out: the diagonal and the b sub-diagonals of A hold the band B; below the band,
+ *      A(c+b+1 : n-1, c) holds the SBR Householder vector of column c (unit entry at row c+b implicit),
+ *      tau1[c] its scalar (tau1[c] = 0 for c >= n-b-1).  tau1 has n entries.
+ * b  : band width = panel width, 1 <= b <= TRID_MAX_B.
+ * nb : inner block of the panel QR (R5), 1 <= nb <= b, b % nb == 0 (performance knob only).
+ * k  : outer block = syr2k rank, k == 0 -> trid_default_k(n, b); else k >= b, k % b == 0.
+ * b >= n-1 is a legal no-op (tau1 = 0).  dwork: trid_sbr_dbbr_bufsize bytes, 256-byte aligned. */
+int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* tau1,
+                  void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+/* ---- stage 2: bulge chasing on the GPU (sec. 2.4 Fig. 3, Alg. 2; readings R7-R9) -------
+ * In : band B of bandwidth b in A's lower band (diagonal + b sub-diagonals), as left by
+ *      trid_sbr_dbbr.  Entries below the band are ignored.  A is not modified.
+ * Out: d[n], e[n-1] with T = tridiag(e, d, e) (reading R8); V2[trid_bc_total_steps(n,b) * b] and
+ *      tau2[trid_bc_total_steps(n,b)] hold the BC reflectors: step m of sweep s stores its vector
+ *      (v[0] = 1 explicit, zero padded to b) at V2 + (S(s)+m)*b and its scalar at tau2[S(s)+m],
+ *      S(s) = sum_{s'<s} steps(s'); it acts on rows s+1+m*b .. min(s+(m+1)*b, n-1) (reading R7).
+ *      V2 == NULL && tau2 == NULL selects eigenvalues-only mode.
+ * Sweeps run concurrently, pipelined at lag 2 by release/acquire progress counters (R9); the result
+ * is bitwise identical to the sweep-major order. */
+int trid_bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
+                     double* tau2, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+/* ---- both stages: A = Q T Q^T with Q = Q1 Q2 (Q1 from tau1 and the vectors below A's band, Q2 from
+ * V2/tau2).  k = 0 -> trid_default_k.  Argument meanings as above. */
+int trid_sytrd_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* d, double* e,
+                      double* tau1, double* V2, double* tau2, void* dwork, size_t dwork_bytes,
+                      cudaStream_t stream);
+
+/* ---- hot-path building blocks, exposed for unit parity tests ------------ */
+
+/* a1+a2: Householder QR of the m x w panel P (ld ldp), in place: R in the upper triangle, V below it
+ * (unit diagonal implicit), tau[min(m,w)]; T (w x w, ld ldt, upper triangular, dlarft forward
+ * columnwise) and Y (m x min(m,w), ld ldy: V made explicit with unit diagonal and zeros above) such
+ * that H_1 ... H_kk = I - Y T Y^T.  w <= TRID_MAX_B.  Workspace: trid_panel_qr_bufsize. */
+int trid_panel_qr_bufsize(int64_t m, int w, size_t* dwork_bytes);
+int trid_panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt,
+                  double* Y, int64_t ldy, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+/* a5 / a4: C -= Y Z^T + Z Y^T on the lower triangle of the m x m matrix C (strict upper untouched);
+ * Y, Z are m x kk.  The DMMA syr2k of Alg. 1 l.15 (Fig. 7). */
+int trid_syr2k_lower(int64_t m, int64_t kk, double* C, int64_t ldc, const double* Y, int64_t ldy,
+                     const double* Z, int64_t ldz, cudaStream_t stream);
+
+/* a3: X = A W for A (m x m symmetric, lower referenced, ld lda) and W (m x w), then
+ * Z = X - 1/2 Y (W^T X) (Eq. (1)).  Workspace: trid_zy_bufsize. */
+int trid_zy_bufsize(int64_t m, int w, size_t* dwork_bytes);
+int trid_zy(int64_t m, int w, const double* A, int64_t lda, const double* W, int64_t ldw, const double* Y,
+            int64_t ldy, double* Z, int64_t ldz, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TRID_H */

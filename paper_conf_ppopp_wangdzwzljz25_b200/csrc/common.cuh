@@ -1,0 +1,99 @@
+// common.cuh — device helpers shared by the libtrid kernels (sm_100a only).
+// FP64 tensor-core math on Blackwell: tcgen05 has no f64 kind, so FP64 contractions use the warp-level
+// DMMA path (mma.sync ... f64, SASS DMMA.8x8x4).  Measured on this pool's B200: 37.0 TFLOP/s for DMMA
+// and 36.7 for DFMA at 1965 MHz (profiles/r01_fp64_microbench.jsonl).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ != 1000)
+#error "libtrid is written for sm_100a only"
+#endif
+
+namespace trid {
+
+constexpr int kNumSMsB200 = 148;
+
+// D(16x8) += A(16x8) * B(8x8), fp64.  Fragment layout (verified on B200, tools/microbench_fp64.cu):
+//   g = lane>>2, t = lane&3;  a[i] = A[g + 8*(i&1)][t + 4*(i>>1)];  b[i] = B[t + 4*i][g];
+//   c[0] = C[g][2t], c[1] = C[g][2t+1], c[2] = C[g+8][2t], c[3] = C[g+8][2t+1].
+__device__ __forceinline__ void dmma_16x8x8(double (&c)[4], const double (&a)[4], const double (&b)[2]) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k8.row.col.f64.f64.f64.f64 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};\n"
+      : "+d"(c[0]), "+d"(c[1]), "+d"(c[2]), "+d"(c[3])
+      : "d"(a[0]), "d"(a[1]), "d"(a[2]), "d"(a[3]), "d"(b[0]), "d"(b[1]));
+}
+
+// 8-byte async copy global -> shared; pred == false zero-fills without reading global memory.
+__device__ __forceinline__ void cp_async8(double* smem, const double* gmem, bool pred) {
+  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  int sz = pred ? 8 : 0;
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(sz) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int ld_acquire_s32(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_s32(int* p, int v) {
+  asm volatile("st.release.gpu.global.s32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
+}
+
+// Grid-wide barrier for a cooperatively launched grid.  `counter` is zero at launch; `epoch` is a
+// per-CTA register copy of how many barriers this CTA has passed.  Monotone counter: no reset race.
+__device__ __forceinline__ void grid_barrier(unsigned* counter, unsigned nblocks, unsigned& epoch) {
+  __syncthreads();
+  epoch += 1;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(counter, 1u);
+    const unsigned target = epoch * nblocks;
+    while (ld_acquire_u32(counter) < target) {
+    }
+  }
+  __syncthreads();
+}
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// LAPACK dlarfg sign convention (R1/R1'): beta = -sign(alpha)*sqrt(alpha^2+sigma) with the
+// sign taken from the sign bit; sigma == 0 -> tau = 0, beta = alpha, scale = 0 (no reflection).
+struct House {
+  double beta, tau, scale;
+};
+__device__ __forceinline__ House make_house(double alpha, double sigma) {
+  House h;
+  if (sigma == 0.0) {
+    h.beta = alpha;
+    h.tau = 0.0;
+    h.scale = 0.0;
+  } else {
+    double nrm = sqrt(alpha * alpha + sigma);
+    h.beta = signbit(alpha) ? nrm : -nrm;
+    h.tau = (h.beta - alpha) / h.beta;
+    h.scale = 1.0 / (alpha - h.beta);
+  }
+  return h;
+}
+
+}  // namespace trid
+
+#define TRID_CUDA_TRY(x)                        \
+  do {                                          \
+    cudaError_t _e = (x);                       \
+    if (_e != cudaSuccess) return TRID_ERR_CUDA; \
+  } while (0)

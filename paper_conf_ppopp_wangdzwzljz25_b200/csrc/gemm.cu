@@ -1,0 +1,393 @@
+// gemm.cu — FP64 DMMA contraction engine for the DBBR hot path.
+//
+// One templated CTA-tile mainloop (cp.async 3-stage smem ring, DMMA m16n8k8 f64 from padded smem
+// fragments) serves:
+//   * the deferred syr2k  C -= Y Z^T + Z Y^T, lower triangle only, triangular tile grid  (Alg. 1 l.15,
+//     Fig. 7: independent square tiles, reorderable)
+//   * the next-panel update                                                    (Alg. 1 l.8-12)
+//   * W = Y T, corrections and Z = X - 1/2 Y (W^T X)                            (Eq. (1))
+//   * the SYMM X = A W of the Z builder (symm_kernel: row strip + transposed column strip per row
+//     block, so the lower-stored trailing matrix is read without atomics; deterministic split-K).
+// Padded smem strides keep DMMA fragment loads at the 2-wavefront minimum (row stride = 8 mod 16
+// doubles for m-inner tiles, 4 mod 16 for k-inner tiles).
+#include "common.cuh"
+#include "gemm.cuh"
+
+namespace trid {
+
+constexpr int BK = 16;
+constexpr int STAGES = 3;
+
+template <int BM, int OPA>
+struct ATile {
+  static constexpr int LD = OPA == OP_N ? BM + 8 : BK + 4;
+  static constexpr int ELEMS = OPA == OP_N ? BK * (BM + 8) : BM * (BK + 4);
+  __device__ static __forceinline__ int idx(int r, int k) { return OPA == OP_N ? k * LD + r : r * LD + k; }
+};
+template <int BN, int OPB>
+struct BTile {
+  static constexpr int LD = OPB == OP_T ? BN + 8 : BK + 4;
+  static constexpr int ELEMS = OPB == OP_T ? BK * (BN + 8) : BN * (BK + 4);
+  __device__ static __forceinline__ int idx(int k, int c) { return OPB == OP_T ? k * LD + c : c * LD + k; }
+};
+
+template <int BM, int BN>
+constexpr int stage_elems_max() {
+  return (ATile<BM, OP_N>::ELEMS > ATile<BM, OP_T>::ELEMS ? ATile<BM, OP_N>::ELEMS : ATile<BM, OP_T>::ELEMS) +
+         (BTile<BN, OP_N>::ELEMS > BTile<BN, OP_T>::ELEMS ? BTile<BN, OP_N>::ELEMS : BTile<BN, OP_T>::ELEMS);
+}
+
+// MASK: 0 none; 1 keep (k <= row)  [SYMM row strip incl. diagonal]; 2 keep (k > row) [SYMM column strip]
+template <int BM, int BN, int NT, int OPA, int OPB, int MASK>
+__device__ __forceinline__ void load_stage(double* As, double* Bs, const double* A, int64_t lda, const double* B,
+                                           int64_t ldb, int64_t m0, int64_t n0, int64_t M, int64_t N, int64_t k0,
+                                           int64_t kend) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int e = tid; e < BM * BK; e += NT) {
+    int r, kk;
+    if (OPA == OP_N) { r = e % BM; kk = e / BM; } else { kk = e % BK; r = e / BK; }
+    const int64_t row = m0 + r, k = k0 + kk;
+    bool p = row < M && k < kend;
+    if (MASK == 1) p = p && (k <= row);
+    if (MASK == 2) p = p && (k > row);
+    const double* src = A;
+    if (p) src = OPA == OP_N ? A + row + k * lda : A + k + row * lda;
+    cp_async8(As + ATile<BM, OPA>::idx(r, kk), src, p);
+  }
+#pragma unroll
+  for (int e = tid; e < BN * BK; e += NT) {
+    int c, kk;
+    if (OPB == OP_T) { c = e % BN; kk = e / BN; } else { kk = e % BK; c = e / BK; }
+    const int64_t col = n0 + c, k = k0 + kk;
+    const bool p = col < N && k < kend;
+    const double* src = B;
+    if (p) src = OPB == OP_N ? B + k + col * ldb : B + col + k * ldb;
+    cp_async8(Bs + BTile<BN, OPB>::idx(kk, c), src, p);
+  }
+}
+
+// Accumulate op(A)[m0:m0+BM, kbeg:kend] * op(B)[kbeg:kend, n0:n0+BN] into acc.
+template <int BM, int BN, int WGM, int WGN, int OPA, int OPB, int MASK>
+__device__ __forceinline__ void mainloop(double (&acc)[BM / WGM / 16][BN / WGN / 8][4], double* smem, const double* A,
+                                         int64_t lda, const double* B, int64_t ldb, int64_t m0, int64_t n0,
+                                         int64_t M, int64_t N, int64_t kbeg, int64_t kend) {
+  constexpr int NT = WGM * WGN * 32;
+  constexpr int WTM = BM / WGM, WTN = BN / WGN;
+  constexpr int MT = WTM / 16, NTL = WTN / 8;
+  constexpr int AE = ATile<BM, OPA>::ELEMS, BE = BTile<BN, OPB>::ELEMS;
+  if (kend <= kbeg) return;
+  const int ntile = (int)((kend - kbeg + BK - 1) / BK);
+  double* As = smem;
+  double* Bs = smem + STAGES * AE;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int wm = warp % WGM, wn = warp / WGM;
+  const int g = lane >> 2, t = lane & 3;
+  __syncthreads();  // previous users of smem are done
+#pragma unroll
+  for (int s = 0; s < STAGES - 1; ++s) {
+    if (s < ntile)
+      load_stage<BM, BN, NT, OPA, OPB, MASK>(As + s * AE, Bs + s * BE, A, lda, B, ldb, m0, n0, M, N, kbeg + s * BK,
+                                             kend);
+    cp_async_commit();
+  }
+  for (int it = 0; it < ntile; ++it) {
+    cp_async_wait<STAGES - 2>();
+    __syncthreads();
+    const int nxt = it + STAGES - 1;
+    if (nxt < ntile) {
+      const int st = nxt % STAGES;
+      load_stage<BM, BN, NT, OPA, OPB, MASK>(As + st * AE, Bs + st * BE, A, lda, B, ldb, m0, n0, M, N,
+                                             kbeg + (int64_t)nxt * BK, kend);
+    }
+    cp_async_commit();
+    const double* Ast = As + (it % STAGES) * AE;
+    const double* Bst = Bs + (it % STAGES) * BE;
+#pragma unroll
+    for (int ks = 0; ks < BK; ks += 8) {
+      double af[MT][4], bf[NTL][2];
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt) {
+        const int r = wm * WTM + mt * 16 + g;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) af[mt][i] = Ast[ATile<BM, OPA>::idx(r + 8 * (i & 1), ks + t + 4 * (i >> 1))];
+      }
+#pragma unroll
+      for (int nt = 0; nt < NTL; ++nt) {
+        const int c = wn * WTN + nt * 8 + g;
+#pragma unroll
+        for (int i = 0; i < 2; ++i) bf[nt][i] = Bst[BTile<BN, OPB>::idx(ks + t + 4 * i, c)];
+      }
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTL; ++nt) dmma_16x8x8(acc[mt][nt], af[mt], bf[nt]);
+    }
+  }
+  cp_async_wait<0>();
+}
+
+__device__ __forceinline__ void tri_tile(int64_t t, int& tm, int& tn) {
+  int64_t r = (int64_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+  while (r * (r + 1) / 2 > t) --r;
+  while ((r + 1) * (r + 2) / 2 <= t) ++r;
+  tm = (int)r;
+  tn = (int)(t - r * (r + 1) / 2);
+}
+
+template <int BM, int BN, int WGM, int WGN, int OPA, int OPB>
+__global__ void __launch_bounds__(WGM* WGN * 32) gemm_kernel(GemmArgs a) {
+  constexpr int WTM = BM / WGM, WTN = BN / WGN;
+  constexpr int MT = WTM / 16, NTL = WTN / 8;
+  extern __shared__ __align__(16) double smem[];
+  int tm, tn;
+  if (a.tri) {
+    tri_tile(blockIdx.x, tm, tn);
+  } else {
+    tm = blockIdx.x;
+    tn = blockIdx.y;
+  }
+  const int64_t m0 = (int64_t)tm * BM, n0 = (int64_t)tn * BN;
+  if (a.lower && m0 + BM - 1 + a.diag_off < n0) return;
+  double acc[MT][NTL][4];
+#pragma unroll
+  for (int i = 0; i < MT; ++i)
+#pragma unroll
+    for (int j = 0; j < NTL; ++j)
+#pragma unroll
+      for (int q = 0; q < 4; ++q) acc[i][j][q] = 0.0;
+
+  // split-K over the concatenated, BK-aligned segments
+  const int64_t kt0 = (a.K[0] + BK - 1) / BK, kt1 = a.nseg > 1 ? (a.K[1] + BK - 1) / BK : 0;
+  const int64_t total = kt0 + kt1;
+  const int z = blockIdx.z;
+  const int64_t per = (total + a.splits - 1) / a.splits;
+  const int64_t tb = (int64_t)z * per, te = (tb + per < total) ? tb + per : total;
+  if (tb < kt0) {
+    const int64_t e = te < kt0 ? te : kt0;
+    const int64_t kb = tb * BK, ke = (e * BK < a.K[0]) ? e * BK : a.K[0];
+    mainloop<BM, BN, WGM, WGN, OPA, OPB, 0>(acc, smem, a.A[0], a.lda[0], a.B[0], a.ldb[0], m0, n0, a.M, a.N, kb, ke);
+  }
+  if (te > kt0) {
+    const int64_t b0 = (tb > kt0 ? tb : kt0) - kt0, e = te - kt0;
+    const int64_t kb = b0 * BK, ke = (e * BK < a.K[1]) ? e * BK : a.K[1];
+    mainloop<BM, BN, WGM, WGN, OPA, OPB, 0>(acc, smem, a.A[1], a.lda[1], a.B[1], a.ldb[1], m0, n0, a.M, a.N, kb, ke);
+  }
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int wm = warp % WGM, wn = warp / WGM;
+  const int g = lane >> 2, t = lane & 3;
+#pragma unroll
+  for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < NTL; ++nt)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int64_t r = m0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
+        const int64_t c = n0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
+        if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= c)) {
+          if (a.splits > 1) {
+            a.part[z * a.part_stride + r + c * a.part_ld] = acc[mt][nt][i];
+          } else {
+            double v = a.alpha * acc[mt][nt][i];
+            if (a.beta != 0.0) v += a.beta * a.Cin[r + c * a.ldcin];
+            a.C[r + c * a.ldc] = v;
+          }
+        }
+      }
+}
+
+__global__ void reduce_partials_kernel(GemmArgs a) {
+  const int64_t total = a.M * a.N;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = idx % a.M, c = idx / a.M;
+    if (a.lower && r + a.diag_off < c) continue;
+    double s = 0.0;
+    for (int z = 0; z < a.splits; ++z) s += a.part[z * a.part_stride + r + c * a.part_ld];
+    double v = a.alpha * s;
+    if (a.beta != 0.0) v += a.beta * a.Cin[r + c * a.ldcin];
+    a.C[r + c * a.ldc] = v;
+  }
+}
+
+template <int BM, int BN, int WGM, int WGN, int OPA, int OPB>
+static cudaError_t launch_tile(const GemmArgs& a, cudaStream_t st) {
+  constexpr int NT = WGM * WGN * 32;
+  constexpr size_t smem = sizeof(double) * STAGES * (ATile<BM, OPA>::ELEMS + BTile<BN, OPB>::ELEMS);
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BM, BN, WGM, WGN, OPA, OPB>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  const int64_t tm = (a.M + BM - 1) / BM, tn = (a.N + BN - 1) / BN;
+  dim3 grid;
+  if (a.tri) {
+    grid = dim3((unsigned)(tm * (tm + 1) / 2), 1, (unsigned)a.splits);
+  } else {
+    grid = dim3((unsigned)tm, (unsigned)tn, (unsigned)a.splits);
+  }
+  gemm_kernel<BM, BN, WGM, WGN, OPA, OPB><<<grid, NT, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+template <int OPA, int OPB>
+static cudaError_t launch_ops(const GemmArgs& a, int tile, cudaStream_t st) {
+  switch (tile) {
+    case TILE_128x128: return launch_tile<128, 128, 2, 4, OPA, OPB>(a, st);
+    case TILE_128x64: return launch_tile<128, 64, 4, 2, OPA, OPB>(a, st);
+    default: return launch_tile<64, 64, 2, 2, OPA, OPB>(a, st);
+  }
+}
+
+cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
+  if (a.M <= 0 || a.N <= 0) return cudaSuccess;
+  if (a.K[0] <= 0 && (a.nseg < 2 || a.K[1] <= 0)) {
+    // pure scaling: C = beta * Cin (K == 0); reuse the reduction kernel with zero splits
+    GemmArgs r = a;
+    r.splits = 0;
+    reduce_partials_kernel<<<592, 256, 0, st>>>(r);
+    return cudaGetLastError();
+  }
+  if (a.splits < 1) a.splits = 1;
+  cudaError_t e;
+  if (opA == OP_N && opB == OP_N) e = launch_ops<OP_N, OP_N>(a, tile, st);
+  else if (opA == OP_N && opB == OP_T) e = launch_ops<OP_N, OP_T>(a, tile, st);
+  else if (opA == OP_T && opB == OP_N) e = launch_ops<OP_T, OP_N>(a, tile, st);
+  else e = launch_ops<OP_T, OP_T>(a, tile, st);
+  if (e != cudaSuccess || a.splits == 1) return e;
+  int64_t total = a.M * a.N;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 4 * kNumSMsB200 * 4) blocks = 4 * kNumSMsB200 * 4;
+  reduce_partials_kernel<<<blocks, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems) {
+  const int bm = tile == TILE_64x64 ? 64 : 128, bn = tile == TILE_128x128 ? 128 : 64;
+  const int64_t tiles = ((M + bm - 1) / bm) * ((N + bn - 1) / bn);
+  const int64_t target = 2 * kNumSMsB200;
+  int64_t s = (target + tiles - 1) / tiles;
+  const int64_t maxk = (K + 255) / 256;  // keep >= 256 of K per split
+  if (s > maxk) s = maxk;
+  if (s * M * N > max_part_elems) s = max_part_elems / (M * N);
+  if (s < 1) s = 1;
+  if (s > 128) s = 128;
+  return (int)s;
+}
+
+// ------------------------------------------------------------------------------------------------
+// SYMM: X[r0:r0+BM, c0:c0+BN] = sum_k Asym(r, k) W(k, c) over the CTA's K chunk.
+//   phase 1 (row strip):    Asym(r, k) = A(r, k)   for k <= r   (k in [k0, min(k1, r0+BM)))
+//   phase 2 (column strip): Asym(r, k) = A(k, r)   for k >  r   (k in [max(k0, r0), k1))
+// Every CTA owns whole output tiles -> no atomics; split-K partials are reduced in fixed order.
+struct SymmArgs {
+  int64_t m, w;
+  const double* A;
+  int64_t lda;
+  const double* W;
+  int64_t ldw;
+  double* X;
+  int64_t ldx;
+  int64_t chunk;
+  int nchunk;
+  double* part;
+  int64_t part_stride;
+};
+
+constexpr int SY_BM = 128, SY_BN = 64, SY_WGM = 4, SY_WGN = 2;
+
+__global__ void __launch_bounds__(SY_WGM* SY_WGN * 32) symm_kernel(SymmArgs a) {
+  constexpr int WTM = SY_BM / SY_WGM, WTN = SY_BN / SY_WGN;
+  constexpr int MT = WTM / 16, NTL = WTN / 8;
+  extern __shared__ __align__(16) double smem[];
+  const int64_t r0 = (int64_t)blockIdx.x * SY_BM, c0 = (int64_t)blockIdx.y * SY_BN;
+  const int z = blockIdx.z;
+  const int64_t k0 = (int64_t)z * a.chunk;
+  const int64_t k1 = (k0 + a.chunk < a.m) ? k0 + a.chunk : a.m;
+  double acc[MT][NTL][4];
+#pragma unroll
+  for (int i = 0; i < MT; ++i)
+#pragma unroll
+    for (int j = 0; j < NTL; ++j)
+#pragma unroll
+      for (int q = 0; q < 4; ++q) acc[i][j][q] = 0.0;
+  {
+    const int64_t e1 = (k1 < r0 + SY_BM) ? k1 : r0 + SY_BM;
+    mainloop<SY_BM, SY_BN, SY_WGM, SY_WGN, OP_N, OP_N, 1>(acc, smem, a.A, a.lda, a.W, a.ldw, r0, c0, a.m, a.w, k0, e1);
+    const int64_t s2 = (k0 > r0) ? k0 : r0;
+    mainloop<SY_BM, SY_BN, SY_WGM, SY_WGN, OP_T, OP_N, 2>(acc, smem, a.A, a.lda, a.W, a.ldw, r0, c0, a.m, a.w, s2, k1);
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int wm = warp % SY_WGM, wn = warp / SY_WGM;
+  const int g = lane >> 2, t = lane & 3;
+#pragma unroll
+  for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+    for (int nt = 0; nt < NTL; ++nt)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int64_t r = r0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
+        const int64_t c = c0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
+        if (r < a.m && c < a.w) {
+          if (a.nchunk > 1) a.part[z * a.part_stride + r + c * a.m] = acc[mt][nt][i];
+          else a.X[r + c * a.ldx] = acc[mt][nt][i];
+        }
+      }
+}
+
+static int symm_nchunk(int64_t m, int64_t w) {
+  const int64_t blocks = ((m + SY_BM - 1) / SY_BM) * ((w + SY_BN - 1) / SY_BN);
+  const int64_t target = 3 * kNumSMsB200;  // ~3 CTAs per SM in flight for balance
+  int64_t c = (target + blocks - 1) / blocks;
+  const int64_t maxc = (m + 1023) / 1024;  // >= 1024 strip columns per chunk
+  if (c > maxc) c = maxc;
+  if (c > 32) c = 32;
+  if (c < 1) c = 1;
+  return (int)c;
+}
+
+int64_t symm_part_elems(int64_t m, int64_t w) {
+  int c = symm_nchunk(m, w);
+  return c > 1 ? (int64_t)c * m * w : 0;
+}
+
+cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw,
+                       double* X, int64_t ldx, double* part, int64_t part_elems, cudaStream_t st) {
+  if (m <= 0 || w <= 0) return cudaSuccess;
+  constexpr size_t smem =
+      sizeof(double) * STAGES *
+      ((ATile<SY_BM, OP_N>::ELEMS > ATile<SY_BM, OP_T>::ELEMS ? ATile<SY_BM, OP_N>::ELEMS : ATile<SY_BM, OP_T>::ELEMS) +
+       BTile<SY_BN, OP_N>::ELEMS);
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(symm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  SymmArgs a;
+  a.m = m; a.w = w; a.A = A; a.lda = lda; a.W = W; a.ldw = ldw; a.X = X; a.ldx = ldx;
+  int nc = symm_nchunk(m, w);
+  if ((int64_t)nc * m * w > part_elems) nc = 1;
+  a.nchunk = nc;
+  a.chunk = (((m + nc - 1) / nc) + BK - 1) / BK * BK;
+  a.nchunk = (int)((m + a.chunk - 1) / a.chunk);
+  a.part = part;
+  a.part_stride = m * w;
+  dim3 grid((unsigned)((m + SY_BM - 1) / SY_BM), (unsigned)((w + SY_BN - 1) / SY_BN), (unsigned)a.nchunk);
+  symm_kernel<<<grid, SY_WGM * SY_WGN * 32, smem, st>>>(a);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || a.nchunk == 1) return e;
+  GemmArgs r;
+  r.M = m; r.N = w; r.alpha = 1.0; r.beta = 0.0; r.C = X; r.ldc = ldx;
+  r.splits = a.nchunk; r.part = part; r.part_ld = m; r.part_stride = m * w;
+  int64_t total = m * w;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 16 * kNumSMsB200) blocks = 16 * kNumSMsB200;
+  reduce_partials_kernel<<<blocks, 256, 0, st>>>(r);
+  return cudaGetLastError();
+}
+
+}  // namespace trid

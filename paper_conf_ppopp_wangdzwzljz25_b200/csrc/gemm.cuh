@@ -1,0 +1,53 @@
+// gemm.cuh — FP64 DMMA contraction engine (host launchers).  See gemm.cu.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace trid {
+
+enum { OP_N = 0, OP_T = 1 };
+enum { TILE_128x128 = 0, TILE_128x64 = 1, TILE_64x64 = 2 };
+
+// C = alpha * sum_seg op(A_seg) op(B_seg) + beta * Cin, M x N, column-major.
+//   op(A) = A   : A is M x K  (element (m,k) at A[m + k*lda])        OP_N
+//   op(A) = A^T : A is K x M  (element (k,m) at A[k + m*lda])        OP_T
+//   op(B) = B   : B is K x N  (element (k,n) at B[k + n*ldb])        OP_N
+//   op(B) = B^T : B is N x K  (element (n,k) at B[n + k*ldb])        OP_T
+// lower != 0: only elements with row + diag_off >= col are written (tiles wholly above are skipped).
+// tri != 0  : blockIdx.x enumerates the lower-triangular tiles of a square tiling (syr2k, Fig. 7).
+// splits > 1: deterministic split-K; partial z goes to part + z*part_stride (ld part_ld), then
+//             reduce_partials() forms C in fixed order.
+struct GemmArgs {
+  int64_t M = 0, N = 0;
+  int nseg = 1;
+  const double* A[2] = {nullptr, nullptr};
+  int64_t lda[2] = {1, 1};
+  const double* B[2] = {nullptr, nullptr};
+  int64_t ldb[2] = {1, 1};
+  int64_t K[2] = {0, 0};
+  double alpha = 1.0, beta = 0.0;
+  const double* Cin = nullptr;
+  int64_t ldcin = 1;
+  double* C = nullptr;
+  int64_t ldc = 1;
+  int lower = 0;
+  int64_t diag_off = 0;
+  int tri = 0;
+  int splits = 1;
+  double* part = nullptr;
+  int64_t part_ld = 1, part_stride = 0;
+};
+
+// Launch; when a.splits > 1 also launches the reduction.  Returns the first CUDA error.
+cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st);
+
+// Choose a split count so the grid fills the machine for a tall reduction (K >> M, N).
+int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems);
+
+// X = Asym * W (m x w), Asym lower-referenced, ld lda.  Split-K over the strip when the row-block grid
+// is too small; partials need symm_part_elems() doubles.
+cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw,
+                       double* X, int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);
+int64_t symm_part_elems(int64_t m, int64_t w);
+
+}  // namespace trid

@@ -1,0 +1,21 @@
+// panel.cuh — host launchers for the panel QR (panel_qr.cu) and the bulge chase (bulge.cu).
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+namespace trid {
+
+// Panel QR + T + explicit Y (see panel_qr.cu).  red: panel_red_bytes(w) bytes; bar: one zeroed word.
+size_t panel_red_bytes(int w);
+cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
+                     int64_t ldy, double* red, unsigned* bar, cudaStream_t st);
+
+// Bulge chasing (see bulge.cu).
+int bc_ldab(int64_t n, int b);
+int64_t bc_total_steps(int64_t n, int b);
+size_t bc_work_bytes(int64_t n, int b);
+cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
+                        double* tau2, void* work, cudaStream_t st);
+
+}  // namespace trid

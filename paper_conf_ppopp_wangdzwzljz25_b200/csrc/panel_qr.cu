@@ -1,0 +1,204 @@
+// panel_qr.cu — tall-skinny Householder panel QR for DBBR (Alg. 1 line 5) plus the
+// compact-WY factor T (dlarft forward-columnwise) and the explicit Y = V.
+//
+// B200 design: one cooperative persistent grid of G <= 148 CTAs; CTA g owns a contiguous block of
+// panel rows, staged in shared memory when it fits (<= ~220 KB).  Column t needs ONE grid-wide
+// reduction: every CTA contributes the Gram row  sum_{r>t} x_r P(r,j)  (x = column t below row t,
+// unscaled) for all j and the owner of row t contributes P(t, :).  From those totals every CTA
+// derives, identically and deterministically, beta/tau/scale of the reflector (R1), the update
+// vector w_j = v^T P(:,j) = P(t,j) + scale * sum x_r P(r,j) (j > t) and the T-factor inner products
+// v_t^T v_q (q < t), then applies the rank-1 update to its own rows.  Totals are summed in a fixed
+// CTA order, so every CTA (and every run) sees bitwise-identical values.
+#include "common.cuh"
+#include "panel.cuh"
+
+namespace trid {
+
+constexpr int PQ_NT = 256;
+
+struct PanelArgs {
+  int64_t m;
+  int w, kk;
+  double* P;
+  int64_t ldp;
+  double* tau;
+  double* T;
+  int64_t ldt;
+  double* Y;
+  int64_t ldy;
+  double* red;
+  unsigned* bar;
+  int rows;      // rows per CTA
+  int smem_ld;   // > 0: rows staged in shared memory with this leading dimension
+};
+
+__global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
+  extern __shared__ __align__(16) double sm[];
+  const int g = blockIdx.x, G = gridDim.x, tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
+  constexpr int NW = PQ_NT / 32;
+  const int w = a.w, RS = 2 * w;
+  const int64_t rlo = (int64_t)g * a.rows;
+  const int nr = (int)((rlo + a.rows <= a.m) ? a.rows : (a.m > rlo ? a.m - rlo : 0));
+
+  double* L;
+  int64_t ldl;
+  double* scr;
+  if (a.smem_ld > 0) {
+    L = sm;
+    ldl = a.smem_ld;
+    scr = sm + (size_t)a.smem_ld * w;
+    for (int idx = tid; idx < nr * w; idx += PQ_NT) {
+      const int i = idx % nr, j = idx / nr;
+      L[(size_t)j * ldl + i] = a.P[(rlo + i) + (int64_t)j * a.ldp];
+    }
+  } else {
+    L = a.P + rlo;
+    ldl = a.ldp;
+    scr = sm;
+  }
+  double* tot = scr;            // RS totals
+  double* wv = tot + RS;        // w: update vector (j > t) / v_t^T v_q (q < t)
+  double* tmp = wv + w;         // H*RS <= PQ_NT partial totals
+  double* hs = tmp + PQ_NT;     // beta, tau, scale
+  __syncthreads();
+
+  unsigned epoch = 0;
+  const int H = (RS <= PQ_NT) ? PQ_NT / RS : 1;
+  for (int t = 0; t < a.kk; ++t) {
+    double* red = a.red + (size_t)(t & 1) * G * RS;
+    // ---- partial Gram row: slot j = sum_{r > t, r owned} P(r,t) P(r,j);  slot w+j = P(t,j) (owner)
+    const int i0 = (int)((t + 1 - rlo) > 0 ? (t + 1 - rlo) : 0);
+    const double* xc = L + (size_t)t * ldl;
+    for (int j = warp; j < w; j += NW) {
+      const double* pc = L + (size_t)j * ldl;
+      double s = 0.0;
+      for (int i = i0 + lane; i < nr; i += 32) s += xc[i] * pc[i];
+      s = warp_sum(s);
+      if (lane == 0) red[(size_t)g * RS + j] = s;
+    }
+    const bool owner = (t >= rlo) && (t < rlo + nr);
+    for (int j = tid; j < w; j += PQ_NT) red[(size_t)g * RS + w + j] = owner ? L[(size_t)j * ldl + (t - rlo)] : 0.0;
+    grid_barrier(a.bar, (unsigned)G, epoch);
+    // ---- totals, fixed order over CTAs (identical in every CTA)
+    if (H > 1) {
+      if (tid < H * RS) {
+        const int s = tid % RS, h = tid / RS;
+        double acc = 0.0;
+        for (int gg = h; gg < G; gg += H) acc += __ldcg(&a.red[(size_t)(t & 1) * G * RS + (size_t)gg * RS + s]);
+        tmp[h * RS + s] = acc;
+      }
+      __syncthreads();
+      for (int s = tid; s < RS; s += PQ_NT) {
+        double acc = 0.0;
+        for (int h = 0; h < H; ++h) acc += tmp[h * RS + s];
+        tot[s] = acc;
+      }
+    } else {
+      for (int s = tid; s < RS; s += PQ_NT) {
+        double acc = 0.0;
+        for (int gg = 0; gg < G; ++gg) acc += __ldcg(&a.red[(size_t)(t & 1) * G * RS + (size_t)gg * RS + s]);
+        tot[s] = acc;
+      }
+    }
+    __syncthreads();
+    // ---- reflector (R1), update vector, T inner products
+    const House h = make_house(tot[w + t], tot[t]);
+    for (int j = tid; j < w; j += PQ_NT) {
+      if (j != t) wv[j] = tot[w + j] + h.scale * tot[j];
+    }
+    if (tid == 0) { hs[0] = h.beta; hs[1] = h.tau; hs[2] = h.scale; }
+    __syncthreads();
+    // ---- apply to owned rows:  v_r = scale * x_r (r > t), v_t = 1;  P(r,j) -= tau * w_j * v_r (j > t)
+    for (int i = tid; i < nr; i += PQ_NT) {
+      const int64_t r = rlo + i;
+      if (r > t) {
+        const double v = h.scale * L[(size_t)t * ldl + i];
+        L[(size_t)t * ldl + i] = v;
+        const double tv = h.tau * v;
+        for (int j = t + 1; j < w; ++j) L[(size_t)j * ldl + i] -= tv * wv[j];
+      } else if (r == t) {
+        L[(size_t)t * ldl + i] = h.beta;
+        for (int j = t + 1; j < w; ++j) L[(size_t)j * ldl + i] -= h.tau * wv[j];
+      }
+    }
+    // ---- T(:, t) (CTA 0): T(t,t) = tau; T(0:t,t) = -tau T(0:t,0:t) (V^T v_t); zeros below
+    if (g == 0) {
+      for (int q = tid; q < w; q += PQ_NT) {
+        double v = 0.0;
+        if (q < t) {
+          double s = 0.0;
+          for (int p = q; p < t; ++p) s += a.T[q + (int64_t)p * a.ldt] * wv[p];
+          v = -h.tau * s;
+        } else if (q == t) {
+          v = h.tau;
+        }
+        a.T[q + (int64_t)t * a.ldt] = v;
+      }
+      if (tid == 0) a.tau[t] = h.tau;
+    }
+    __syncthreads();
+  }
+  // zero the unused columns of T (kk < w)
+  if (g == 0) {
+    for (int idx = tid; idx < (w - a.kk) * w; idx += PQ_NT) {
+      const int q = idx % w, c = a.kk + idx / w;
+      a.T[q + (int64_t)c * a.ldt] = 0.0;
+    }
+  }
+  // ---- write back (R above, V below) and explicit Y = V (unit diagonal, zeros above)
+  if (a.smem_ld > 0) {
+    for (int idx = tid; idx < nr * w; idx += PQ_NT) {
+      const int i = idx % nr, j = idx / nr;
+      a.P[(rlo + i) + (int64_t)j * a.ldp] = L[(size_t)j * ldl + i];
+    }
+  }
+  for (int idx = tid; idx < nr * a.kk; idx += PQ_NT) {
+    const int i = idx % nr, c = idx / nr;
+    const int64_t r = rlo + i;
+    const double v = r > c ? L[(size_t)c * ldl + i] : (r == c ? 1.0 : 0.0);
+    a.Y[r + (int64_t)c * a.ldy] = v;
+  }
+}
+
+static int panel_grid(int64_t m) {
+  int64_t G = (m + 63) / 64;
+  if (G > kNumSMsB200) G = kNumSMsB200;
+  if (G < 1) G = 1;
+  return (int)G;
+}
+
+size_t panel_red_bytes(int w) { return sizeof(double) * 2 * (size_t)kNumSMsB200 * 2 * (size_t)w; }
+
+cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
+                     int64_t ldy, double* red, unsigned* bar, cudaStream_t st) {
+  if (m <= 0 || w <= 0) return cudaSuccess;
+  const int G = panel_grid(m);
+  PanelArgs a;
+  a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);
+  a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.red = red; a.bar = bar;
+  a.rows = (int)((m + G - 1) / G);
+  const size_t scr = sizeof(double) * (size_t)(2 * w + w + PQ_NT + 8);
+  const size_t full = sizeof(double) * (size_t)a.rows * w + scr;
+  const size_t kMaxSmem = 227 * 1024;
+  size_t smem;
+  if (full <= kMaxSmem) {
+    a.smem_ld = a.rows;
+    smem = full;
+  } else {
+    a.smem_ld = 0;
+    smem = scr;
+  }
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(panel_qr_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess) return e;
+  void* args[] = {&a};
+  return cudaLaunchCooperativeKernel((const void*)panel_qr_kernel, dim3(G), dim3(PQ_NT), args, smem, st);
+}
+
+}  // namespace trid
