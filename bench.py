@@ -1,0 +1,353 @@
+"""Benchmark: full two-stage FP64 tridiagonalization (DBBR + GPU bulge chasing) on B200.
+
+Metric (BASELINE.json): FP64 TFLOPs = (4 n^3 / 3) / (t_SBR + t_BC), n = 32768 headline (configs[2],
+b = 64, nb = 16, k = 1024), with the SBR/BC time split.  One "step" = restore A from a resident
+copy (D2D, 8.6 GB, included in the step time) + trid_sytrd_2stage (both stages, Q reflectors stored).
+Inputs live in HBM before the timed region; the 8.6 GB matrix is far larger than the 126 MB L2, so no
+explicit flush is needed between steps.
+
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--n N --b B ...]
+Multi-GPU (torchrun): every rank runs an independent replica (stage 1 sharding is future work, see
+DESIGN.md); time is the max over ranks; value is the whole-job aggregate.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAK_FP64_DMMA_TFLOPS = 37.0     # measured: profiles/r01_fp64_microbench.jsonl (DMMA m16n8k8, 1965 MHz)
+CONFIGS = {
+    "n256": dict(n=256, b=32, nb=8, k=256, seed=1001, desc="n=256 random symmetric FP64, b=32, nb=8"),
+    "n8192": dict(n=8192, b=64, nb=16, k=1024, seed=2001, desc="n=8192 random symmetric FP64, b=64, nb=16"),
+    "n32768": dict(n=32768, b=64, nb=16, k=1024, seed=3001,
+                   desc="n=32768 random symmetric FP64, b=64, nb=16, k=1024 on 1xB200"),
+    "n32768b128": dict(n=32768, b=128, nb=16, k=1024, seed=3001,
+                       desc="n=32768 random symmetric FP64, b=128, nb=16, k=1024 on 1xB200"),
+}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p.get("hbm_gbs", 6549.4)), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+# ------------------------------------------------------------------ algorithmic work (pure counting)
+def dbbr_flops(n, b, k):
+    """Per-class algorithmic flops of the DBBR loop structure (same loop bounds as Alg. 1 / R4)."""
+    fl = {"symm": 0.0, "syr2k": 0.0, "symm_launches": 0, "syr2k_launches": 0}
+    i = 0
+    while i + b + 1 < n:
+        ncols, j, jlast = 0, i, i
+        while j < i + k and j + b + 1 < n:
+            m = n - j - b
+            kk = min(b, m)
+            fl["symm"] += 2.0 * m * m * kk
+            fl["symm_launches"] += 1
+            ncols += kk
+            jlast = j
+            j += b
+        e = jlast + b
+        if e < n:
+            M = n - e
+            fl["syr2k"] += 2.0 * M * (M + 1) * ncols
+            fl["syr2k_launches"] += 1
+        i += k
+    return fl
+
+
+def bc_bytes(n, b):
+    """Algorithmic bytes of the chase: per step read+write of the lower triangle of D_m,
+    read+write of O_m, and the write of v: 8 (2 L(L+1)/2 + 2 L2 L + L)."""
+    import numpy as np
+    if b < 2 or n < 3:
+        return 0.0
+    total = 0.0
+    s = np.arange(0, n - 2, dtype=np.int64)
+    nst = (n - 3 - s) // b + 1
+    mmax = int(nst.max())
+    for m in range(mmax):
+        sel = s[nst > m]
+        r0 = sel + 1 + m * b
+        r1 = np.minimum(sel + (m + 1) * b, n - 1)
+        L = r1 - r0 + 1
+        L2 = np.minimum(r1 + b, n - 1) - r1
+        total += float(np.sum(8.0 * (L * (L + 1) + 2 * L2 * L + L)))
+    return total
+
+
+# ------------------------------------------------------------------ clocks
+class Clocks:
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,power.draw")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.rows = []
+        if self.p is None:
+            return
+        self.p.terminate()
+        out = self.p.communicate()[0]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 7 and f[0].replace(".", "").isdigit():
+                self.rows.append(f)
+
+    def summary(self):
+        if not getattr(self, "rows", None):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows]
+        mx = max(float(r[1]) for r in self.rows)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(sm), "power_w_max": max(float(r[6]) for r in self.rows if r[6] not in ("[N/A]",))}
+
+
+# ------------------------------------------------------------------ CPU oracle timing (test infra)
+def oracle_sample(n_s=1536, b=64, seed=3001):
+    import oracle
+    import trid_gen
+    A = trid_gen.random_symmetric_np(n_s, seed)
+    t0 = time.perf_counter()
+    oracle.tridiagonalize(A, b, None)
+    dt = time.perf_counter() - t0
+    return {"value": round(4.0 * n_s ** 3 / 3.0 / dt / 1e12, 6), "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"oracle O2a naive SBR + O2b naive bulge chase, n={n_s}, b={b}, seed {seed}, "
+                      f"single-threaded C (gcc -O2), {dt:.2f} s; same 4n^3/3 flop convention",
+            "seconds": round(dt, 3)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    cfg = CONFIGS[args.config]
+    n_s = args.ref_n
+    times = []
+    for i in range(args.warmup + args.steps):
+        r = oracle_sample(n_s, cfg["b"], cfg["seed"])
+        if i >= args.warmup:
+            times.append(r["seconds"])
+    t = sum(times)
+    value = 4.0 * n_s ** 3 / 3.0 * args.steps / t / 1e12
+    line = {"impl": "reference", "metric": "FP64 TFLOPs (4n^3/3) full tridiag", "value": round(value, 6),
+            "unit": "TFLOP/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(1e3 * t / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg["desc"], "n": cfg["n"], "b": cfg["b"], "nb": cfg["nb"], "k": cfg["k"],
+                       "seed": cfg["seed"], "sample_n": n_s},
+            "cpu_baseline": {"value": round(value, 6), "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
+                             "sample": f"each step = CPU oracle (naive SBR + naive BC) at n={n_s}, b={cfg['b']}"},
+            "e2e": {"value": round(value, 6), "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="n32768", choices=sorted(CONFIGS))
+    ap.add_argument("--n", type=int, default=0)
+    ap.add_argument("--b", type=int, default=0)
+    ap.add_argument("--k", type=int, default=-1)
+    ap.add_argument("--nb", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=1)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--ref-n", type=int, default=1024)
+    ap.add_argument("--eig-only", action="store_true", help="eigenvalues-only BC (V2 = NULL)")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_wangdzwzljz25_b200 as trid
+    import trid_gen
+
+    ws, rank, local = dist_env()
+    if ws > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl")
+    dev = torch.device("cuda", local if ws > 1 else 0)
+    torch.cuda.set_device(dev)
+    cfg = dict(CONFIGS[args.config])
+    if args.n:
+        cfg["n"] = args.n
+    if args.b:
+        cfg["b"] = args.b
+    if args.k >= 0:
+        cfg["k"] = args.k
+    if args.nb:
+        cfg["nb"] = args.nb
+    n, b, nb, k = cfg["n"], cfg["b"], min(cfg["nb"], cfg["b"]), cfg["k"] or trid.default_k(cfg["n"], cfg["b"])
+    if args.n or args.b or args.k >= 0:
+        cfg["desc"] = f"n={n} random symmetric FP64, b={b}, nb={nb}, k={k}"
+
+    A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
+    A = torch.empty_like(A0)
+    nbytes, v2len, t2len = trid.sytrd_2stage_bufsize(n, b, nb, k)
+    work = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
+    want = not args.eig_only
+    out = (torch.empty(n, dtype=torch.float64, device=dev), torch.empty(max(n - 1, 1), dtype=torch.float64, device=dev),
+           torch.empty(n, dtype=torch.float64, device=dev),
+           torch.empty(max(v2len, 1), dtype=torch.float64, device=dev) if want else None,
+           torch.empty(max(t2len, 1), dtype=torch.float64, device=dev) if want else None)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        A.copy_(A0)
+        trid.sytrd_2stage(A, b, nb=nb, k=k, want_vectors=want, work=work, out=out)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(dev.index) as clk:
+        trid.profile_begin()
+        l0 = trid.kernel_launches()
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if ws > 1:
+            dist.barrier()
+        launches = trid.kernel_launches() - l0
+        stages = trid.profile_end()
+    ms = ev0.elapsed_time(ev1)
+    if ws > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    flop = 4.0 * n ** 3 / 3.0
+    value = ws * flop * args.steps / (ms * 1e-3) / 1e12
+    per = {c: (v[0] / args.steps, v[1] / args.steps) for c, v in stages.items()}
+    t_bc = per["bulge_chase"][0]
+    t_sbr = sum(v[0] for c, v in per.items() if c != "bulge_chase")
+
+    # roofline: the dominant DBBR contraction (largest time share) against the measured FP64 DMMA peak
+    fl = dbbr_flops(n, b, k)
+    cand = {"symm": (fl["symm"], stages["symm"]), "syr2k": (fl["syr2k"], stages["syr2k"])}
+    dom = max(cand, key=lambda c: cand[c][1][0])
+    dflops, (dms, dcalls) = cand[dom]
+    achieved = (dflops / max(dcalls, 1)) / ((dms / max(dcalls, 1)) * 1e-3) / 1e12 if dcalls else 0.0
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get(f"{cfg.get('name', args.config)}:{dom}")
+        except Exception:
+            traffic = None
+    hbm, hbm_kind = peaks()
+    bcb = bc_bytes(n, b)
+    bc_gbs = bcb / (t_bc * 1e-3) / 1e9 if t_bc > 0 else 0.0
+
+    line = {
+        "metric": "FP64 TFLOPs (4n^3/3) full tridiag at n=32768, SBR/BC time split, 1/2/4/8 GPU",
+        "value": round(value, 4), "unit": "TFLOP/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": cfg["desc"], "n": n, "b": b, "nb": nb, "k": k, "seed": cfg["seed"],
+                   "parallelism": "replicas" if ws > 1 else "single-gpu",
+                   "l2": "inputs larger than L2 (n^2*8 B matrix restored from a resident copy each step)",
+                   "vectors": "stored (V1 in A, tau1, V2, tau2)" if want else "eigenvalues-only"},
+        "t_sbr_ms": round(t_sbr, 3), "t_bc_ms": round(t_bc, 3),
+        "split": {"sbr": round(t_sbr / (t_sbr + t_bc), 4) if t_sbr + t_bc > 0 else None,
+                  "bc": round(t_bc / (t_sbr + t_bc), 4) if t_sbr + t_bc > 0 else None},
+        "stages_ms_per_step": {c: round(v[0], 3) for c, v in per.items()},
+        "stage_calls_per_step": {c: v[1] for c, v in per.items()},
+        "roofline": {"bound": "tensor", "kernel": dom, "achieved": round(achieved, 3),
+                     "peak": PEAK_FP64_DMMA_TFLOPS, "unit": "TFLOP/s", "frac": round(achieved / PEAK_FP64_DMMA_TFLOPS, 4),
+                     "traffic": traffic,
+                     "peak_source": "measured FP64 DMMA microbenchmark (profiles/r01_fp64_microbench.jsonl); "
+                                    "MEASURED_PEAKS.json has no FP64 figure"},
+        "roofline_bc": {"bound": "hbm", "kernel": "bulge_chase", "achieved": round(bc_gbs, 1), "peak": hbm,
+                        "unit": "GB/s", "frac": round(bc_gbs / hbm, 4), "traffic": None,
+                        "algorithmic_bytes": bcb, "peak_source": hbm_kind},
+        "sbr_tflops": round(flop / (t_sbr * 1e-3) / 1e12, 3) if t_sbr > 0 else None,
+        "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+    }
+
+    # ---- end to end through the public API with host buffers (pinned H2D of A, D2H of d, e, tau1)
+    if not args.no_e2e and args.e2e_steps > 0:
+        Ah = torch.empty((n, n), dtype=torch.float64, pin_memory=True)
+        Ah.copy_(A0)
+        dh = torch.empty(n, dtype=torch.float64, pin_memory=True)
+        eh = torch.empty(max(n - 1, 1), dtype=torch.float64, pin_memory=True)
+        th = torch.empty(n, dtype=torch.float64, pin_memory=True)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        if ws > 1:
+            dist.barrier()
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            A.copy_(Ah, non_blocking=True)
+            trid.sytrd_2stage(A, b, nb=nb, k=k, want_vectors=want, work=work, out=out)
+            dh.copy_(out[0], non_blocking=True)
+            eh.copy_(out[1], non_blocking=True)
+            th.copy_(out[2], non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        if ws > 1:
+            t = torch.tensor([ems], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        line["e2e"] = {"value": round(ws * flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
+                       "h2d_bytes_per_step": 8 * n * n, "d2h_bytes_per_step": 8 * (n + (n - 1) + n),
+                       "note": "V1/V2 reflectors stay device-resident for the back transformation"}
+        del Ah
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = oracle_sample(1536, b, cfg["seed"])
+        line["cpu_baseline"].pop("seconds", None)
+    if rank == 0:
+        print(json.dumps(line))
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -97,6 +97,18 @@ int trid_sytrd_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, d
                       double* tau1, double* V2, double* tau2, void* dwork, size_t dwork_bytes,
                       cudaStream_t stream);
 
+/* ---- profiling (host-side, optional; used by bench.py) ------------------------------------------
+ * trid_profile_begin(): from now on every hot-path stage launched by the library is bracketed by a pair
+ * of CUDA events recorded on the stream it runs on.  trid_profile_end(ms, calls, nclass) synchronizes
+ * those events and returns, per stage class, the summed elapsed milliseconds and the number of stage
+ * instances; classes: 0 panel QR (a1/a2), 1 W = Y T, 2 SYMM X = A W (a3), 3 Z-builder corrections and
+ * Z = X - 1/2 Y W^T X (a3), 4 next-panel update (a4), 5 deferred syr2k (a5), 6 bulge chase incl. band
+ * pack and d/e extraction (a6/a7).  Either pointer may be NULL.  Process-global state (not reentrant).
+ * trid_kernel_launches(): total number of CUDA kernels this library has launched in the process. */
+int trid_profile_begin(void);
+int trid_profile_end(double* ms, int64_t* calls, int nclass);
+int64_t trid_kernel_launches(void);
+
 /* ---- hot-path building blocks, exposed for unit parity tests ------------ */
 
 /* a1+a2: Householder QR of the m x w panel P (ld ldp), in place: R in the upper triangle, V below it

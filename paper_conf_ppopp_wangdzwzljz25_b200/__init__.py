@@ -59,6 +59,10 @@ def lib():
         L.trid_syr2k_lower.argtypes = [_I64, _I64, _P, _I64, _P, _I64, _P, _I64, _P]
         L.trid_zy_bufsize.argtypes = [_I64, _INT, ctypes.POINTER(_SZ)]
         L.trid_zy.argtypes = [_I64, _INT, _P, _I64, _P, _I64, _P, _I64, _P, _I64, _P, _SZ, _P]
+        L.trid_profile_begin.restype = _INT
+        L.trid_profile_end.restype = _INT
+        L.trid_profile_end.argtypes = [_P, _P, _INT]
+        L.trid_kernel_launches.restype = _I64
         for name in ("trid_sbr_dbbr_bufsize", "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize",
                      "trid_sbr_dbbr", "trid_bulge_chase", "trid_sytrd_2stage", "trid_panel_qr_bufsize",
                      "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize", "trid_zy"):
@@ -70,7 +74,26 @@ def lib():
 EXPORTS = ("trid_status_string", "trid_version", "trid_default_k", "trid_bc_total_steps", "trid_sbr_dbbr_bufsize",
            "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize", "trid_sbr_dbbr", "trid_bulge_chase",
            "trid_sytrd_2stage", "trid_panel_qr_bufsize", "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize",
-           "trid_zy")
+           "trid_zy", "trid_profile_begin", "trid_profile_end", "trid_kernel_launches")
+
+PROF_CLASSES = ("panel_qr", "wy", "symm", "zy", "next_panel", "syr2k", "bulge_chase")
+
+
+def profile_begin():
+    _check(lib().trid_profile_begin(), "trid_profile_begin")
+
+
+def profile_end():
+    """Returns {class: (ms, calls)} for the stages launched since profile_begin()."""
+    import numpy as np
+    ms = np.zeros(len(PROF_CLASSES))
+    calls = np.zeros(len(PROF_CLASSES), dtype=np.int64)
+    _check(lib().trid_profile_end(ms.ctypes.data, calls.ctypes.data, len(PROF_CLASSES)), "trid_profile_end")
+    return {c: (float(ms[i]), int(calls[i])) for i, c in enumerate(PROF_CLASSES)}
+
+
+def kernel_launches() -> int:
+    return int(lib().trid_kernel_launches())
 
 
 def _check(status: int, what: str):

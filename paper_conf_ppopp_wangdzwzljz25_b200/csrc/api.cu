@@ -13,14 +13,42 @@
 #include <stdio.h>
 #include <string.h>
 
+#include <atomic>
+#include <mutex>
+#include <vector>
+
 #include "../../include/trid.h"
 #include "common.cuh"
 #include "gemm.cuh"
 #include "panel.cuh"
+#include "prof.cuh"
 
 using namespace trid;
 
 namespace {
+
+// ---- optional stage profiling (trid_profile_*) and launch counting ------------------------------
+std::atomic<long long> g_launches{0};
+struct ProfState {
+  std::mutex mu;
+  bool on = false;
+  std::vector<cudaEvent_t> pool;
+  size_t used = 0;
+  cudaEvent_t open[PROF_NCLASS] = {};
+  std::vector<cudaEvent_t> begins[PROF_NCLASS], ends[PROF_NCLASS];
+};
+ProfState& prof() {
+  static ProfState p;
+  return p;
+}
+cudaEvent_t prof_event(ProfState& p) {
+  if (p.used == p.pool.size()) {
+    cudaEvent_t ev;
+    if (cudaEventCreate(&ev) != cudaSuccess) return nullptr;
+    p.pool.push_back(ev);
+  }
+  return p.pool[p.used++];
+}
 
 size_t align256(size_t x) { return (x + 255) / 256 * 256; }
 
@@ -88,8 +116,13 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
                      const double* Yp, const double* Yprev, const double* Zprev, int64_t ldyz, int64_t nprev,
                      double* Zp, double* X, int64_t ldx, double* U1, double* U2, int64_t ldu, double* S, int64_t lds,
                      double* part, int64_t part_elems, cudaStream_t st) {
-  cudaError_t e = symm_lower(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
+  cudaError_t e;
+  {
+    ProfScope ps(PROF_SYMM, st);
+    e = symm_lower(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
+  }
   if (e != cudaSuccess) return e;
+  ProfScope ps(PROF_ZY, st);
   if (nprev > 0) {
     // U1 = Z_<^T W, U2 = Y_<^T W   (TN, K = m, deterministic split-K)
     GemmArgs g;
@@ -132,6 +165,26 @@ int check_common(int64_t n, const void* A, int64_t lda, int b) {
 
 }  // namespace
 
+
+namespace trid {
+void count_launches(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+void prof_mark(int cls, bool begin, cudaStream_t st) {
+  ProfState& p = prof();
+  if (!p.on) return;
+  std::lock_guard<std::mutex> lk(p.mu);
+  cudaEvent_t ev = prof_event(p);
+  if (!ev) return;
+  cudaEventRecord(ev, st);
+  if (begin) {
+    p.open[cls] = ev;
+  } else if (p.open[cls]) {
+    p.begins[cls].push_back(p.open[cls]);
+    p.ends[cls].push_back(ev);
+    p.open[cls] = nullptr;
+  }
+}
+}  // namespace trid
+
 extern "C" {
 
 const char* trid_status_string(int status) {
@@ -150,6 +203,41 @@ const char* trid_status_string(int status) {
       return "unknown status";
   }
 }
+
+int trid_profile_begin(void) {
+  ProfState& p = prof();
+  std::lock_guard<std::mutex> lk(p.mu);
+  p.on = true;
+  p.used = 0;
+  for (int c = 0; c < PROF_NCLASS; ++c) {
+    p.open[c] = nullptr;
+    p.begins[c].clear();
+    p.ends[c].clear();
+  }
+  return TRID_SUCCESS;
+}
+
+int trid_profile_end(double* ms, int64_t* calls, int nclass) {
+  ProfState& p = prof();
+  std::lock_guard<std::mutex> lk(p.mu);
+  p.on = false;
+  for (int c = 0; c < nclass; ++c) {
+    if (ms) ms[c] = 0.0;
+    if (calls) calls[c] = 0;
+  }
+  for (int c = 0; c < PROF_NCLASS && c < nclass; ++c) {
+    for (size_t i = 0; i < p.begins[c].size(); ++i) {
+      float t = 0.f;
+      if (cudaEventSynchronize(p.ends[c][i]) != cudaSuccess) return TRID_ERR_CUDA;
+      if (cudaEventElapsedTime(&t, p.begins[c][i], p.ends[c][i]) != cudaSuccess) return TRID_ERR_CUDA;
+      if (ms) ms[c] += t;
+      if (calls) calls[c] += 1;
+    }
+  }
+  return TRID_SUCCESS;
+}
+
+int64_t trid_kernel_launches(void) { return (int64_t)g_launches.load(); }
 
 const char* trid_version(void) { return "trid-b200 0.1 sm_100a"; }
 
@@ -218,12 +306,16 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
       double* Yp = w.Y + o + ncols * ld;
       double* Zp = w.Z + o + ncols * ld;
       // l.5: panel QR (V in place, T, explicit Y_p)
-      TRID_CUDA_TRY(panel_qr(m, b, A + o + j * lda, lda, tau1 + j, w.T, b, Yp, ld, w.red, w.bar, stream));
+      {
+        ProfScope ps(PROF_PANEL, stream);
+        TRID_CUDA_TRY(panel_qr(m, b, A + o + j * lda, lda, tau1 + j, w.T, b, Yp, ld, w.red, w.bar, stream));
+      }
       // W_p = Y_p T
       {
         GemmArgs g;
         g.M = m; g.N = kk; g.K[0] = kk; g.A[0] = Yp; g.lda[0] = ld; g.B[0] = w.T; g.ldb[0] = b;
         g.C = w.W; g.ldc = ld;
+        ProfScope ps(PROF_WY, stream);
         TRID_CUDA_TRY(gemm(g, OP_N, OP_N, TILE_128x64, stream));
       }
       // Z builder against the implicitly updated trailing matrix (R4e)
@@ -241,6 +333,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
         g.alpha = -1.0; g.beta = 1.0;
         g.C = A + o + o * lda; g.ldc = lda; g.Cin = g.C; g.ldcin = lda;
         g.lower = 1; g.diag_off = 0;
+        ProfScope ps(PROF_NEXT, stream);
         TRID_CUDA_TRY(gemm(g, OP_N, OP_T, TILE_128x64, stream));
       }
     }
@@ -253,6 +346,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
       g.alpha = -1.0; g.beta = 1.0;
       g.C = A + e + e * lda; g.ldc = lda; g.Cin = g.C; g.ldcin = lda;
       g.lower = 1; g.tri = 1;
+      ProfScope ps(PROF_SYR2K, stream);
       TRID_CUDA_TRY(gemm(g, OP_N, OP_T, TILE_128x128, stream));
     }
   }
@@ -272,6 +366,7 @@ int trid_bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, 
   trid_bulge_chase_bufsize(n, b, &need, nullptr, nullptr);
   if (!dwork) return -9;
   if (dwork_bytes < need) return TRID_ERR_WORKSPACE;
+  ProfScope ps(PROF_BC, stream);
   TRID_CUDA_TRY(bulge_chase(n, b, A, lda, d, e, V2, tau2, dwork, stream));
   return TRID_SUCCESS;
 }

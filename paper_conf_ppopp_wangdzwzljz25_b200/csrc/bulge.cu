@@ -16,6 +16,7 @@
 //     scheduling.
 #include "common.cuh"
 #include "panel.cuh"
+#include "prof.cuh"
 
 namespace trid {
 
@@ -330,6 +331,7 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     int blocks = (int)((total + 255) / 256);
     if (blocks > 8 * kNumSMsB200 * 4) blocks = 8 * kNumSMsB200 * 4;
     band_pack_kernel<<<blocks, 256, 0, st>>>(n, beff, ldab, A, lda, band);
+    count_launches(1);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess) return err;
   }
@@ -357,6 +359,7 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     if (grid > n - 2) grid = n - 2;
     if (use_sm) bc_kernel<true><<<(unsigned)grid, BC_NT, smem, st>>>(a);
     else bc_kernel<false><<<(unsigned)grid, BC_NT, smem, st>>>(a);
+    count_launches(1);
     err = cudaGetLastError();
     if (err != cudaSuccess) return err;
   }
@@ -364,6 +367,7 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     int blocks = (int)((n + 255) / 256);
     if (blocks > 4 * kNumSMsB200) blocks = 4 * kNumSMsB200;
     band_extract_kernel<<<blocks, 256, 0, st>>>(n, ldab, band, d, e);
+    count_launches(1);
     return cudaGetLastError();
   }
 }

@@ -12,6 +12,7 @@
 // doubles for m-inner tiles, 4 mod 16 for k-inner tiles).
 #include "common.cuh"
 #include "gemm.cuh"
+#include "prof.cuh"
 
 namespace trid {
 
@@ -230,6 +231,7 @@ static cudaError_t launch_tile(const GemmArgs& a, cudaStream_t st) {
     grid = dim3((unsigned)tm, (unsigned)tn, (unsigned)a.splits);
   }
   gemm_kernel<BM, BN, WGM, WGN, OPA, OPB><<<grid, NT, smem, st>>>(a);
+  count_launches(1);
   return cudaGetLastError();
 }
 
@@ -249,6 +251,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
     GemmArgs r = a;
     r.splits = 0;
     reduce_partials_kernel<<<592, 256, 0, st>>>(r);
+    count_launches(1);
     return cudaGetLastError();
   }
   if (a.splits < 1) a.splits = 1;
@@ -262,6 +265,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
   int blocks = (int)((total + 255) / 256);
   if (blocks > 4 * kNumSMsB200 * 4) blocks = 4 * kNumSMsB200 * 4;
   reduce_partials_kernel<<<blocks, 256, 0, st>>>(a);
+  count_launches(1);
   return cudaGetLastError();
 }
 
@@ -378,6 +382,7 @@ cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const
   a.part_stride = m * w;
   dim3 grid((unsigned)((m + SY_BM - 1) / SY_BM), (unsigned)((w + SY_BN - 1) / SY_BN), (unsigned)a.nchunk);
   symm_kernel<<<grid, SY_WGM * SY_WGN * 32, smem, st>>>(a);
+  count_launches(1);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess || a.nchunk == 1) return e;
   GemmArgs r;
@@ -387,6 +392,7 @@ cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const
   int blocks = (int)((total + 255) / 256);
   if (blocks > 16 * kNumSMsB200) blocks = 16 * kNumSMsB200;
   reduce_partials_kernel<<<blocks, 256, 0, st>>>(r);
+  count_launches(1);
   return cudaGetLastError();
 }
 

@@ -11,6 +11,7 @@
 // CTA order, so every CTA (and every run) sees bitwise-identical values.
 #include "common.cuh"
 #include "panel.cuh"
+#include "prof.cuh"
 
 namespace trid {
 
@@ -198,6 +199,7 @@ cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, doub
   cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), st);
   if (e != cudaSuccess) return e;
   void* args[] = {&a};
+  count_launches(1);
   return cudaLaunchCooperativeKernel((const void*)panel_qr_kernel, dim3(G), dim3(PQ_NT), args, smem, st);
 }
 
