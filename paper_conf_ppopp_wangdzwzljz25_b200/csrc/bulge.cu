@@ -18,10 +18,11 @@
 #include "panel.cuh"
 #include "prof.cuh"
 
+#include <stdlib.h>
+
 namespace trid {
 
 constexpr int BC_NT = 256;
-constexpr int BC_SMEM_MAXB = 64;
 
 struct BcArgs {
   int64_t n;
@@ -30,9 +31,26 @@ struct BcArgs {
   double* band;
   double* V2;
   double* tau2;
-  int* prog;
+  int* prog;        // prog[s] = m+1: column 0 of step (s, m) published
+  int* prog_full;   // prog_full[s] = m+1: all columns of step (s, m) stored
   unsigned* ticket;
+  long long* trace;     // debug (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1
+  int64_t trace_sweep;
 };
+
+__device__ __forceinline__ long long gtimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define BC_TRACE(k)                                                                             \
+  do {                                                                                          \
+    if (a.trace && tid == 0 && (s == a.trace_sweep || s == a.trace_sweep + 1) && m < 1024) {   \
+      a.trace[((s - a.trace_sweep) * 1024 + m) * 16 + (k)] = gtimer();                          \
+      if ((k) == 2 || (k) == 3) a.trace[((s - a.trace_sweep) * 1024 + m) * 16 + 8 + (k)] = clock64(); \
+      if ((k) >= 12) a.trace[((s - a.trace_sweep) * 1024 + m) * 16 + (k)] = clock64();         \
+    }                                                                                           \
+  } while (0)
 
 __host__ __device__ inline int64_t bc_steps(int64_t n, int b, int64_t s) {
   if (b < 2 || s < 0 || s > n - 3) return 0;
@@ -71,91 +89,56 @@ __global__ void band_extract_kernel(int64_t n, int ldab, const double* band, dou
   }
 }
 
-// ---- block-level helpers (deterministic fixed-order reductions) ---------------------------------
-// out[i] = sum_j M(i, j) x[j], i < R, j < C, via accessor get(i, j).  scratch >= BC_NT doubles.
-template <class Get>
-__device__ __forceinline__ void block_matvec(Get get, int R, int C, const double* x, double* out, double* scratch) {
-  const int tid = threadIdx.x;
-  const int q = R > 0 ? BC_NT / R : 1;
-  if (R > 0 && tid < q * R) {
-    const int i = tid % R, c = tid / R;
-    double s = 0.0;
-    for (int j = c; j < C; j += q) s += get(i, j) * x[j];
-    scratch[c * R + i] = s;
-  }
-  __syncthreads();
-  if (tid < R) {
-    double s = 0.0;
-    for (int c = 0; c < q; ++c) s += scratch[c * R + tid];
-    out[tid] = s;
-  }
-  __syncthreads();
-}
-
-// Sum of x[lo..hi) computed by warp 0 in a fixed order; result broadcast through *res.
-__device__ __forceinline__ void warp0_sumsq_tail(const double* x, int lo, int hi, double* res) {
-  if (threadIdx.x < 32) {
-    double s = 0.0;
-    for (int i = lo + (int)threadIdx.x; i < hi; i += 32) s += x[i] * x[i];
-    s = warp_sum(s);
-    if (threadIdx.x == 0) *res = s;
-  }
-}
-__device__ __forceinline__ void warp0_dot(const double* x, const double* y, int nn, double* res) {
-  if (threadIdx.x < 32) {
-    double s = 0.0;
-    for (int i = threadIdx.x; i < nn; i += 32) s += x[i] * y[i];
-    s = warp_sum(s);
-    if (threadIdx.x == 0) *res = s;
-  }
-}
-
-// Window accessors.  SMEM: dense symmetric D (LD = b+1) and dense O in shared memory.
-// Global: directly on the compact band, D lower-only (symmetric reads mirror), O below it.
+// ---- the chase ---------------------------------------------------------------------------------
+// Window of step (s, m): compact columns r0 .. r0+L-1 (each ldab doubles: rows c .. c+ldab-1).
+//   D = B_d  (L x L symmetric):  D(i,j) = C[j*ldab + i-j] (i >= j)
+//   O = B_od (L2 x L, the block below, where the bulge appears):  O(i,j) = C[j*ldab + L+i-j]
 template <bool SM>
-struct Win {
-  double* Dm;   // SM: dense L x L (ld LD);  global: band + r0*ldab
-  double* Om;   // SM: dense L2 x L (ld LD)
-  int LD;       // SM: leading dimension; global: ldab
-  int L;
-  __device__ __forceinline__ double D(int i, int j) const {
-    if (SM) return Dm[j * LD + i];
-    return i >= j ? __ldcg(Dm + (int64_t)j * LD + (i - j)) : __ldcg(Dm + (int64_t)i * LD + (j - i));
+struct CWin {
+  double* C;
+  int ldab, L;
+  __device__ __forceinline__ double ld(int off) const {
+    if constexpr (SM) return C[off];
+    else return __ldcg(C + off);
   }
-  __device__ __forceinline__ void Dsub(int i, int j, double v) const {  // i >= j (and mirror in SM)
-    if (SM) {
-      Dm[j * LD + i] -= v;
-      if (i != j) Dm[i * LD + j] -= v;
-    } else {
-      double* p = Dm + (int64_t)j * LD + (i - j);
-      __stcg(p, __ldcg(p) - v);
-    }
+  __device__ __forceinline__ void st(int off, double v) const {
+    if constexpr (SM) C[off] = v;
+    else __stcg(C + off, v);
   }
-  __device__ __forceinline__ double* Optr(int i, int j) const {
-    if (SM) return Om + j * LD + i;
-    return Dm + (int64_t)j * LD + (L + i - j);
-  }
-  __device__ __forceinline__ double O(int i, int j) const { return SM ? *Optr(i, j) : __ldcg(Optr(i, j)); }
-  __device__ __forceinline__ void Oset(int i, int j, double v) const {
-    if (SM) *Optr(i, j) = v; else __stcg(Optr(i, j), v);
-  }
+  __device__ __forceinline__ int dof(int i, int j) const { return i >= j ? j * ldab + (i - j) : i * ldab + (j - i); }
+  __device__ __forceinline__ int oof(int i, int j) const { return j * ldab + L + i - j; }
 };
 
+// Window load: 16-byte cp.async (all copies of a thread in flight at once, no registers held).
+__device__ __forceinline__ void load_span(double* dst, const double* src, int count) {
+  const int n2 = count >> 1;
+  for (int i = threadIdx.x; i < n2; i += BC_NT) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst + 2 * i);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src + 2 * i) : "memory");
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+// Window store: 16-byte st.global.cg (fire and forget).
+__device__ __forceinline__ void store_span(double* dst, const double* src, int count) {
+  const int n2 = count >> 1;
+  const double2* s2 = reinterpret_cast<const double2*>(src);
+  double2* d2 = reinterpret_cast<double2*>(dst);
+  for (int i = threadIdx.x; i < n2; i += BC_NT) __stcg(d2 + i, s2[i]);
+}
+
 template <bool SM>
-__global__ void __launch_bounds__(BC_NT) bc_kernel(BcArgs a) {
+__global__ void __launch_bounds__(BC_NT, 3) bc_kernel(BcArgs a) {
   extern __shared__ __align__(16) double sm[];
-  const int b = a.b, tid = threadIdx.x;
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31;
   const int64_t n = a.n;
-  const int LD = b + 1;
-  double* Dm = sm;
-  double* Om = SM ? sm + LD * b : sm;
-  double* vec = SM ? Om + LD * b : sm;
-  double* v = vec;            // b   current reflector
-  double* vn = v + b;         // b   next reflector
-  double* p = vn + b;         // b   D v / O v / v^T O
-  double* wv = p + b;         // b
-  double* scratch = wv + b;   // BC_NT
-  double* sc = scratch + BC_NT;  // scalars: [0] sum, [1] tau, [2] tau_next, [3] beta
+  double* win = sm;
+  double* vec = SM ? sm + (size_t)b * ldab : sm;
+  double* v = vec;               // b   reflector of this step
+  double* vn = v + b;            // b   reflector of the next step
+  double* p = vn + b;            // b   tau * D v
+  double* y = p + b;             // b   O v
+  double* z = y + b;             // b   vn^T O
+  double* scratch = z + b;       // 2 * BC_NT partial sums
   __shared__ int64_t s_sweep;
 
   for (;;) {
@@ -167,6 +150,7 @@ __global__ void __launch_bounds__(BC_NT) bc_kernel(BcArgs a) {
     const int64_t nst = bc_steps(n, b, s);
     const int64_t off = bc_offset(n, b, s);
     const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+    double tau = 0.0;
     for (int64_t m = 0; m < nst; ++m) {
       const int64_t r0 = s + 1 + m * b;
       const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
@@ -177,144 +161,416 @@ __global__ void __launch_bounds__(BC_NT) bc_kernel(BcArgs a) {
       if (s > 0) {
         if (tid == 0) {
           const int need = (int)((m + 2 < nprev) ? m + 2 : nprev);
-          while (ld_acquire_s32(a.prog + (s - 1)) < need) {
-          }
+          wait_geq(a.prog + (s - 1), need);
         }
         __syncthreads();
       }
-      // ---- step 0: reflector from column s (rows s+1 .. s+L), compact column s offsets 1..L
+      // ---- step 0: the reflector annihilating column s below its first subdiagonal
       if (m == 0) {
-        double* col = a.band + s * a.ldab;
-        for (int i = tid; i < L; i += BC_NT) v[i] = __ldcg(col + 1 + i);
-        __syncthreads();
-        warp0_sumsq_tail(v, 1, L, sc);
-        __syncthreads();
-        const House h = make_house(v[0], sc[0]);
-        __syncthreads();
+        double* col = a.band + s * a.ldab + 1;
+        double sig = 0.0;
+        for (int i = 1 + lane; i < L; i += 32) {
+          const double x = __ldcg(col + i);
+          sig += x * x;
+        }
+        sig = warp_sum(sig);  // every warp computes the same value in the same order
+        const House h = make_house(__ldcg(col), sig);
+        __syncthreads();      // all reads of column s done before it is overwritten
         for (int i = tid; i < L; i += BC_NT) {
-          const double x = v[i];
-          v[i] = i == 0 ? 1.0 : h.scale * x;
-          __stcg(col + 1 + i, i == 0 ? h.beta : 0.0);
+          v[i] = i == 0 ? 1.0 : h.scale * __ldcg(col + i);
         }
-        if (tid == 0) sc[1] = h.tau;
         __syncthreads();
+        for (int i = tid; i < L; i += BC_NT) __stcg(col + i, i == 0 ? h.beta : 0.0);
+        tau = h.tau;
       }
-      const double tau = sc[1];
-      Win<SM> W;
+      CWin<SM> W;
+      W.ldab = ldab;
       W.L = L;
-      if (SM) {
-        W.Dm = Dm; W.Om = Om; W.LD = LD;
-        const double* src = a.band + r0 * a.ldab;
-        const int span = L * a.ldab;
-        for (int idx = tid; idx < span; idx += BC_NT) {
-          const int j = idx / a.ldab, o = idx - j * a.ldab;
-          const double x = __ldcg(src + idx);
-          if (j + o < L) {
-            Dm[j * LD + (j + o)] = x;
-            Dm[(j + o) * LD + j] = x;
-          } else if (j + o - L < L2) {
-            Om[j * LD + (j + o - L)] = x;
-          }
-        }
+      if constexpr (SM) {
+        W.C = win;
+        load_span(win, a.band + r0 * ldab, L * ldab);
       } else {
-        W.Dm = a.band + r0 * a.ldab; W.Om = nullptr; W.LD = a.ldab;
+        W.C = a.band + r0 * ldab;
       }
       __syncthreads();
+      // ---- two-sided on B_d and right-apply to B_od (the bulge), from ONE pass of matvecs
       if (tau != 0.0) {
-        // ---- two-sided on B_d:  p = tau D v;  wv = p - 1/2 tau (p^T v) v;  D -= v wv^T + wv v^T
-        block_matvec([&](int i, int j) { return W.D(i, j); }, L, L, v, p, scratch);
-        for (int i = tid; i < L; i += BC_NT) p[i] *= tau;
-        __syncthreads();
-        warp0_dot(p, v, L, sc);   // pv = p^T v with p = tau D v
-        __syncthreads();
-        const double pv = sc[0];
-        for (int i = tid; i < L; i += BC_NT) wv[i] = p[i] - 0.5 * tau * pv * v[i];
-        __syncthreads();
-        for (int idx = tid; idx < L * L; idx += BC_NT) {
-          const int i = idx % L, j = idx / L;
-          if (i >= j) W.Dsub(i, j, v[i] * wv[j] + wv[i] * v[j]);
-        }
-        __syncthreads();
-        // ---- right-apply to B_od (creates the bulge):  O -= tau (O v) v^T
-        if (L2 > 0) {
-          block_matvec([&](int i, int j) { return W.O(i, j); }, L2, L, v, p, scratch);
-          for (int idx = tid; idx < L2 * L; idx += BC_NT) {
-            const int i = idx % L2, j = idx / L2;
-            W.Oset(i, j, W.O(i, j) - tau * p[i] * v[j]);
+        const int R = L + L2;
+        const int q = R < BC_NT ? BC_NT / R : 1;
+        for (int task = tid; task < R * q; task += BC_NT) {
+          const int i = task % R, c = task / R;
+          double acc = 0.0;
+          if (i < L) {
+            for (int j = c; j < L; j += q) acc += W.ld(W.dof(i, j)) * v[j];
+          } else {
+            for (int j = c; j < L; j += q) acc += W.ld(W.oof(i - L, j)) * v[j];
           }
-          __syncthreads();
+          scratch[c * R + i] = acc;
         }
+        __syncthreads();
+        for (int i = tid; i < R; i += BC_NT) {
+          double acc = 0.0;
+          for (int c = 0; c < q; ++c) acc += scratch[c * R + i];
+          if (i < L) p[i] = tau * acc;
+          else y[i - L] = acc;
+        }
+        __syncthreads();
+        double pv = 0.0;  // p^T v, per warp (identical in every warp)
+        for (int i = lane; i < L; i += 32) pv += p[i] * v[i];
+        pv = warp_sum(pv);
+        const double hp = 0.5 * tau * pv;
+        // D -= v w^T + w v^T (lower), w = p - 1/2 tau (p^T v) v;   O -= tau (O v) v^T
+        const int nd = L * L, no = L2 * L;
+        for (int idx = tid; idx < nd + no; idx += BC_NT) {
+          if (idx < nd) {
+            const int i = idx % L, j = idx / L;
+            if (i >= j) {
+              const double wi = p[i] - hp * v[i], wj = p[j] - hp * v[j];
+              const int o = j * ldab + (i - j);
+              W.st(o, W.ld(o) - (v[i] * wj + wi * v[j]));
+            }
+          } else {
+            const int k = idx - nd, i = k % L2, j = k / L2;
+            const int o = W.oof(i, j);
+            W.st(o, W.ld(o) - tau * y[i] * v[j]);
+          }
+        }
+        __syncthreads();
       }
-      // ---- next reflector from the bulge's first column, left-apply to O(:, 1:)
+      // ---- next reflector from the bulge's first column; left-apply to O(:, 1:)
+      double tau_next = 0.0;
       if (L2 > 0) {
-        for (int i = tid; i < L2; i += BC_NT) vn[i] = W.O(i, 0);
-        __syncthreads();
-        warp0_sumsq_tail(vn, 1, L2, sc);
-        __syncthreads();
-        const House h = make_house(vn[0], sc[0]);
-        __syncthreads();
-        for (int i = tid; i < L2; i += BC_NT) {
-          vn[i] = i == 0 ? 1.0 : h.scale * vn[i];
-          W.Oset(i, 0, i == 0 ? h.beta : 0.0);
+        double sig = 0.0;
+        for (int i = 1 + lane; i < L2; i += 32) {
+          const double x = W.ld(W.oof(i, 0));
+          sig += x * x;
         }
-        if (tid == 0) sc[2] = h.tau;
-        __syncthreads();
+        sig = warp_sum(sig);
+        const House h = make_house(W.ld(W.oof(0, 0)), sig);
+        tau_next = h.tau;
         if (h.tau != 0.0 && L > 1) {
-          // z_j = vn^T O(:, j), j = 1..L-1 (stored in p[j])
           const int C = L - 1;
-          const int q = BC_NT / C;
-          if (tid < q * C) {
-            const int j = 1 + tid % C, c = tid / C;
+          const int q = C < BC_NT ? BC_NT / C : 1;
+          for (int task = tid; task < C * q; task += BC_NT) {
+            const int j = 1 + task % C, c = task / C;
             double acc = 0.0;
-            for (int i = c; i < L2; i += q) acc += vn[i] * W.O(i, j);
+            for (int i = c; i < L2; i += q) {
+              const double vi = i == 0 ? 1.0 : h.scale * W.ld(W.oof(i, 0));
+              acc += vi * W.ld(W.oof(i, j));
+            }
             scratch[c * C + (j - 1)] = acc;
           }
           __syncthreads();
-          if (tid < C) {
+          for (int j = tid; j < C; j += BC_NT) {
             double acc = 0.0;
-            for (int c = 0; c < q; ++c) acc += scratch[c * C + tid];
-            p[tid + 1] = acc;
+            for (int c = 0; c < q; ++c) acc += scratch[c * C + j];
+            z[j + 1] = acc;
           }
           __syncthreads();
           for (int idx = tid; idx < L2 * C; idx += BC_NT) {
             const int i = idx % L2, j = 1 + idx / L2;
-            W.Oset(i, j, W.O(i, j) - h.tau * vn[i] * p[j]);
+            const double vi = i == 0 ? 1.0 : h.scale * W.ld(W.oof(i, 0));
+            const int o = W.oof(i, j);
+            W.st(o, W.ld(o) - h.tau * vi * z[j]);
           }
         }
-        __syncthreads();
-      }
-      // ---- write back the window, the reflector of this step, then publish progress
-      if (SM) {
-        double* dst = a.band + r0 * a.ldab;
-        const int span = L * a.ldab;
-        for (int idx = tid; idx < span; idx += BC_NT) {
-          const int j = idx / a.ldab, o = idx - j * a.ldab;
-          if (j + o < L) __stcg(dst + idx, Dm[j * LD + (j + o)]);
-          else if (j + o - L < L2) __stcg(dst + idx, Om[j * LD + (j + o - L)]);
+        __syncthreads();  // every read of O(:, 0) is done
+        for (int i = tid; i < L2; i += BC_NT) {
+          const int o = W.oof(i, 0);
+          vn[i] = i == 0 ? 1.0 : h.scale * W.ld(o);
+          W.st(o, i == 0 ? h.beta : 0.0);
         }
       }
+      __syncthreads();
+      // ---- write back, store the reflector of this step, publish progress
+      if constexpr (SM) store_span(a.band + r0 * ldab, win, L * ldab);
       if (a.V2) {
         double* vd = a.V2 + (off + m) * a.vs;
         for (int i = tid; i < a.vs; i += BC_NT) vd[i] = i < L ? v[i] : 0.0;
         if (tid == 0) a.tau2[off + m] = tau;
       }
       __syncthreads();
+      if (tid == 0) st_release_s32(a.prog + s, (int)(m + 1));  // cumulative over the CTA's stores (bar.sync above)
+      for (int i = tid; i < L2; i += BC_NT) v[i] = vn[i];
+      tau = tau_next;
+      __syncthreads();
+    }
+  }
+}
+
+// ---- fast path for b <= B (B = 32 or 64) -----------------------------------------------------------
+// Step (s, m) owns the compact columns R_m = [r0, r0+L).  Its window M = [D; O] ((L+L2) x L) is loaded
+// into shared memory by the bulk-copy engine and held in registers, one row slice per thread; a warp
+// covers 32 consecutive rows of one column group, so every compact-window access is bank-conflict free.
+// Dependencies (R9, refined by column ownership):
+//   * column 0 of step (s, m) is final as soon as the next reflector has been generated; it is the
+//     only column sweep s+1 needs to START its step m-1.  It is published first (1 KB bulk store,
+//     then prog[s] = m+1).
+//   * columns 1..L-1 are stored asynchronously afterwards and signalled with prog_full[s] = m+1 at the
+//     start of the next step; sweep s+1 only needs them for its prefetch of step m.
+//   * the window of step m+1 except its last column is prefetched while step m computes; after
+//     prog[s-1] >= m+2 only that last column (sweep s-1's published column 0) is loaded.
+// All sums are in a fixed order: results are bitwise reproducible and identical to sweep-major order.
+template <int B, int NTH>
+__global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
+  constexpr int TPR = NTH / (2 * B);   // column groups
+  constexpr int CPT = B / TPR;         // columns per thread
+  constexpr int RW = (2 * B) / 32;     // warps per column group
+  constexpr int NW = NTH / 32;
+  constexpr int CPW = B / NW;          // columns per warp in the z pass
+  static_assert(CPW == 4, "z-pass butterfly assumes 4 columns per warp");
+  extern __shared__ __align__(16) double sm[];
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
+  const int lda1 = ldab - 1;
+  const int64_t n = a.n;
+  const int wsz = B * ldab;
+  double* vb = sm + 2 * wsz;                 // 2 x B   (v / vn)
+  double* pyv = vb + 2 * B;                  // 2B      tau*D v | O v
+  double* zv = pyv + 2 * B;                  // B
+  double* part = zv + B;                     // TPR x 2B matvec partials
+  __shared__ int64_t s_sweep;
+  __shared__ __align__(8) uint64_t mbar[2];   // window buffers: 2 arrivals + tx bytes per use
+  if (tid == 0) {
+    mbar_init(&mbar[0], 2);
+    mbar_init(&mbar[1], 2);
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  unsigned phase[2] = {0u, 0u};
+  int cur = 0;
+
+  for (;;) {
+    if (tid == 0) s_sweep = (int64_t)atomicAdd(a.ticket, 1u);
+    __syncthreads();
+    const int64_t s = s_sweep;
+    __syncthreads();
+    if (s > n - 3) return;
+    const int64_t nst = bc_steps(n, b, s);
+    const int64_t off = bc_offset(n, b, s);
+    const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+    double tau = 0.0;
+    for (int64_t m = 0; m < nst; ++m) {
+      const int64_t r0 = s + 1 + m * b;
+      const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+      const int L = (int)(r1 - r0 + 1);
+      const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
+      const int L2 = (int)(r2 - r1);
+      double* win = sm + cur * wsz;
+      double* v = vb + (m & 1) * B;
+      double* vn = vb + ((m & 1) ^ 1) * B;
+      BC_TRACE(0);
       if (tid == 0) {
-        __threadfence();
+        if (m > 0) {  // step m-1's columns 1..L-1 are in L2 -> signal the prefetch of sweep s+1
+          bulk_wait_all();
+          fence_proxy_async_global();
+          st_release_s32(a.prog_full + s, (int)m);
+        }
+        if (s > 0) {
+          if (m == 0) wait_geq(a.prog_full + (s - 1), 1);
+          wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        }
+      }
+      __syncthreads();
+      BC_TRACE(1);
+      const double* gsrc = a.band + r0 * ldab;
+      if (m == 0) {
+        double* col = a.band + s * ldab + 1;
+        double sig = 0.0;
+        for (int i = 1 + lane; i < L; i += 32) {
+          const double x = __ldcg(col + i);
+          sig += x * x;
+        }
+        sig = warp_sum(sig);
+        const House hh = make_house(__ldcg(col), sig);
+        if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * __ldcg(col + tid) : 0.0);
+        __syncthreads();
+        if (tid < L) __stcg(col + tid, tid == 0 ? hh.beta : 0.0);
+        tau = hh.tau;
+        if (tid == 0) {
+          fence_proxy_async_smem();
+          fence_proxy_async_global();
+          mbar_arrive_expect_tx(&mbar[cur], (unsigned)(L * ldab * 8));
+          bulk_g2s(win, gsrc, (unsigned)(L * ldab * 8), &mbar[cur]);
+          mbar_arrive(&mbar[cur]);
+        }
+      } else if (tid == 0) {
+        fence_proxy_async_global();
+        mbar_arrive_expect_tx(&mbar[cur], (unsigned)(ldab * 8));
+        bulk_g2s(win + (L - 1) * ldab, gsrc + (L - 1) * ldab, (unsigned)(ldab * 8), &mbar[cur]);
+      }
+      mbar_wait(&mbar[cur], phase[cur]);
+      phase[cur] ^= 1u;
+      BC_TRACE(2);
+      const bool active = r < L + L2;
+      const bool isO = r >= L && active;
+      const int lo_base = j0 * lda1 + r;   // j <= r: j*(ldab-1) + r
+      const int hi_base = r * lda1 + j0;   // j >  r: r*(ldab-1) + j
+      double e[CPT];
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        e[jj] = win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
+      }
+      if (tau != 0.0) {
+        double acc0 = 0.0, acc1 = 0.0;
+#pragma unroll
+        for (int jj = 0; jj < CPT; jj += 2) {
+          acc0 = fma(e[jj], v[j0 + jj], acc0);
+          acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
+        }
+        part[hg * 2 * B + r] = acc0 + acc1;
+        __syncthreads();
+        if (tid < 2 * B) {
+          double acc = 0.0;
+#pragma unroll
+          for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + tid];
+          pyv[tid] = (tid >= L) ? acc : tau * acc;
+        }
+        __syncthreads();
+        BC_TRACE(3);
+        double pv = 0.0;
+        for (int i = lane; i < L; i += 32) pv += pyv[i] * v[i];
+        pv = warp_sum(pv);
+        const double hp = 0.5 * tau * pv;
+        if (isO) {
+          const double ty = tau * pyv[r];
+#pragma unroll
+          for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
+        } else {
+          const double vr = r < L ? v[r] : 0.0;
+          const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
+#pragma unroll
+          for (int jj = 0; jj < CPT; ++jj) {
+            const double vj = v[j0 + jj];
+            const double wj = fma(-hp, vj, pyv[j0 + jj]);
+            e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
+          }
+        }
+      }
+      // write back the lower part of D and all of O
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
+      }
+      __syncthreads();
+      BC_TRACE(4);
+      // ---- next reflector from x = O(:, 0) (raw, at win[L + i]); every warp derives it identically
+      double tau_next = 0.0;
+      House h2;
+      h2.beta = 0.0;
+      h2.tau = 0.0;
+      h2.scale = 0.0;
+      if (L2 > 0) {
+        double sg = 0.0;
+        for (int i = 1 + lane; i < L2; i += 32) sg = fma(win[L + i], win[L + i], sg);
+        sg = warp_sum(sg);
+        h2 = make_house(win[L], sg);
+        tau_next = h2.tau;
+        if (tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : h2.scale * win[L + tid]) : 0.0;
+      }
+      // ---- z_j = vn^T O(:, j) = O(0, j) + scale * sum_{i>=1} x_i O(i, j), j >= 1 (reads raw column 0)
+      if (L2 > 0 && h2.tau != 0.0 && L > 1) {
+        const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
+        const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
+        double c[CPW];
+#pragma unroll
+        for (int q = 0; q < CPW; ++q) {
+          const int j = warp + q * NW;
+          double acc = 0.0;
+          if (j >= 1 && j < L) {
+            const int ob = j * lda1 + L;
+            if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
+            if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
+          }
+          c[q] = acc;
+        }
+        // transposed butterfly: 4 columns over 32 lanes in 6 shuffles, fixed partners
+        {
+          const bool up16 = (lane & 16) != 0;
+          const double s0 = up16 ? c[0] : c[2], s1 = up16 ? c[1] : c[3];
+          const double k0 = up16 ? c[2] : c[0], k1 = up16 ? c[3] : c[1];
+          double d0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 16);
+          double d1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 16);
+          const bool up8 = (lane & 8) != 0;
+          const double s2 = up8 ? d0 : d1, k2 = up8 ? d1 : d0;
+          double f = k2 + __shfl_xor_sync(0xffffffffu, s2, 8);
+          f += __shfl_xor_sync(0xffffffffu, f, 4);
+          f += __shfl_xor_sync(0xffffffffu, f, 2);
+          f += __shfl_xor_sync(0xffffffffu, f, 1);
+          if ((lane & 7) == 0) {
+            const int q = (up16 ? 2 : 0) + (up8 ? 1 : 0);
+            const int j = warp + q * NW;
+            if (j >= 1 && j < L) zv[j] = fma(h2.scale, f, win[j * lda1 + L]);
+          }
+        }
+      }
+      __syncthreads();   // all reads of the raw O(:, 0) done; zv ready
+      BC_TRACE(5);
+      // ---- finalize and publish column 0 (D(:,0) and the annihilated bulge column)
+      if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
+      __syncthreads();
+      if (tid == 0) {
+        fence_proxy_async_smem();
+        bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
+        bulk_commit();
+        bulk_wait_all();
+        fence_proxy_async_global();
         st_release_s32(a.prog + s, (int)(m + 1));
       }
-      // hand the next reflector to step m+1
-      for (int i = tid; i < L2; i += BC_NT) v[i] = vn[i];
-      if (tid == 0) sc[1] = sc[2];
+      BC_TRACE(6);
+      // ---- left-apply the next reflector to O(:, 1:)
+      if (L2 > 0 && h2.tau != 0.0 && isO) {
+        const double vni = vn[r - L];
+        const double tv = h2.tau * vni;
+#pragma unroll
+        for (int jj = 0; jj < CPT; ++jj) {
+          const int j = j0 + jj;
+          if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
+        }
+      }
       __syncthreads();
+      BC_TRACE(7);
+      if (tid == 0) {
+        if (L > 1) {
+          fence_proxy_async_smem();
+          bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
+          bulk_commit();
+        }
+        // prefetch the next step's window (all but its last column) into the other buffer
+        if (m + 1 < nst) {
+          if (s > 0) wait_geq(a.prog_full + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+          const int64_t q0 = r1 + 1;
+          const int64_t q1 = (r1 + b < n - 1) ? r1 + b : n - 1;
+          const unsigned bytes = (unsigned)((q1 - q0) * ldab * 8);   // (Lnext - 1) columns
+          fence_proxy_async_global();
+          mbar_arrive_expect_tx(&mbar[cur ^ 1], bytes);
+          if (bytes) bulk_g2s(sm + (cur ^ 1) * wsz, a.band + q0 * ldab, bytes, &mbar[cur ^ 1]);
+        }
+      }
+      if (a.V2) {
+        double* vd = a.V2 + (off + m) * a.vs;
+        for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
+        if (tid == 0) a.tau2[off + m] = tau;
+      }
+      BC_TRACE(8);
+      cur ^= 1;
+      tau = tau_next;
+    }
+    if (tid == 0) {
+      bulk_wait_all();
+      fence_proxy_async_global();
+      st_release_s32(a.prog_full + s, (int)nst);
     }
   }
 }
 
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
-  const size_t flags = sizeof(int) * (size_t)(n + 64);
-  return ((band + 255) / 256) * 256 + ((flags + 255) / 256) * 256;
+  const size_t flags = sizeof(int) * (size_t)(2 * n + 128);
+  const size_t trace = sizeof(long long) * 2 * 1024 * 16;
+  return ((band + 255) / 256) * 256 + ((flags + 255) / 256) * 256 + trace;
 }
 
 cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
@@ -325,7 +581,11 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
   double* band = (double*)work;
   const size_t band_bytes = ((sizeof(double) * (size_t)n * ldab + 255) / 256) * 256;
   int* prog = (int*)((char*)work + band_bytes);
-  unsigned* ticket = (unsigned*)(prog + n + 32);
+  int* prog_full = prog + n + 32;
+  unsigned* ticket = (unsigned*)(prog_full + n + 32);
+  const size_t flags_bytes = ((sizeof(int) * (size_t)(2 * n + 128) + 255) / 256) * 256;
+  long long* trace = (long long*)((char*)work + band_bytes + flags_bytes);
+  const char* tr = getenv("TRID_BC_TRACE");
   {
     int64_t total = n * (int64_t)ldab;
     int blocks = (int)((total + 255) / 256);
@@ -336,29 +596,47 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     if (err != cudaSuccess) return err;
   }
   if (beff >= 2 && n >= 3) {
-    cudaError_t err = cudaMemsetAsync(prog, 0, sizeof(int) * (size_t)(n + 64), st);
+    cudaError_t err = cudaMemsetAsync(prog, 0, sizeof(int) * (size_t)(2 * n + 128), st);
     if (err != cudaSuccess) return err;
     BcArgs a;
     // beff = min(b, n-1) gives the same step geometry as b (for b >= n-1 every sweep is one step on
     // rows s+1..n-1); V2 keeps the caller's stride b (header contract).
     a.n = n; a.b = beff; a.ldab = ldab; a.vs = b; a.band = band; a.V2 = V2; a.tau2 = tau2; a.prog = prog;
+    a.prog_full = prog_full;
     a.ticket = ticket;
-    const size_t vec = sizeof(double) * (size_t)(4 * beff + BC_NT + 8);
-    const bool use_sm = beff <= BC_SMEM_MAXB;
-    const size_t smem = use_sm ? vec + sizeof(double) * 2 * (size_t)(beff + 1) * beff : vec;
+    a.trace = tr ? trace : nullptr;
+    a.trace_sweep = tr ? atoll(tr) : -1;
     int occ = 1;
-    if (use_sm) {
-      cudaFuncSetAttribute(bc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<true>, BC_NT, smem);
+    if (beff <= 64) {
+      const int B = beff <= 32 ? 32 : 64;
+      const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
+      const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256> : (const void*)bc_fast_kernel<64, 512>;
+      const int nth = B == 32 ? 256 : 512;
+      cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, nth, smem);
+      if (occ < 1) occ = 1;
+      int64_t grid = (int64_t)kNumSMsB200 * occ;
+      if (grid > n - 2) grid = n - 2;
+      if (B == 32) bc_fast_kernel<32, 256><<<(unsigned)grid, 256, smem, st>>>(a);
+      else bc_fast_kernel<64, 512><<<(unsigned)grid, 512, smem, st>>>(a);
     } else {
-      cudaFuncSetAttribute(bc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<false>, BC_NT, smem);
+      const size_t vec = sizeof(double) * (size_t)(5 * beff + 2 * BC_NT + 8);
+      const size_t winb = sizeof(double) * (size_t)beff * ldab;
+      const bool use_sm = vec + winb <= 200 * 1024;
+      const size_t smem = use_sm ? vec + winb : vec;
+      if (use_sm) {
+        cudaFuncSetAttribute(bc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<true>, BC_NT, smem);
+      } else {
+        cudaFuncSetAttribute(bc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<false>, BC_NT, smem);
+      }
+      if (occ < 1) occ = 1;
+      int64_t grid = (int64_t)kNumSMsB200 * occ;
+      if (grid > n - 2) grid = n - 2;
+      if (use_sm) bc_kernel<true><<<(unsigned)grid, BC_NT, smem, st>>>(a);
+      else bc_kernel<false><<<(unsigned)grid, BC_NT, smem, st>>>(a);
     }
-    if (occ < 1) occ = 1;
-    int64_t grid = (int64_t)kNumSMsB200 * occ;
-    if (grid > n - 2) grid = n - 2;
-    if (use_sm) bc_kernel<true><<<(unsigned)grid, BC_NT, smem, st>>>(a);
-    else bc_kernel<false><<<(unsigned)grid, BC_NT, smem, st>>>(a);
     count_launches(1);
     err = cudaGetLastError();
     if (err != cudaSuccess) return err;

@@ -28,6 +28,7 @@ struct PanelArgs {
   double* Y;
   int64_t ldy;
   double* red;
+  double* tot;
   unsigned* bar;
   int rows;      // rows per CTA
   int smem_ld;   // > 0: rows staged in shared memory with this leading dimension
@@ -65,7 +66,6 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
   __syncthreads();
 
   unsigned epoch = 0;
-  const int H = (RS <= PQ_NT) ? PQ_NT / RS : 1;
   for (int t = 0; t < a.kk; ++t) {
     double* red = a.red + (size_t)(t & 1) * G * RS;
     // ---- partial Gram row: slot j = sum_{r > t, r owned} P(r,t) P(r,j);  slot w+j = P(t,j) (owner)
@@ -81,27 +81,26 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
     const bool owner = (t >= rlo) && (t < rlo + nr);
     for (int j = tid; j < w; j += PQ_NT) red[(size_t)g * RS + w + j] = owner ? L[(size_t)j * ldl + (t - rlo)] : 0.0;
     grid_barrier(a.bar, (unsigned)G, epoch);
-    // ---- totals, fixed order over CTAs (identical in every CTA)
-    if (H > 1) {
-      if (tid < H * RS) {
-        const int s = tid % RS, h = tid / RS;
-        double acc = 0.0;
-        for (int gg = h; gg < G; gg += H) acc += __ldcg(&a.red[(size_t)(t & 1) * G * RS + (size_t)gg * RS + s]);
-        tmp[h * RS + s] = acc;
-      }
-      __syncthreads();
-      for (int s = tid; s < RS; s += PQ_NT) {
-        double acc = 0.0;
-        for (int h = 0; h < H; ++h) acc += tmp[h * RS + s];
-        tot[s] = acc;
-      }
-    } else {
-      for (int s = tid; s < RS; s += PQ_NT) {
-        double acc = 0.0;
-        for (int gg = 0; gg < G; ++gg) acc += __ldcg(&a.red[(size_t)(t & 1) * G * RS + (size_t)gg * RS + s]);
-        tot[s] = acc;
+    // ---- distributed reduction: CTA g sums slots s = g, g+G, ... over all CTAs in a fixed order
+    {
+      const double* src = a.red + (size_t)(t & 1) * G * RS;
+      double* dst = a.tot + (size_t)(t & 1) * RS;
+      for (int s = g; s < RS; s += G) {
+        double x = 0.0;
+        for (int gg = tid; gg < G; gg += PQ_NT) x += __ldcg(src + (size_t)gg * RS + s);
+        x = warp_sum(x);
+        if (lane == 0) tmp[warp] = x;
+        __syncthreads();
+        if (tid == 0) {
+          double acc = 0.0;
+          for (int q = 0; q < NW; ++q) acc += tmp[q];
+          __stcg(dst + s, acc);
+        }
+        __syncthreads();
       }
     }
+    grid_barrier(a.bar, (unsigned)G, epoch);
+    for (int s = tid; s < RS; s += PQ_NT) tot[s] = __ldcg(a.tot + (size_t)(t & 1) * RS + s);
     __syncthreads();
     // ---- reflector (R1), update vector, T inner products
     const House h = make_house(tot[w + t], tot[t]);
@@ -169,7 +168,7 @@ static int panel_grid(int64_t m) {
   return (int)G;
 }
 
-size_t panel_red_bytes(int w) { return sizeof(double) * 2 * (size_t)kNumSMsB200 * 2 * (size_t)w; }
+size_t panel_red_bytes(int w) { return sizeof(double) * (2 * (size_t)kNumSMsB200 * 2 * (size_t)w + 2 * 2 * (size_t)w); }
 
 cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
                      int64_t ldy, double* red, unsigned* bar, cudaStream_t st) {
@@ -177,7 +176,7 @@ cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, doub
   const int G = panel_grid(m);
   PanelArgs a;
   a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);
-  a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.red = red; a.bar = bar;
+  a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.red = red; a.tot = red + 2 * (size_t)kNumSMsB200 * 2 * w; a.bar = bar;
   a.rows = (int)((m + G - 1) / G);
   const size_t scr = sizeof(double) * (size_t)(2 * w + w + PQ_NT + 8);
   const size_t full = sizeof(double) * (size_t)a.rows * w + scr;
