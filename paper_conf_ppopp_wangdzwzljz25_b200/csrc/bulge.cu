@@ -311,21 +311,21 @@ __global__ void __launch_bounds__(BC_NT, 3) bc_kernel(BcArgs a) {
 //   * the window of step m+1 except its last column is prefetched while step m computes; after
 //     prog[s-1] >= m+2 only that last column (sweep s-1's published column 0) is loaded.
 // All sums are in a fixed order: results are bitwise reproducible and identical to sweep-major order.
-template <int B, int NTH>
-__global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
+template <int B, int NTH, int NBUF>
+__global__ void __launch_bounds__(NTH, 3 - NBUF) bc_fast_kernel(BcArgs a) {
   constexpr int TPR = NTH / (2 * B);   // column groups
   constexpr int CPT = B / TPR;         // columns per thread
   constexpr int RW = (2 * B) / 32;     // warps per column group
   constexpr int NW = NTH / 32;
   constexpr int CPW = B / NW;          // columns per warp in the z pass
-  static_assert(CPW == 4, "z-pass butterfly assumes 4 columns per warp");
+  static_assert(CPW == 4 || CPW == 8, "z-pass butterfly assumes 4 or 8 columns per warp");
   extern __shared__ __align__(16) double sm[];
   const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
   const int lda1 = ldab - 1;
   const int64_t n = a.n;
   const int wsz = B * ldab;
-  double* vb = sm + 2 * wsz;                 // 2 x B   (v / vn)
+  double* vb = sm + NBUF * wsz;              // 2 x B   (v / vn)
   double* pyv = vb + 2 * B;                  // 2B      tau*D v | O v
   double* zv = pyv + 2 * B;                  // B
   double* part = zv + B;                     // TPR x 2B matvec partials
@@ -356,7 +356,8 @@ __global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
       const int L = (int)(r1 - r0 + 1);
       const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
       const int L2 = (int)(r2 - r1);
-      double* win = sm + cur * wsz;
+      const int bi = NBUF == 2 ? cur : 0;
+      double* win = sm + bi * wsz;
       double* v = vb + (m & 1) * B;
       double* vn = vb + ((m & 1) ^ 1) * B;
       BC_TRACE(0);
@@ -390,17 +391,17 @@ __global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
         if (tid == 0) {
           fence_proxy_async_smem();
           fence_proxy_async_global();
-          mbar_arrive_expect_tx(&mbar[cur], (unsigned)(L * ldab * 8));
-          bulk_g2s(win, gsrc, (unsigned)(L * ldab * 8), &mbar[cur]);
-          mbar_arrive(&mbar[cur]);
+          mbar_arrive_expect_tx(&mbar[bi], (unsigned)(L * ldab * 8));
+          bulk_g2s(win, gsrc, (unsigned)(L * ldab * 8), &mbar[bi]);
+          mbar_arrive(&mbar[bi]);
         }
       } else if (tid == 0) {
         fence_proxy_async_global();
-        mbar_arrive_expect_tx(&mbar[cur], (unsigned)(ldab * 8));
-        bulk_g2s(win + (L - 1) * ldab, gsrc + (L - 1) * ldab, (unsigned)(ldab * 8), &mbar[cur]);
+        mbar_arrive_expect_tx(&mbar[bi], (unsigned)(ldab * 8));
+        bulk_g2s(win + (L - 1) * ldab, gsrc + (L - 1) * ldab, (unsigned)(ldab * 8), &mbar[bi]);
       }
-      mbar_wait(&mbar[cur], phase[cur]);
-      phase[cur] ^= 1u;
+      mbar_wait(&mbar[bi], phase[bi]);
+      phase[bi] ^= 1u;
       BC_TRACE(2);
       const bool active = r < L + L2;
       const bool isO = r >= L && active;
@@ -486,22 +487,26 @@ __global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
           }
           c[q] = acc;
         }
-        // transposed butterfly: 4 columns over 32 lanes in 6 shuffles, fixed partners
+        // transposed butterfly: CPW columns over 32 lanes, halving levels then full levels, fixed partners
         {
-          const bool up16 = (lane & 16) != 0;
-          const double s0 = up16 ? c[0] : c[2], s1 = up16 ? c[1] : c[3];
-          const double k0 = up16 ? c[2] : c[0], k1 = up16 ? c[3] : c[1];
-          double d0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 16);
-          double d1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 16);
-          const bool up8 = (lane & 8) != 0;
-          const double s2 = up8 ? d0 : d1, k2 = up8 ? d1 : d0;
-          double f = k2 + __shfl_xor_sync(0xffffffffu, s2, 8);
-          f += __shfl_xor_sync(0xffffffffu, f, 4);
-          f += __shfl_xor_sync(0xffffffffu, f, 2);
-          f += __shfl_xor_sync(0xffffffffu, f, 1);
-          if ((lane & 7) == 0) {
-            const int q = (up16 ? 2 : 0) + (up8 ? 1 : 0);
-            const int j = warp + q * NW;
+          int qbase = 0;
+#pragma unroll
+          for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
+            const bool up = (lane & o) != 0;
+#pragma unroll
+            for (int i = 0; i < K / 2; ++i) {
+              const double send = up ? c[i] : c[i + K / 2];
+              const double keep = up ? c[i + K / 2] : c[i];
+              c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+            }
+            if (up) qbase += K / 2;
+          }
+          constexpr int LV = CPW == 4 ? 2 : 3;   // halving levels used
+          double f = c[0];
+#pragma unroll
+          for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+          if ((lane & ((32 >> LV) - 1)) == 0) {
+            const int j = warp + qbase * NW;
             if (j >= 1 && j < L) zv[j] = fma(h2.scale, f, win[j * lda1 + L]);
           }
         }
@@ -544,9 +549,12 @@ __global__ void __launch_bounds__(NTH, 1) bc_fast_kernel(BcArgs a) {
           const int64_t q0 = r1 + 1;
           const int64_t q1 = (r1 + b < n - 1) ? r1 + b : n - 1;
           const unsigned bytes = (unsigned)((q1 - q0) * ldab * 8);   // (Lnext - 1) columns
+          const int nb2 = NBUF == 2 ? (cur ^ 1) : 0;
+          if (NBUF == 1) bulk_wait_read();   // single buffer: the stores above must have read it
+          fence_proxy_async_smem();
           fence_proxy_async_global();
-          mbar_arrive_expect_tx(&mbar[cur ^ 1], bytes);
-          if (bytes) bulk_g2s(sm + (cur ^ 1) * wsz, a.band + q0 * ldab, bytes, &mbar[cur ^ 1]);
+          mbar_arrive_expect_tx(&mbar[nb2], bytes);
+          if (bytes) bulk_g2s(sm + nb2 * wsz, a.band + q0 * ldab, bytes, &mbar[nb2]);
         }
       }
       if (a.V2) {
@@ -608,17 +616,25 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     a.trace_sweep = tr ? atoll(tr) : -1;
     int occ = 1;
     if (beff <= 64) {
+      // B = 64: 1 CTA/SM x 512 threads with a double-buffered window (default; n=32768: 458 ms) or, forced,
+      // 2 CTAs/SM x 256 threads with a single buffer (580 ms: the chase is dependency-chain bound).
       const int B = beff <= 32 ? 32 : 64;
-      const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
-      const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256> : (const void*)bc_fast_kernel<64, 512>;
-      const int nth = B == 32 ? 256 : 512;
+      bool two = false;   // measured: the chase is chain bound at every n in configs (1 CTA/SM, 512 thr wins)
+      const char* force = getenv("TRID_BC_FORCE");   // debug/test: "1" single-buffer 2 CTAs/SM, "2" double
+      if (force && B == 64) two = force[0] == '1';
+      const int nbuf = (B == 64 && two) ? 1 : 2;
+      const int nth = B == 32 ? 256 : (two ? 256 : 512);
+      const size_t smem = sizeof(double) * (nbuf * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
+      const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256, 2>
+                               : (two ? (const void*)bc_fast_kernel<64, 256, 1> : (const void*)bc_fast_kernel<64, 512, 2>);
       cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, nth, smem);
       if (occ < 1) occ = 1;
       int64_t grid = (int64_t)kNumSMsB200 * occ;
       if (grid > n - 2) grid = n - 2;
-      if (B == 32) bc_fast_kernel<32, 256><<<(unsigned)grid, 256, smem, st>>>(a);
-      else bc_fast_kernel<64, 512><<<(unsigned)grid, 512, smem, st>>>(a);
+      if (B == 32) bc_fast_kernel<32, 256, 2><<<(unsigned)grid, 256, smem, st>>>(a);
+      else if (two) bc_fast_kernel<64, 256, 1><<<(unsigned)grid, 256, smem, st>>>(a);
+      else bc_fast_kernel<64, 512, 2><<<(unsigned)grid, 512, smem, st>>>(a);
     } else {
       const size_t vec = sizeof(double) * (size_t)(5 * beff + 2 * BC_NT + 8);
       const size_t winb = sizeof(double) * (size_t)beff * ldab;

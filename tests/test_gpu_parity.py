@@ -132,6 +132,23 @@ def test_bulge_chase_parity(n, b, dev):
     assert np.max(np.abs(V2.cpu().numpy() - V_o), initial=0) <= 1e-9
 
 
+@pytest.mark.parametrize("variant", ["1", "2"])
+def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
+    """Both B=64 kernels (2 CTAs/SM single buffer, 1 CTA/SM double buffer) against the oracle."""
+    monkeypatch.setenv("TRID_BC_FORCE", variant)
+    n, b = 700, 64
+    Bm = band_from_lower(trid_gen.random_symmetric_np(n, 99), b)
+    d_o, e_o, V_o, t_o = oracle.bc_naive(Bm, b)
+    d, e, V2, tau2 = trid.bulge_chase(to_dev(Bm), b)
+    tol = 64 * n * U * np.linalg.norm(Bm)
+    assert np.max(np.abs(d.cpu().numpy() - d_o)) <= tol
+    assert np.max(np.abs(e.cpu().numpy() - e_o)) <= tol
+    assert np.max(np.abs(V2.cpu().numpy() - V_o)) <= 1e-9
+    r1 = [x.clone() for x in trid.bulge_chase(to_dev(Bm), b)]
+    for x, y in zip(r1, (d, e, V2, tau2)):
+        assert torch.equal(x, y)
+
+
 def test_bulge_chase_bitwise_deterministic(dev):
     n, b = 2000, 32
     Bm = band_from_lower(trid_gen.random_symmetric_np(n, 11), b)
