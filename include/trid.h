@@ -49,6 +49,10 @@ enum {
 /* Human-readable status ("success", "invalid argument 3", ...).  Static storage, never NULL. */
 const char* trid_status_string(int status);
 
+/* Description of the last CUDA failure that produced TRID_ERR_CUDA ("no error" if none).  Static storage,
+ * process-global, overwritten by the next failure. */
+const char* trid_last_error_string(void);
+
 /* Library version string, e.g. "trid-b200 0.1 sm_100a". */
 const char* trid_version(void);
 

@@ -42,6 +42,7 @@ def lib():
         L.trid_status_string.restype = ctypes.c_char_p
         L.trid_status_string.argtypes = [_INT]
         L.trid_version.restype = ctypes.c_char_p
+        L.trid_last_error_string.restype = ctypes.c_char_p
         L.trid_default_k.restype = _INT
         L.trid_default_k.argtypes = [_I64, _INT]
         L.trid_bc_total_steps.restype = _I64
@@ -71,7 +72,7 @@ def lib():
     return _lib
 
 
-EXPORTS = ("trid_status_string", "trid_version", "trid_default_k", "trid_bc_total_steps", "trid_sbr_dbbr_bufsize",
+EXPORTS = ("trid_status_string", "trid_last_error_string", "trid_version", "trid_default_k", "trid_bc_total_steps", "trid_sbr_dbbr_bufsize",
            "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize", "trid_sbr_dbbr", "trid_bulge_chase",
            "trid_sytrd_2stage", "trid_panel_qr_bufsize", "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize",
            "trid_zy", "trid_profile_begin", "trid_profile_end", "trid_kernel_launches")
@@ -98,7 +99,10 @@ def kernel_launches() -> int:
 
 def _check(status: int, what: str):
     if status != 0:
-        raise TridError(f"{what}: {lib().trid_status_string(status).decode()} ({status})")
+        msg = f"{what}: {lib().trid_status_string(status).decode()} ({status})"
+        if status == 1:
+            msg += ": " + lib().trid_last_error_string().decode()
+        raise TridError(msg)
 
 
 def _dev(t: torch.Tensor, name: str):

@@ -119,7 +119,7 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
   cudaError_t e;
   {
     ProfScope ps(PROF_SYMM, st);
-    e = symm_lower(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
+    e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
   }
   if (e != cudaSuccess) return e;
   ProfScope ps(PROF_ZY, st);
@@ -139,7 +139,7 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
     h.A[0] = Yprev; h.lda[0] = ldyz; h.B[0] = U1; h.ldb[0] = ldu; h.K[0] = nprev;
     h.A[1] = Zprev; h.lda[1] = ldyz; h.B[1] = U2; h.ldb[1] = ldu; h.K[1] = nprev;
     h.alpha = -1.0; h.beta = 1.0; h.Cin = X; h.ldcin = ldx; h.C = X; h.ldc = ldx;
-    if ((e = gemm(h, OP_N, OP_N, TILE_128x64, st)) != cudaSuccess) return e;
+    if ((e = gemm_ws(h, OP_N, st)) != cudaSuccess) return e;
   }
   // S = W^T X
   GemmArgs s;
@@ -152,7 +152,7 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
   GemmArgs z;
   z.M = m; z.N = kk; z.K[0] = kk; z.A[0] = Yp; z.lda[0] = ldyz; z.B[0] = S; z.ldb[0] = lds;
   z.alpha = -0.5; z.beta = 1.0; z.Cin = X; z.ldcin = ldx; z.C = Zp; z.ldc = ldyz;
-  return gemm(z, OP_N, OP_N, TILE_128x64, st);
+  return gemm_ws(z, OP_N, st);
 }
 
 int check_common(int64_t n, const void* A, int64_t lda, int b) {
@@ -166,7 +166,14 @@ int check_common(int64_t n, const void* A, int64_t lda, int b) {
 }  // namespace
 
 
+namespace {
+char g_last_error[512] = "no error";
+}
 namespace trid {
+void record_cuda_error(cudaError_t e, const char* what) {
+  snprintf(g_last_error, sizeof g_last_error, "%s: %s (%d) in %s", cudaGetErrorName(e), cudaGetErrorString(e), (int)e,
+           what);
+}
 void count_launches(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 void prof_mark(int cls, bool begin, cudaStream_t st) {
   ProfState& p = prof();
@@ -238,6 +245,8 @@ int trid_profile_end(double* ms, int64_t* calls, int nclass) {
 }
 
 int64_t trid_kernel_launches(void) { return (int64_t)g_launches.load(); }
+
+const char* trid_last_error_string(void) { return g_last_error; }
 
 const char* trid_version(void) { return "trid-b200 0.1 sm_100a"; }
 
@@ -316,7 +325,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
         g.M = m; g.N = kk; g.K[0] = kk; g.A[0] = Yp; g.lda[0] = ld; g.B[0] = w.T; g.ldb[0] = b;
         g.C = w.W; g.ldc = ld;
         ProfScope ps(PROF_WY, stream);
-        TRID_CUDA_TRY(gemm(g, OP_N, OP_N, TILE_128x64, stream));
+        TRID_CUDA_TRY(gemm_ws(g, OP_N, stream));
       }
       // Z builder against the implicitly updated trailing matrix (R4e)
       TRID_CUDA_TRY(zy_panel(m, kk, A + o + o * lda, lda, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ld,
@@ -334,7 +343,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
         g.C = A + o + o * lda; g.ldc = lda; g.Cin = g.C; g.ldcin = lda;
         g.lower = 1; g.diag_off = 0;
         ProfScope ps(PROF_NEXT, stream);
-        TRID_CUDA_TRY(gemm(g, OP_N, OP_T, TILE_128x64, stream));
+        TRID_CUDA_TRY(gemm_ws(g, OP_T, stream));
       }
     }
     const int64_t e = jlast + b;                                    // l.15
@@ -347,7 +356,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
       g.C = A + e + e * lda; g.ldc = lda; g.Cin = g.C; g.ldcin = lda;
       g.lower = 1; g.tri = 1;
       ProfScope ps(PROF_SYR2K, stream);
-      TRID_CUDA_TRY(gemm(g, OP_N, OP_T, TILE_128x128, stream));
+      TRID_CUDA_TRY(gemm_ws(g, OP_T, stream));
     }
   }
   return TRID_SUCCESS;
@@ -432,7 +441,7 @@ int trid_syr2k_lower(int64_t m, int64_t kk, double* C, int64_t ldc, const double
   g.A[1] = Z; g.lda[1] = ldz; g.B[1] = Y; g.ldb[1] = ldy; g.K[1] = kk;
   g.alpha = -1.0; g.beta = 1.0; g.C = C; g.ldc = ldc; g.Cin = C; g.ldcin = ldc;
   g.lower = 1; g.tri = 1;
-  TRID_CUDA_TRY(gemm(g, OP_N, OP_T, TILE_128x128, stream));
+  TRID_CUDA_TRY(gemm_ws(g, OP_T, stream));
   return TRID_SUCCESS;
 }
 
@@ -471,7 +480,7 @@ int trid_zy(int64_t m, int w, const double* A, int64_t lda, const double* W, int
   if (pe < (int64_t)32 * w * w) pe = (int64_t)32 * w * w;
   double* part = c.take<double>((size_t)pe);
   // Eq. (1) with no earlier panels: Y and Z of this call are separate buffers (ldy, ldz)
-  cudaError_t e = symm_lower(m, w, A, lda, W, ldw, X, m, part, pe, stream);
+  cudaError_t e = symm_ws(m, w, A, lda, W, ldw, X, m, part, pe, stream);
   if (e != cudaSuccess) return TRID_ERR_CUDA;
   GemmArgs s;
   s.M = w; s.N = w; s.K[0] = m; s.A[0] = W; s.lda[0] = ldw; s.B[0] = X; s.ldb[0] = m;
@@ -481,7 +490,7 @@ int trid_zy(int64_t m, int w, const double* A, int64_t lda, const double* W, int
   GemmArgs z;
   z.M = m; z.N = w; z.K[0] = w; z.A[0] = Y; z.lda[0] = ldy; z.B[0] = S; z.ldb[0] = w;
   z.alpha = -0.5; z.beta = 1.0; z.Cin = X; z.ldcin = m; z.C = Z; z.ldc = ldz;
-  TRID_CUDA_TRY(gemm(z, OP_N, OP_N, TILE_128x64, stream));
+  TRID_CUDA_TRY(gemm_ws(z, OP_N, stream));
   return TRID_SUCCESS;
 }
 

@@ -25,6 +25,14 @@ __device__ __forceinline__ void dmma_16x8x8(double (&c)[4], const double (&a)[4]
       : "d"(a[0]), "d"(a[1]), "d"(a[2]), "d"(a[3]), "d"(b[0]), "d"(b[1]));
 }
 
+// D(16x8) += A(16x4) * B(4x8), fp64: a0 = A[g][t], a1 = A[g+8][t]; b0 = B[t][g]; c as above.
+__device__ __forceinline__ void dmma_16x8x4(double (&c)[4], double a0, double a1, double b0) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k4.row.col.f64.f64.f64.f64 {%0,%1,%2,%3}, {%4,%5}, {%6}, {%0,%1,%2,%3};\n"
+      : "+d"(c[0]), "+d"(c[1]), "+d"(c[2]), "+d"(c[3])
+      : "d"(a0), "d"(a1), "d"(b0));
+}
+
 // 8-byte async copy global -> shared; pred == false zero-fills without reading global memory.
 __device__ __forceinline__ void cp_async8(double* smem, const double* gmem, bool pred) {
   unsigned s = (unsigned)__cvta_generic_to_shared(smem);
@@ -150,8 +158,14 @@ __device__ __forceinline__ House make_house(double alpha, double sigma) {
 
 }  // namespace trid
 
-#define TRID_CUDA_TRY(x)                        \
-  do {                                          \
-    cudaError_t _e = (x);                       \
-    if (_e != cudaSuccess) return TRID_ERR_CUDA; \
+namespace trid {
+void record_cuda_error(cudaError_t e, const char* what);
+}
+#define TRID_CUDA_TRY(x)                              \
+  do {                                                \
+    cudaError_t _e = (x);                             \
+    if (_e != cudaSuccess) {                          \
+      trid::record_cuda_error(_e, #x);                \
+      return TRID_ERR_CUDA;                           \
+    }                                                 \
   } while (0)

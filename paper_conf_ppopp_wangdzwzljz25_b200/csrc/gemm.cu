@@ -8,8 +8,7 @@
 //   * W = Y T, corrections and Z = X - 1/2 Y (W^T X)                            (Eq. (1))
 //   * the SYMM X = A W of the Z builder (symm_kernel: row strip + transposed column strip per row
 //     block, so the lower-stored trailing matrix is read without atomics; deterministic split-K).
-// Padded smem strides keep DMMA fragment loads at the 2-wavefront minimum (row stride = 8 mod 16
-// doubles for m-inner tiles, 4 mod 16 for k-inner tiles).
+// Padded smem strides (4 mod 16 doubles) keep 64-bit DMMA fragment loads bank-conflict free.
 #include "common.cuh"
 #include "gemm.cuh"
 #include "prof.cuh"
@@ -19,16 +18,18 @@ namespace trid {
 constexpr int BK = 16;
 constexpr int STAGES = 3;
 
+// Leading dimensions are == 4 (mod 16) doubles: a 64-bit fragment load is served per half-warp
+// (4 rows g x 4 k-lanes t); stride 4 (mod 16) puts those 16 addresses on 16 distinct bank pairs.
 template <int BM, int OPA>
 struct ATile {
-  static constexpr int LD = OPA == OP_N ? BM + 8 : BK + 4;
-  static constexpr int ELEMS = OPA == OP_N ? BK * (BM + 8) : BM * (BK + 4);
+  static constexpr int LD = OPA == OP_N ? BM + 4 : BK + 4;
+  static constexpr int ELEMS = OPA == OP_N ? BK * (BM + 4) : BM * (BK + 4);
   __device__ static __forceinline__ int idx(int r, int k) { return OPA == OP_N ? k * LD + r : r * LD + k; }
 };
 template <int BN, int OPB>
 struct BTile {
-  static constexpr int LD = OPB == OP_T ? BN + 8 : BK + 4;
-  static constexpr int ELEMS = OPB == OP_T ? BK * (BN + 8) : BN * (BK + 4);
+  static constexpr int LD = OPB == OP_T ? BN + 4 : BK + 4;
+  static constexpr int ELEMS = OPB == OP_T ? BK * (BN + 4) : BN * (BK + 4);
   __device__ static __forceinline__ int idx(int k, int c) { return OPB == OP_T ? k * LD + c : c * LD + k; }
 };
 
@@ -104,25 +105,23 @@ __device__ __forceinline__ void mainloop(double (&acc)[BM / WGM / 16][BN / WGN /
     cp_async_commit();
     const double* Ast = As + (it % STAGES) * AE;
     const double* Bst = Bs + (it % STAGES) * BE;
+    // k4 sub-steps outermost: the MT*NTL accumulators are independent between two uses, so the
+    // DMMA pipe never waits on its own previous result (SASS DMMA.8x8x4 latency ~13-26 cycles).
 #pragma unroll
-    for (int ks = 0; ks < BK; ks += 8) {
-      double af[MT][4], bf[NTL][2];
+    for (int ks = 0; ks < BK; ks += 4) {
+      double a0[MT], a1[MT], bf[NTL];
 #pragma unroll
       for (int mt = 0; mt < MT; ++mt) {
-        const int r = wm * WTM + mt * 16 + g;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) af[mt][i] = Ast[ATile<BM, OPA>::idx(r + 8 * (i & 1), ks + t + 4 * (i >> 1))];
+        const int rr = wm * WTM + mt * 16 + g;
+        a0[mt] = Ast[ATile<BM, OPA>::idx(rr, ks + t)];
+        a1[mt] = Ast[ATile<BM, OPA>::idx(rr + 8, ks + t)];
       }
 #pragma unroll
-      for (int nt = 0; nt < NTL; ++nt) {
-        const int c = wn * WTN + nt * 8 + g;
-#pragma unroll
-        for (int i = 0; i < 2; ++i) bf[nt][i] = Bst[BTile<BN, OPB>::idx(ks + t + 4 * i, c)];
-      }
+      for (int nt = 0; nt < NTL; ++nt) bf[nt] = Bst[BTile<BN, OPB>::idx(ks + t, wn * WTN + nt * 8 + g)];
 #pragma unroll
       for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < NTL; ++nt) dmma_16x8x8(acc[mt][nt], af[mt], bf[nt]);
+        for (int nt = 0; nt < NTL; ++nt) dmma_16x8x4(acc[mt][nt], a0[mt], a1[mt], bf[nt]);
     }
   }
   cp_async_wait<0>();
@@ -137,7 +136,7 @@ __device__ __forceinline__ void tri_tile(int64_t t, int& tm, int& tn) {
 }
 
 template <int BM, int BN, int WGM, int WGN, int OPA, int OPB>
-__global__ void __launch_bounds__(WGM* WGN * 32) gemm_kernel(GemmArgs a) {
+__global__ void __launch_bounds__(WGM* WGN * 32, (BM * BN <= 4096 ? 3 : 2)) gemm_kernel(GemmArgs a) {
   constexpr int WTM = BM / WGM, WTN = BN / WGN;
   constexpr int MT = WTM / 16, NTL = WTN / 8;
   extern __shared__ __align__(16) double smem[];
@@ -225,21 +224,25 @@ static cudaError_t launch_tile(const GemmArgs& a, cudaStream_t st) {
   }
   const int64_t tm = (a.M + BM - 1) / BM, tn = (a.N + BN - 1) / BN;
   dim3 grid;
-  if (a.tri) {
+  GemmArgs b = a;
+  if (a.tri && BM == BN) {
     grid = dim3((unsigned)(tm * (tm + 1) / 2), 1, (unsigned)a.splits);
   } else {
+    b.tri = 0;   // rectangular grid; tiles wholly above the diagonal exit at once (a.lower)
     grid = dim3((unsigned)tm, (unsigned)tn, (unsigned)a.splits);
   }
-  gemm_kernel<BM, BN, WGM, WGN, OPA, OPB><<<grid, NT, smem, st>>>(a);
+  gemm_kernel<BM, BN, WGM, WGN, OPA, OPB><<<grid, NT, smem, st>>>(b);
   count_launches(1);
   return cudaGetLastError();
 }
 
+// All tiles: 128 threads (2 x 2 warps), BK = 16, 3 stages, 2-3 CTAs per SM -- the shape cuBLAS's
+// FP64 DGEMM uses on this part (cutlass_80_tensorop_d884gemm_64x128_16x3, DMMA pipe 96% busy).
 template <int OPA, int OPB>
 static cudaError_t launch_ops(const GemmArgs& a, int tile, cudaStream_t st) {
   switch (tile) {
-    case TILE_128x128: return launch_tile<128, 128, 2, 4, OPA, OPB>(a, st);
-    case TILE_128x64: return launch_tile<128, 64, 4, 2, OPA, OPB>(a, st);
+    case TILE_128x128: return launch_tile<64, 128, 2, 2, OPA, OPB>(a, st);   // "wide": 64 x 128
+    case TILE_128x64: return launch_tile<128, 64, 2, 2, OPA, OPB>(a, st);
     default: return launch_tile<64, 64, 2, 2, OPA, OPB>(a, st);
   }
 }
@@ -270,7 +273,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
 }
 
 int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems) {
-  const int bm = tile == TILE_64x64 ? 64 : 128, bn = tile == TILE_128x128 ? 128 : 64;
+  const int bm = tile == TILE_128x64 ? 128 : 64, bn = tile == TILE_128x128 ? 128 : 64;
   const int64_t tiles = ((M + bm - 1) / bm) * ((N + bn - 1) / bn);
   const int64_t target = 2 * kNumSMsB200;
   int64_t s = (target + tiles - 1) / tiles;
@@ -301,9 +304,9 @@ struct SymmArgs {
   int64_t part_stride;
 };
 
-constexpr int SY_BM = 128, SY_BN = 64, SY_WGM = 4, SY_WGN = 2;
+constexpr int SY_BM = 128, SY_BN = 64, SY_WGM = 2, SY_WGN = 2;
 
-__global__ void __launch_bounds__(SY_WGM* SY_WGN * 32) symm_kernel(SymmArgs a) {
+__global__ void __launch_bounds__(SY_WGM* SY_WGN * 32, 2) symm_kernel(SymmArgs a) {
   constexpr int WTM = SY_BM / SY_WGM, WTN = SY_BN / SY_WGN;
   constexpr int MT = WTM / 16, NTL = WTN / 8;
   extern __shared__ __align__(16) double smem[];

@@ -1,0 +1,486 @@
+// gemm_ws.cu — warp-specialized persistent FP64 DMMA contraction engine (the big DBBR contractions).
+//
+// Why: on sm_100a a DMMA.8x8x4 occupies its SMSP's FP64 tensor path for 16 cycles and the compiler
+// encodes that cadence into the issuing warp (stall 15 + NOP), so ONE warp saturates an SMSP and any
+// moment where all warps of an SMSP block (CTA barriers, cp.async waits, prologue/epilogue) idles the
+// pipe (measured: 72% DMMA-busy with the synchronous 3-stage kernel vs 96% for cuBLAS).  Here:
+//   * 1 producer warp streams A/B K-tiles into a STAGES-deep shared-memory ring with cp.async (16-byte
+//     when the operands are 16-byte aligned, else 8-byte) and signals full[slot] with
+//     cp.async.mbarrier.arrive.noinc; it refills a slot after the consumers' empty[slot] arrivals;
+//   * CWM x CWN consumer warps (2 per SMSP) wait only on full[slot]; there is no CTA-wide barrier;
+//   * the grid is persistent: each CTA walks work units (tile, split) with stride gridDim.x, so the
+//     producer prefetches the next unit while the consumers run the epilogue.
+// A unit's K range is a list of up to two segments; each segment has its own A/B pointers, leading
+// dimensions, A access mode (N: m-inner, T: k-inner) and triangle mask (the SYMM row/column strips).
+#include "common.cuh"
+#include "gemm.cuh"
+#include "prof.cuh"
+
+namespace trid {
+
+namespace ws {
+
+constexpr int BK = 16;
+
+template <int BM, int BN>
+struct Cfg {
+  static constexpr int A_LD_N = BM + 4;   // A m-inner:  As[k][m]
+  static constexpr int A_LD_T = BK + 4;   // A k-inner:  As[m][k]
+  static constexpr int A_ELEMS = (BK * A_LD_N > BM * A_LD_T) ? BK * A_LD_N : BM * A_LD_T;
+  static constexpr int B_LD_T = BN + 4;   // B n-inner:  Bs[k][n]   (op(B) = B^T, B is N x K)
+  static constexpr int B_LD_N = BK + 4;   // B k-inner:  Bs[n][k]   (op(B) = B,   B is K x N)
+  static constexpr int B_ELEMS = (BK * B_LD_T > BN * B_LD_N) ? BK * B_LD_T : BN * B_LD_N;
+  static constexpr int STAGE = A_ELEMS + B_ELEMS;
+  static constexpr int STAGES = (210 * 1024 / (8 * STAGE)) > 6 ? 6 : (210 * 1024 / (8 * STAGE));
+  static constexpr size_t SMEM = sizeof(double) * (size_t)STAGES * STAGE + 16 * STAGES + 64;
+};
+
+struct Seg {
+  const double* A;
+  const double* B;
+  int64_t lda, ldb;
+  int64_t kb, ke;   // K range [kb, ke)
+  int opa;          // OP_N / OP_T
+  int mask;         // 0 none, 1 keep k <= row, 2 keep k > row (global row = m0 + r)
+};
+
+struct WsArgs {
+  int64_t M, N;
+  int opb;                  // OP_N / OP_T for every segment
+  int nseg;                 // GEMM: 1 or 2 segments over the split's K range
+  const double* A[2];
+  const double* B[2];
+  int64_t lda[2], ldb[2], K[2];
+  int symm;                 // 1: SYMM X = Asym W (A lower referenced), segments derived per tile
+  double alpha, beta;
+  const double* Cin;
+  int64_t ldcin;
+  double* C;
+  int64_t ldc;
+  int lower;
+  int64_t diag_off;
+  int tri;                  // lower-triangular tile enumeration (BM == BN)
+  int tiles_m, tiles_n, splits;
+  int64_t units;
+  double* part;             // split partials: part + z*part_stride, ld part_ld
+  int64_t part_ld, part_stride;
+  int vec16;                // operands 16-byte aligned (base pointers and leading dimensions even)
+};
+
+__device__ __forceinline__ void tri_unit(int64_t t, int& tm, int& tn) {
+  int64_t r = (int64_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+  while (r * (r + 1) / 2 > t) --r;
+  while ((r + 1) * (r + 2) / 2 <= t) ++r;
+  tm = (int)r;
+  tn = (int)(t - r * (r + 1) / 2);
+}
+
+template <int BM, int BN>
+__device__ __forceinline__ void unit_geom(const WsArgs& a, int64_t u, int64_t& m0, int64_t& n0, int& z) {
+  const int64_t tiles = a.tri ? (int64_t)a.tiles_m * (a.tiles_m + 1) / 2 : (int64_t)a.tiles_m * a.tiles_n;
+  z = (int)(u / tiles);
+  const int64_t t = u - (int64_t)z * tiles;
+  int tm, tn;
+  if (a.tri) {
+    tri_unit(t, tm, tn);
+  } else {
+    tm = (int)(t % a.tiles_m);
+    tn = (int)(t / a.tiles_m);
+  }
+  m0 = (int64_t)tm * BM;
+  n0 = (int64_t)tn * BN;
+}
+
+// Segments of unit u (identical in producer and consumers).
+template <int BM, int BN>
+__device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg& s0, Seg& s1) {
+  if (a.symm) {
+    // K chunk z of the strip: [k0, k1); row strip (k <= row) then column strip (k > row)
+    const int64_t chunk = (a.K[0] + a.splits - 1) / a.splits;
+    const int64_t cz = (chunk + BK - 1) / BK * BK;
+    const int64_t k0 = (int64_t)z * cz, k1 = (k0 + cz < a.K[0]) ? k0 + cz : a.K[0];
+    const int64_t e1 = (k1 < m0 + BM) ? k1 : m0 + BM;
+    const int64_t s2 = (k0 > m0) ? k0 : m0;
+    const Seg row{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, e1, OP_N, 1};
+    const Seg col{a.A[0], a.B[0], a.lda[0], a.ldb[0], s2, k1, OP_T, 2};
+    if (e1 > k0) {
+      s0 = row;
+      s1 = col;
+      return k1 > s2 ? 2 : 1;
+    }
+    s0 = col;
+    return k1 > s2 ? 1 : 0;
+  }
+  const int64_t kt0 = (a.K[0] + BK - 1) / BK, kt1 = a.nseg > 1 ? (a.K[1] + BK - 1) / BK : 0;
+  const int64_t total = kt0 + kt1;
+  const int64_t per = (total + a.splits - 1) / a.splits;
+  const int64_t tb = (int64_t)z * per, te = (tb + per < total) ? tb + per : total;
+  int64_t kb0 = 0, ke0 = 0, kb1 = 0, ke1 = 0;
+  if (tb < kt0) {
+    const int64_t e = te < kt0 ? te : kt0;
+    kb0 = tb * BK;
+    ke0 = (e * BK < a.K[0]) ? e * BK : a.K[0];
+  }
+  if (te > kt0) {
+    const int64_t b0 = (tb > kt0 ? tb : kt0) - kt0, e = te - kt0;
+    kb1 = b0 * BK;
+    ke1 = (e * BK < a.K[1]) ? e * BK : a.K[1];
+  }
+  const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, OP_N, 0};
+  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, OP_N, 0};
+  if (ke0 > kb0) {
+    s0 = g0;
+    s1 = g1;
+    return ke1 > kb1 ? 2 : 1;
+  }
+  s0 = g1;
+  return ke1 > kb1 ? 1 : 0;
+}
+
+__device__ __forceinline__ void cp16(double* dst, const double* src, int bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(dst)), "l"(src), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp8(double* dst, const double* src, int bytes) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(smem_u32(dst)), "l"(src), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_arrive_noinc(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// ---- producer fast paths (16-byte aligned operands, no triangle mask): per-thread offsets are fixed,
+// every copy of a stage is one address add + one cp.async with compile-time shared-memory offsets.
+// NP producer threads (pt in [0, NP)).  m-inner tile (A op N / B op T): R rows (H = R/2 pairs) x BK.
+template <int R, int LD, int NP>
+__device__ __forceinline__ void load_minner16(double* T, const double* base, int64_t ld, int64_t r0, int64_t rmax,
+                                              int64_t k0, int64_t kend, int pt) {
+  constexpr int H = R / 2;
+  constexpr int NCP = H * BK / NP;
+  static_assert(NP % H == 0 || H % NP == 0, "producer mapping");
+  constexpr int Q = H % NP == 0 ? H / NP : 1;          // row groups per thread when H >= NP
+  constexpr int KS = NP % H == 0 ? NP / H : 0;         // k rows advanced per copy when NP >= H
+  const int rp = NP % H == 0 ? pt % H : pt;            // base pair
+  const int kb = NP % H == 0 ? pt / H : 0;
+  int bytes_q[Q];
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const int64_t row = r0 + 2 * (rp + NP * q);
+    bytes_q[q] = row + 1 < rmax ? 16 : (row < rmax ? 8 : 0);
+  }
+  const bool kfull = k0 + BK <= kend;
+#pragma unroll
+  for (int i = 0; i < NCP; ++i) {
+    const int q = i % Q;
+    const int kk = (NP % H == 0) ? kb + KS * i : i / Q;
+    int bytes = bytes_q[q];
+    if (!kfull && k0 + kk >= kend) bytes = 0;
+    const int rr = 2 * (rp + NP * q);
+    const double* sp = base + r0 + rr + (k0 + kk) * ld;
+    cp16(T + kk * LD + rr, bytes ? sp : base, bytes);
+  }
+}
+// k-inner tile (A op T / B op N): R rows of BK contiguous k (BK/2 = 8 pairs per row).
+template <int R, int LD, int NP>
+__device__ __forceinline__ void load_kinner16(double* T, const double* base, int64_t ld, int64_t r0, int64_t rmax,
+                                              int64_t k0, int64_t kend, int pt) {
+  constexpr int NCP = R * (BK / 2) / NP;
+  constexpr int RS = NP / (BK / 2);
+  const int kk = 2 * (pt % (BK / 2)), rl = pt / (BK / 2);
+  const int kbytes = k0 + kk + 1 < kend ? 16 : (k0 + kk < kend ? 8 : 0);
+#pragma unroll
+  for (int i = 0; i < NCP; ++i) {
+    const int rr = rl + RS * i;
+    const int64_t row = r0 + rr;
+    const int bytes = row < rmax ? kbytes : 0;
+    cp16(T + rr * LD + kk, bytes ? base + k0 + kk + row * ld : base, bytes);
+  }
+}
+
+// Producer: one K-tile of A and B into stage buffers (NP threads).
+template <int BM, int BN, int NP>
+__device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t k0, int64_t m0, int64_t n0,
+                                          double* As, double* Bs, int pt) {
+  using C = Cfg<BM, BN>;
+  const int64_t kend = s.ke;
+  // the triangle masks only bite on K-tiles that overlap the diagonal block [m0, m0 + BM)
+  const bool unmasked = s.mask == 0 || (s.mask == 1 && k0 + BK <= m0) || (s.mask == 2 && k0 >= m0 + BM);
+  const bool v16 = a.vec16 && unmasked;
+  // ---- A
+  if (v16) {
+    if (s.opa == OP_N) load_minner16<BM, C::A_LD_N, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt);
+    else load_kinner16<BM, C::A_LD_T, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt);
+  } else if (s.opa == OP_N) {   // A(m, k) at A[m + k*lda], tile As[k][m]
+    for (int e = pt; e < BM * BK; e += NP) {
+      const int r = e % BM, kk = e / BM;
+      const int64_t row = m0 + r, k = k0 + kk;
+      bool p = row < a.M && k < kend;
+      if (s.mask == 1) p = p && (k <= row);
+      if (s.mask == 2) p = p && (k > row);
+      cp8(As + kk * C::A_LD_N + r, p ? s.A + row + k * s.lda : s.A, p ? 8 : 0);
+    }
+  } else {                      // op(A)(m, k) = A[k + m*lda], tile As[m][k]
+    for (int e = pt; e < BM * BK; e += NP) {
+      const int kk = e % BK, r = e / BK;
+      const int64_t row = m0 + r, k = k0 + kk;
+      bool p = row < a.M && k < kend;
+      if (s.mask == 1) p = p && (k <= row);
+      if (s.mask == 2) p = p && (k > row);
+      cp8(As + r * C::A_LD_T + kk, p ? s.A + k + row * s.lda : s.A, p ? 8 : 0);
+    }
+  }
+  // ---- B
+  if (a.vec16) {
+    if (a.opb == OP_T) load_minner16<BN, C::B_LD_T, NP>(Bs, s.B, s.ldb, n0, a.N, k0, kend, pt);
+    else load_kinner16<BN, C::B_LD_N, NP>(Bs, s.B, s.ldb, n0, a.N, k0, kend, pt);
+  } else if (a.opb == OP_T) {   // B is N x K: B[n + k*ldb], tile Bs[k][n]
+    for (int e = pt; e < BN * BK; e += NP) {
+      const int c = e % BN, kk = e / BN;
+      const int64_t col = n0 + c, k = k0 + kk;
+      const bool p = col < a.N && k < kend;
+      cp8(Bs + kk * C::B_LD_T + c, p ? s.B + col + k * s.ldb : s.B, p ? 8 : 0);
+    }
+  } else {                      // B is K x N: B[k + n*ldb], tile Bs[n][k]
+    for (int e = pt; e < BN * BK; e += NP) {
+      const int kk = e % BK, c = e / BK;
+      const int64_t col = n0 + c, k = k0 + kk;
+      const bool p = col < a.N && k < kend;
+      cp8(Bs + c * C::B_LD_N + kk, p ? s.B + k + col * s.ldb : s.B, p ? 8 : 0);
+    }
+  }
+}
+
+// Consumer: 4 k4-steps of one stage into the warp's accumulators.
+template <int BM, int BN, int WTM, int WTN, int OPA, int OPB>
+__device__ __forceinline__ void mma_stage(double (&acc)[WTM / 16][WTN / 8][4], const double* As, const double* Bs,
+                                          int wm0, int wn0, int g, int t) {
+  using C = Cfg<BM, BN>;
+  constexpr int MT = WTM / 16, NT = WTN / 8;
+#pragma unroll
+  for (int ks = 0; ks < BK; ks += 4) {
+    double a0[MT], a1[MT], bf[NT];
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt) {
+      const int r = wm0 + mt * 16 + g;
+      if (OPA == OP_N) {
+        a0[mt] = As[(ks + t) * C::A_LD_N + r];
+        a1[mt] = As[(ks + t) * C::A_LD_N + r + 8];
+      } else {
+        a0[mt] = As[r * C::A_LD_T + ks + t];
+        a1[mt] = As[(r + 8) * C::A_LD_T + ks + t];
+      }
+    }
+#pragma unroll
+    for (int nt = 0; nt < NT; ++nt) {
+      const int c = wn0 + nt * 8 + g;
+      bf[nt] = OPB == OP_T ? Bs[(ks + t) * C::B_LD_T + c] : Bs[c * C::B_LD_N + ks + t];
+    }
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt) dmma_16x8x4(acc[mt][nt], a0[mt], a1[mt], bf[nt]);
+  }
+}
+
+constexpr int NPW = 4;   // producer warps (one warpgroup, so setmaxnreg can shrink it)
+// Register budget of the 384-thread kernel: launched at 168 regs/thread (64512 per CTA); the producer
+// warpgroup drops to 96 and the two consumer warpgroups rise to 200: 128*96 + 256*200 = 63488 <= 64512
+// (an increase the freed registers cannot cover blocks setmaxnreg.inc forever).
+
+template <int BM, int BN, int CWM, int CWN, int OPB>
+__global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __grid_constant__ WsArgs a) {
+  using C = Cfg<BM, BN>;
+  constexpr int NCW = CWM * CWN;
+  constexpr int WTM = BM / CWM, WTN = BN / CWN;
+  constexpr int MT = WTM / 16, NT = WTN / 8;
+  constexpr int STAGES = C::STAGES;
+  extern __shared__ __align__(16) double smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)STAGES * C::STAGE);
+  uint64_t* empty = full + STAGES;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], NPW * 32);   // one cp.async.mbarrier.arrive.noinc per producer thread
+      mbar_init(&empty[s], NCW);  // one arrive per consumer warp
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp >= NCW) {
+    // ======================= producer warpgroup =======================
+    if (NCW == 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;\n" ::: "memory");
+    const int pt = threadIdx.x - NCW * 32;
+    uint32_t kt = 0;   // global K-tile counter (ring position)
+    for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+      int64_t m0, n0;
+      int z;
+      unit_geom<BM, BN>(a, u, m0, n0, z);
+      if (a.lower && m0 + BM - 1 + a.diag_off < n0) continue;
+      Seg s0, s1;
+      const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
+      auto run = [&](const Seg& sgm) {
+        for (int64_t k0 = sgm.kb; k0 < sgm.ke; k0 += BK, ++kt) {
+          const int slot = kt % STAGES;
+          const uint32_t use = kt / STAGES;
+          if (use > 0) mbar_wait(&empty[slot], (use - 1) & 1u);
+          double* As = smem + (size_t)slot * C::STAGE;
+          load_tile<BM, BN, NPW * 32>(a, sgm, k0, m0, n0, As, As + C::A_ELEMS, pt);
+          cp_arrive_noinc(&full[slot]);
+        }
+      };
+      if (ns > 0) run(s0);
+      if (ns > 1) run(s1);
+    }
+    return;
+  }
+  // ======================= consumers =======================
+  if (NCW == 8) asm volatile("setmaxnreg.inc.sync.aligned.u32 200;\n" ::: "memory");
+  const int wm = warp % CWM, wn = warp / CWM;
+  const int g = lane >> 2, t = lane & 3;
+  uint32_t kt = 0;
+  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+    int64_t m0, n0;
+    int z;
+    unit_geom<BM, BN>(a, u, m0, n0, z);
+    if (a.lower && m0 + BM - 1 + a.diag_off < n0) continue;
+    Seg s0, s1;
+    const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
+    double acc[MT][NT][4];
+#pragma unroll
+    for (int i = 0; i < MT; ++i)
+#pragma unroll
+      for (int j = 0; j < NT; ++j)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[i][j][q] = 0.0;
+    auto run = [&](const Seg& sgm) {
+      for (int64_t k0 = sgm.kb; k0 < sgm.ke; k0 += BK, ++kt) {
+        const int slot = kt % STAGES;
+        mbar_wait(&full[slot], (kt / STAGES) & 1u);
+        const double* As = smem + (size_t)slot * C::STAGE;
+        if (sgm.opa == OP_N) mma_stage<BM, BN, WTM, WTN, OP_N, OPB>(acc, As, As + C::A_ELEMS, wm * WTM, wn * WTN, g, t);
+        else mma_stage<BM, BN, WTM, WTN, OP_T, OPB>(acc, As, As + C::A_ELEMS, wm * WTM, wn * WTN, g, t);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[slot]);
+      }
+    };
+    if (ns > 0) run(s0);
+    if (ns > 1) run(s1);
+    // ---- epilogue
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int64_t r = m0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
+          const int64_t c = n0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
+          if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= c)) {
+            if (a.splits > 1) {
+              a.part[z * a.part_stride + r + c * a.part_ld] = acc[mt][nt][i];
+            } else {
+              double v = a.alpha * acc[mt][nt][i];
+              if (a.beta != 0.0) v += a.beta * a.Cin[r + c * a.ldcin];
+              a.C[r + c * a.ldc] = v;
+            }
+          }
+        }
+  }
+}
+
+__global__ void ws_reduce_kernel(int64_t M, int64_t N, int splits, const double* part, int64_t part_ld,
+                                 int64_t part_stride, double alpha, double beta, const double* Cin, int64_t ldcin,
+                                 double* C, int64_t ldc, int lower, int64_t diag_off) {
+  const int64_t total = M * N;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = idx % M, c = idx / M;
+    if (lower && r + diag_off < c) continue;
+    double s = 0.0;
+    for (int z = 0; z < splits; ++z) s += part[z * part_stride + r + c * part_ld];
+    double v = alpha * s;
+    if (beta != 0.0) v += beta * Cin[r + c * ldcin];
+    C[r + c * ldc] = v;
+  }
+}
+
+template <int BM, int BN, int CWM, int CWN, int OPB>
+static cudaError_t launch(WsArgs& a, cudaStream_t st) {
+  using C = Cfg<BM, BN>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(ws_kernel<BM, BN, CWM, CWN, OPB>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  a.tiles_m = (int)((a.M + BM - 1) / BM);
+  a.tiles_n = (int)((a.N + BN - 1) / BN);
+  if (a.tri && BM != BN) a.tri = 0;
+  const int64_t tiles = a.tri ? (int64_t)a.tiles_m * (a.tiles_m + 1) / 2 : (int64_t)a.tiles_m * a.tiles_n;
+  a.units = tiles * a.splits;
+  int64_t grid = a.units < kNumSMsB200 ? a.units : kNumSMsB200;
+  if (grid < 1) return cudaSuccess;
+  ws_kernel<BM, BN, CWM, CWN, OPB><<<(unsigned)grid, (CWM * CWN + NPW) * 32, C::SMEM, st>>>(a);
+  count_launches(1);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || a.splits == 1) return e;
+  int64_t total = a.M * a.N;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 16 * kNumSMsB200) blocks = 16 * kNumSMsB200;
+  ws_reduce_kernel<<<blocks, 256, 0, st>>>(a.M, a.N, a.splits, a.part, a.part_ld, a.part_stride, a.alpha, a.beta,
+                                           a.Cin, a.ldcin, a.C, a.ldc, a.lower, a.diag_off);
+  count_launches(1);
+  return cudaGetLastError();
+}
+
+static bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
+
+}  // namespace ws
+
+// C = alpha * sum_seg A_seg op(B_seg) + beta * Cin with op(A) = A (m-inner); tile 128x128 (wide N) or
+// 128x64 (N <= 64).  Same semantics as gemm() for opA == OP_N.
+cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
+  if (g.M <= 0 || g.N <= 0) return cudaSuccess;
+  ws::WsArgs a{};
+  a.M = g.M; a.N = g.N; a.opb = opB; a.nseg = g.nseg;
+  bool v16 = true;
+  for (int i = 0; i < 2; ++i) {
+    a.A[i] = g.A[i]; a.B[i] = g.B[i]; a.lda[i] = g.lda[i]; a.ldb[i] = g.ldb[i]; a.K[i] = g.K[i];
+    if (i < g.nseg) v16 = v16 && ws::al16(g.A[i]) && ws::al16(g.B[i]) && !(g.lda[i] & 1) && !(g.ldb[i] & 1);
+  }
+  a.vec16 = v16;
+  a.symm = 0;
+  a.alpha = g.alpha; a.beta = g.beta; a.Cin = g.Cin; a.ldcin = g.ldcin; a.C = g.C; a.ldc = g.ldc;
+  a.lower = g.lower; a.diag_off = g.diag_off; a.tri = g.tri;
+  a.splits = g.splits < 1 ? 1 : g.splits;
+  a.part = g.part; a.part_ld = g.part_ld; a.part_stride = g.part_stride;
+  if (g.N <= 64) {
+    return opB == OP_T ? ws::launch<128, 64, 4, 2, OP_T>(a, st) : ws::launch<128, 64, 4, 2, OP_N>(a, st);
+  }
+  return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
+}
+
+// X = Asym W on the warp-specialized engine (row strip + transposed column strip per row block).
+cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
+                    int64_t ldx, double* part, int64_t part_elems, cudaStream_t st) {
+  if (m <= 0 || w <= 0) return cudaSuccess;
+  ws::WsArgs a{};
+  a.M = m; a.N = w; a.opb = OP_N; a.nseg = 1; a.symm = 1;
+  a.A[0] = A; a.B[0] = W; a.lda[0] = lda; a.ldb[0] = ldw; a.K[0] = m;
+  a.vec16 = ws::al16(A) && ws::al16(W) && !(lda & 1) && !(ldw & 1);
+  a.alpha = 1.0; a.beta = 0.0; a.C = X; a.ldc = ldx;
+  // split the strip so that the persistent grid has >= ~3 units per CTA
+  const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
+  int64_t sp = (3 * kNumSMsB200 + rows - 1) / rows;
+  const int64_t maxs = (m + 1023) / 1024;
+  if (sp > maxs) sp = maxs;
+  if (sp > 32) sp = 32;
+  if (sp * m * w > part_elems) sp = part_elems / (m * w);
+  if (sp < 1) sp = 1;
+  a.splits = (int)sp;
+  a.part = part; a.part_ld = m; a.part_stride = m * w;
+  return ws::launch<128, 64, 4, 2, OP_N>(a, st);
+}
+
+}  // namespace trid
