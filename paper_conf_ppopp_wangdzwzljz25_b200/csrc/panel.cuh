@@ -11,6 +11,12 @@ size_t panel_red_bytes(int w);
 cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
                      int64_t ldy, double* red, unsigned* bar, cudaStream_t st);
 
+// Register-resident, cluster-reduced panel QR (panel_reg.cu) for w in {16, 32, 64}, m <= 36864.
+bool panel_reg_supported(int64_t m, int w);
+size_t panel_reg_gpart_bytes(int w);
+cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
+                         int64_t ldy, double* gpart, unsigned* bar, cudaStream_t st);
+
 // Bulge chasing (see bulge.cu).
 int bc_ldab(int64_t n, int b);
 int64_t bc_total_steps(int64_t n, int b);

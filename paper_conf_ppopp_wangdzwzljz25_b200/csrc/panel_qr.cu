@@ -13,6 +13,8 @@
 #include "panel.cuh"
 #include "prof.cuh"
 
+#include <stdlib.h>
+
 namespace trid {
 
 constexpr int PQ_NT = 256;
@@ -32,7 +34,19 @@ struct PanelArgs {
   unsigned* bar;
   int rows;      // rows per CTA
   int smem_ld;   // > 0: rows staged in shared memory with this leading dimension
+  int t_smem;    // 1: CTA 0 keeps T in shared memory (w x w) and writes it out at the end
+  long long* trace;   // debug (TRID_PANEL_TRACE): %globaltimer per column phase, CTAs 0 and G-1
 };
+__device__ __forceinline__ long long pq_gtimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define PQ_TRACE(k)                                                                               \
+  do {                                                                                            \
+    if (a.trace && tid == 0 && (g == 0 || g == G - 1) && t < 256)                                 \
+      a.trace[((g == 0 ? 0 : 1) * 256 + t) * 8 + (k)] = pq_gtimer();                              \
+  } while (0)
 
 __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
   extern __shared__ __align__(16) double sm[];
@@ -63,10 +77,14 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
   double* wv = tot + RS;        // w: update vector (j > t) / v_t^T v_q (q < t)
   double* tmp = wv + w;         // H*RS <= PQ_NT partial totals
   double* hs = tmp + PQ_NT;     // beta, tau, scale
+  double* Ts = hs + 8;          // w x w (only if t_smem; CTA 0)
+  double* Tw = a.t_smem ? Ts : a.T;
+  const int64_t ldT = a.t_smem ? w : a.ldt;
   __syncthreads();
 
   unsigned epoch = 0;
   for (int t = 0; t < a.kk; ++t) {
+    PQ_TRACE(0);
     double* red = a.red + (size_t)(t & 1) * G * RS;
     // ---- partial Gram row: slot j = sum_{r > t, r owned} P(r,t) P(r,j);  slot w+j = P(t,j) (owner)
     const int i0 = (int)((t + 1 - rlo) > 0 ? (t + 1 - rlo) : 0);
@@ -80,7 +98,9 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
     }
     const bool owner = (t >= rlo) && (t < rlo + nr);
     for (int j = tid; j < w; j += PQ_NT) red[(size_t)g * RS + w + j] = owner ? L[(size_t)j * ldl + (t - rlo)] : 0.0;
+    PQ_TRACE(1);
     grid_barrier(a.bar, (unsigned)G, epoch);
+    PQ_TRACE(2);
     // ---- distributed reduction: CTA g sums slots s = g, g+G, ... over all CTAs in a fixed order
     {
       const double* src = a.red + (size_t)(t & 1) * G * RS;
@@ -99,9 +119,12 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
         __syncthreads();
       }
     }
+    PQ_TRACE(3);
     grid_barrier(a.bar, (unsigned)G, epoch);
+    PQ_TRACE(4);
     for (int s = tid; s < RS; s += PQ_NT) tot[s] = __ldcg(a.tot + (size_t)(t & 1) * RS + s);
     __syncthreads();
+    PQ_TRACE(5);
     // ---- reflector (R1), update vector, T inner products
     const House h = make_house(tot[w + t], tot[t]);
     for (int j = tid; j < w; j += PQ_NT) {
@@ -122,28 +145,34 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
         for (int j = t + 1; j < w; ++j) L[(size_t)j * ldl + i] -= h.tau * wv[j];
       }
     }
+    PQ_TRACE(6);
     // ---- T(:, t) (CTA 0): T(t,t) = tau; T(0:t,t) = -tau T(0:t,0:t) (V^T v_t); zeros below
     if (g == 0) {
       for (int q = tid; q < w; q += PQ_NT) {
         double v = 0.0;
         if (q < t) {
           double s = 0.0;
-          for (int p = q; p < t; ++p) s += a.T[q + (int64_t)p * a.ldt] * wv[p];
+          for (int p = q; p < t; ++p) s += Tw[q + (int64_t)p * ldT] * wv[p];
           v = -h.tau * s;
         } else if (q == t) {
           v = h.tau;
         }
-        a.T[q + (int64_t)t * a.ldt] = v;
+        Tw[q + (int64_t)t * ldT] = v;
       }
       if (tid == 0) a.tau[t] = h.tau;
     }
     __syncthreads();
+    PQ_TRACE(7);
   }
-  // zero the unused columns of T (kk < w)
+  // zero the unused columns of T (kk < w); write T out if it lived in shared memory
   if (g == 0) {
     for (int idx = tid; idx < (w - a.kk) * w; idx += PQ_NT) {
       const int q = idx % w, c = a.kk + idx / w;
-      a.T[q + (int64_t)c * a.ldt] = 0.0;
+      Tw[q + (int64_t)c * ldT] = 0.0;
+    }
+    if (a.t_smem) {
+      __syncthreads();
+      for (int idx = tid; idx < w * w; idx += PQ_NT) a.T[(idx % w) + (int64_t)(idx / w) * a.ldt] = Ts[idx];
     }
   }
   // ---- write back (R above, V below) and explicit Y = V (unit diagonal, zeros above)
@@ -168,17 +197,26 @@ static int panel_grid(int64_t m) {
   return (int)G;
 }
 
-size_t panel_red_bytes(int w) { return sizeof(double) * (2 * (size_t)kNumSMsB200 * 2 * (size_t)w + 2 * 2 * (size_t)w); }
+size_t panel_red_bytes(int w) {
+  return sizeof(double) * (2 * (size_t)kNumSMsB200 * 2 * (size_t)w + 2 * 2 * (size_t)w) + sizeof(long long) * 2 * 256 * 8;
+}
 
 cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
                      int64_t ldy, double* red, unsigned* bar, cudaStream_t st) {
   if (m <= 0 || w <= 0) return cudaSuccess;
+  if (panel_reg_supported(m, w) && !getenv("TRID_PANEL_SMEM"))
+    return panel_qr_reg(m, w, P, ldp, tau, T, ldt, Y, ldy, red, bar, st);
   const int G = panel_grid(m);
   PanelArgs a;
   a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);
   a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.red = red; a.tot = red + 2 * (size_t)kNumSMsB200 * 2 * w; a.bar = bar;
   a.rows = (int)((m + G - 1) / G);
+  {
+    static const char* tr = getenv("TRID_PANEL_TRACE");   // "m": trace the panel with this many rows
+    a.trace = (tr && atoll(tr) == m) ? (long long*)(red + 2 * (size_t)kNumSMsB200 * 2 * w + 2 * 2 * (size_t)w) : nullptr;
+  }
   const size_t scr = sizeof(double) * (size_t)(2 * w + w + PQ_NT + 8);
+  const size_t tsz = sizeof(double) * (size_t)w * w;
   const size_t full = sizeof(double) * (size_t)a.rows * w + scr;
   const size_t kMaxSmem = 227 * 1024;
   size_t smem;
@@ -189,6 +227,8 @@ cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, doub
     a.smem_ld = 0;
     smem = scr;
   }
+  a.t_smem = smem + tsz <= kMaxSmem ? 1 : 0;
+  if (a.t_smem) smem += tsz;
   static bool attr_done = false;
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(panel_qr_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);

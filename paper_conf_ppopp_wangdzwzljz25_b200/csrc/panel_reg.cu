@@ -1,0 +1,304 @@
+// panel_reg.cu — register-resident, cluster-reduced panel QR for DBBR (Alg. 1 line 5)
+// with the dlarft T factor and the explicit Y = V.  Fast path for w in {16, 32, 64}.
+//
+// Layout: G CTAs (a multiple of 8, launched as clusters of 8) own contiguous row blocks of the m x w
+// panel; inside a CTA, warp wi owns columns [wi*CPW, (wi+1)*CPW) and lane l owns rows l, l+32, ...
+// so the whole panel lives in registers (RL x CPW doubles per thread).  Column t costs:
+//   1. every warp forms its slots of the Gram row  sum_{r>t} x_r P(r, j)  (x = column t below row t,
+//      broadcast through shared memory) with one transposed butterfly, plus the row-t values;
+//   2. cluster barrier; CTA rank c reduces slots c, c+8, ... over the 8 CTAs through DSMEM (fixed
+//      order) and writes the cluster partial to global memory;
+//   3. ONE grid barrier (release/acquire counter);
+//   4. every CTA sums the NC cluster partials in a fixed order -> identical beta/tau/w in all CTAs;
+//   5. register update P(r, j) -= tau w_j v_r, T column in CTA 0's shared memory.
+#include <cooperative_groups.h>
+
+#include "common.cuh"
+#include "panel.cuh"
+#include "prof.cuh"
+
+namespace trid {
+
+namespace cg = cooperative_groups;
+
+constexpr int PR_NT = 256;   // 8 warps
+constexpr int PR_CL = 4;     // cluster size (33 co-resident 4-CTA clusters at 1 CTA/SM on B200)
+constexpr int PR_MAXNC = 40; // max clusters
+constexpr int PR_RL = 8;     // rows per lane (rows per CTA <= 256)
+
+struct PanelRegArgs {
+  int64_t m;
+  int w, kk;
+  double* P;
+  int64_t ldp;
+  double* tau;
+  double* T;
+  int64_t ldt;
+  double* Y;
+  int64_t ldy;
+  double* gpart;     // 2 x NC x 2w cluster partials
+  unsigned* bar;     // grid barrier counter (zero at launch)
+  int rows;          // rows per CTA
+};
+
+template <int CPW>
+__global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_constant__ PanelRegArgs a) {
+  constexpr int W = 8 * CPW;
+  constexpr int RS = 2 * W;
+  extern __shared__ __align__(16) double sm[];
+  double* xs = sm;                    // rows of this CTA: column t (broadcast)
+  double* mypart = xs + 32 * PR_RL;   // 2 x RS   (double-buffered per column parity)
+  double* tot = mypart + 2 * RS;      // RS
+  double* Ts = tot + RS;              // W x W    (CTA 0)
+  cg::cluster_group cl = cg::this_cluster();
+  const int g = blockIdx.x, G = gridDim.x, NC = G / PR_CL;
+  const int crank = (int)cl.block_rank(), cid = g / PR_CL;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t rlo = (int64_t)g * a.rows;
+  const int nr = (int)((rlo + a.rows <= a.m) ? a.rows : (a.m > rlo ? a.m - rlo : 0));
+  const int j0 = warp * CPW;
+
+  double P[PR_RL][CPW];
+#pragma unroll
+  for (int q = 0; q < PR_RL; ++q) {
+    const int i = lane + 32 * q;
+#pragma unroll
+    for (int c = 0; c < CPW; ++c)
+      P[q][c] = (i < nr && j0 + c < a.w) ? a.P[(rlo + i) + (int64_t)(j0 + c) * a.ldp] : 0.0;
+  }
+  // column 0 -> xs
+  if (warp == 0) {
+#pragma unroll
+    for (int q = 0; q < PR_RL; ++q) xs[lane + 32 * q] = P[q][0];
+  }
+  unsigned epoch = 0;
+  __syncthreads();
+
+  for (int t = 0; t < a.kk; ++t) {
+    const int par = t & 1;
+    const int wt = t / CPW, ct = t % CPW;
+    // ---- 1. Gram slots of this warp's columns over rows > t, and row-t values
+    double acc[CPW];
+#pragma unroll
+    for (int c = 0; c < CPW; ++c) acc[c] = 0.0;
+    int qt = -1;   // this lane's q holding row t, if any
+#pragma unroll
+    for (int q = 0; q < PR_RL; ++q) {
+      const int64_t r = rlo + lane + 32 * q;
+      const double x = (r > t && lane + 32 * q < nr) ? xs[lane + 32 * q] : 0.0;
+      if (r == t && lane + 32 * q < nr) qt = q;
+#pragma unroll
+      for (int c = 0; c < CPW; ++c) acc[c] = fma(x, P[q][c], acc[c]);
+    }
+    // transposed butterfly: CPW values over 32 lanes
+    int qb = 0;
+#pragma unroll
+    for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
+      const bool up = (lane & o) != 0;
+#pragma unroll
+      for (int i = 0; i < K / 2; ++i) {
+        const double send = up ? acc[i] : acc[i + K / 2];
+        const double keep = up ? acc[i + K / 2] : acc[i];
+        acc[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+      }
+      if (up) qb += K / 2;
+    }
+    constexpr int LV = CPW >= 8 ? 3 : (CPW == 4 ? 2 : (CPW == 2 ? 1 : 0));
+    double f = acc[0];
+#pragma unroll
+    for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+    double* mp = mypart + par * RS;
+    if ((lane & ((32 >> LV) - 1)) == 0) mp[j0 + qb] = f;
+    // row-t values of this warp's columns (owner lane) or zero
+    {
+      const unsigned own = __ballot_sync(0xffffffffu, qt >= 0);
+      if (own) {
+        const int src = __ffs(own) - 1;
+#pragma unroll
+        for (int c = 0; c < CPW; ++c) {
+          double vv = 0.0;
+#pragma unroll
+          for (int q = 0; q < PR_RL; ++q)
+            if (q == qt) vv = P[q][c];
+          vv = __shfl_sync(0xffffffffu, vv, src);
+          if (lane == 0) mp[W + j0 + c] = vv;
+        }
+      } else if (lane < CPW) {
+        mp[W + j0 + lane] = 0.0;
+      }
+    }
+    // ---- 2. cluster reduction through DSMEM (fixed order over the 8 CTAs)
+    cl.sync();
+    {
+      // thread -> (slot s = crank + 8*k, member c): 8 lanes per slot
+      const int k = tid / PR_CL, c = tid % PR_CL;
+      const int s = crank + PR_CL * k;
+      double v = 0.0;
+      if (s < RS) {
+        const double* rp = cl.map_shared_rank(mypart + par * RS, c);
+        v = rp[s];
+      }
+#pragma unroll
+      for (int o = 1; o < PR_CL; o <<= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+      if (c == 0 && s < RS) __stcg(a.gpart + ((size_t)par * NC + cid) * RS + s, v);
+    }
+    // ---- 3. one grid barrier
+    __syncthreads();
+    epoch += 1;
+    if (tid == 0) {
+      asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar) : "memory");
+      const unsigned target = epoch * (unsigned)G;
+      while (ld_relaxed_u32(a.bar) < target) {
+      }
+      (void)ld_acquire_u32(a.bar);
+    }
+    __syncthreads();
+    // ---- 4. totals over the NC cluster partials, fixed order
+    for (int s = tid; s < RS; s += PR_NT) {
+      double vals[PR_MAXNC];
+#pragma unroll
+      for (int q = 0; q < PR_MAXNC; ++q) vals[q] = q < NC ? __ldcg(a.gpart + ((size_t)par * NC + q) * RS + s) : 0.0;
+      double v = vals[0];
+#pragma unroll
+      for (int q = 1; q < PR_MAXNC; ++q)
+        if (q < NC) v += vals[q];
+      tot[s] = v;
+    }
+    __syncthreads();
+    // ---- 5. reflector, update, T column
+    const House h = make_house(tot[W + t], tot[t]);
+#pragma unroll
+    for (int q = 0; q < PR_RL; ++q) {
+      const int i = lane + 32 * q;
+      const int64_t r = rlo + i;
+      if (i >= nr || r < t) continue;
+      const double vr = r > t ? h.scale * xs[i] : 1.0;
+#pragma unroll
+      for (int c = 0; c < CPW; ++c) {
+        const int j = j0 + c;
+        if (j > t) {
+          const double wj = tot[W + j] + h.scale * tot[j];
+          P[q][c] = fma(-h.tau * wj, vr, P[q][c]);
+        } else if (j == t) {
+          P[q][c] = r > t ? vr : h.beta;
+        }
+      }
+    }
+    if (g == 0) {
+      for (int q2 = tid; q2 < W; q2 += PR_NT) {
+        double v = 0.0;
+        if (q2 < t) {
+          double sacc = 0.0;
+          for (int p = q2; p < t; ++p) sacc += Ts[q2 + p * W] * (tot[W + p] + h.scale * tot[p]);
+          v = -h.tau * sacc;
+        } else if (q2 == t) {
+          v = h.tau;
+        }
+        Ts[q2 + t * W] = v;
+      }
+      if (tid == 0) a.tau[t] = h.tau;
+    }
+    __syncthreads();   // everyone is done with xs / tot of column t
+    // next column -> xs
+    if (t + 1 < a.kk && warp == (t + 1) / CPW) {
+      const int cn = (t + 1) % CPW;
+#pragma unroll
+      for (int q = 0; q < PR_RL; ++q) {
+        double v = 0.0;
+#pragma unroll
+        for (int c = 0; c < CPW; ++c)
+          if (c == cn) v = P[q][c];
+        xs[lane + 32 * q] = v;
+      }
+    }
+    __syncthreads();
+  }
+  // ---- write back R/V, explicit Y, T
+#pragma unroll
+  for (int q = 0; q < PR_RL; ++q) {
+    const int i = lane + 32 * q;
+    if (i >= nr) continue;
+    const int64_t r = rlo + i;
+#pragma unroll
+    for (int c = 0; c < CPW; ++c) {
+      const int j = j0 + c;
+      if (j < a.w) a.P[r + (int64_t)j * a.ldp] = P[q][c];
+      if (j < a.kk) a.Y[r + (int64_t)j * a.ldy] = r > j ? P[q][c] : (r == j ? 1.0 : 0.0);
+    }
+  }
+  if (g == 0) {
+    for (int idx = tid; idx < W * W; idx += PR_NT) {
+      const int q2 = idx % W, c = idx / W;
+      a.T[q2 + (int64_t)c * a.ldt] = (c < a.kk) ? Ts[q2 + c * W] : 0.0;
+    }
+  }
+  cl.sync();   // no CTA leaves while a cluster peer may still read its shared memory
+}
+
+size_t panel_reg_gpart_bytes(int w) { return sizeof(double) * 2 * PR_MAXNC * 2 * (size_t)w; }
+
+bool panel_reg_supported(int64_t m, int w) {
+  // 33 co-resident clusters of 4 (GPC packing on B200, 1 CTA/SM) x 256 rows per CTA
+  return (w == 16 || w == 32 || w == 64) && m <= (int64_t)PR_CL * 33 * 32 * PR_RL && m >= 1;
+}
+
+cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
+                         int64_t ldy, double* gpart, unsigned* bar, cudaStream_t st) {
+  PanelRegArgs a;
+  a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);
+  a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.gpart = gpart; a.bar = bar;
+  const size_t smem = sizeof(double) * (size_t)(32 * PR_RL + 2 * 2 * w + 2 * w + w * w);
+  // co-resident clusters of 8 (a cluster must fit in one GPC): query once per kernel instantiation
+  static int max_clusters[3] = {0, 0, 0};
+  const int wi = w == 16 ? 0 : (w == 32 ? 1 : 2);
+  const void* fn = w == 16 ? (const void*)panel_reg_kernel<2>
+                            : (w == 32 ? (const void*)panel_reg_kernel<4> : (const void*)panel_reg_kernel<8>);
+  if (!max_clusters[wi]) {
+    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaLaunchConfig_t q = {};
+    q.gridDim = dim3(PR_CL * PR_MAXNC);
+    q.blockDim = dim3(PR_NT);
+    q.dynamicSmemBytes = smem;
+    cudaLaunchAttribute qa[1];
+    qa[0].id = cudaLaunchAttributeClusterDimension;
+    qa[0].val.clusterDim.x = PR_CL;
+    qa[0].val.clusterDim.y = 1;
+    qa[0].val.clusterDim.z = 1;
+    q.attrs = qa;
+    q.numAttrs = 1;
+    int nc = 0;
+    if (cudaOccupancyMaxActiveClusters(&nc, fn, &q) != cudaSuccess || nc < 1) nc = 1;
+    max_clusters[wi] = nc > PR_MAXNC ? PR_MAXNC : nc;
+  }
+  // as few rows per CTA as possible within the co-resident clusters
+  int64_t G = (m + 63) / 64;
+  G = (G + PR_CL - 1) / PR_CL * PR_CL;
+  if (G > (int64_t)PR_CL * max_clusters[wi]) G = (int64_t)PR_CL * max_clusters[wi];
+  if (G < PR_CL) G = PR_CL;
+  a.rows = (int)((m + G - 1) / G);
+  if (a.rows > 32 * PR_RL) return cudaErrorInvalidConfiguration;   // caller checks panel_reg_supported
+  cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)G);
+  cfg.blockDim = dim3(PR_NT);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = PR_CL;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeCooperative;
+  attr[1].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 2;
+  count_launches(1);
+  switch (w) {
+    case 16: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<2>, a);
+    case 32: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<4>, a);
+    default: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<8>, a);
+  }
+}
+
+}  // namespace trid
