@@ -76,7 +76,7 @@ int64_t max_symm_part(int64_t n, int b) {
   for (int64_t j = 0; j + b + 1 < n; j += b) {
     const int64_t m = n - j - b;
     const int64_t kk = m < b ? m : b;
-    const int64_t e = symm_part_elems(m, kk);
+    const int64_t e = symm_ws_part_elems(m, kk);
     if (e > best) best = e;
   }
   return best;
@@ -449,7 +449,7 @@ int trid_zy_bufsize(int64_t m, int w, size_t* dwork_bytes) {
   if (m < 0) return -1;
   if (w < 1) return -2;
   if (!dwork_bytes) return -3;
-  int64_t pe = symm_part_elems(m, w);
+  int64_t pe = symm_ws_part_elems(m, w);
   const int64_t tn = (int64_t)32 * w * w;
   if (pe < tn) pe = tn;
   *dwork_bytes = align256(sizeof(double) * (size_t)m * w) + align256(sizeof(double) * (size_t)w * w) +
@@ -476,7 +476,7 @@ int trid_zy(int64_t m, int w, const double* A, int64_t lda, const double* W, int
   Carver c(dwork);
   double* X = c.take<double>((size_t)m * w);
   double* S = c.take<double>((size_t)w * w);
-  int64_t pe = symm_part_elems(m, w);
+  int64_t pe = symm_ws_part_elems(m, w);
   if (pe < (int64_t)32 * w * w) pe = (int64_t)32 * w * w;
   double* part = c.take<double>((size_t)pe);
   // Eq. (1) with no earlier panels: Y and Z of this call are separate buffers (ldy, ldz)

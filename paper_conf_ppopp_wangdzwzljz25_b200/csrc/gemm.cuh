@@ -52,6 +52,8 @@ int64_t symm_part_elems(int64_t m, int64_t w);
 
 // Warp-specialized persistent engine (gemm_ws.cu): op(A) = A only; tiles 128x128 (N > 64) / 128x64.
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
+int64_t symm_ws_splits(int64_t m, int64_t w);
+int64_t symm_ws_part_elems(int64_t m, int64_t w);
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
                     int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);
 

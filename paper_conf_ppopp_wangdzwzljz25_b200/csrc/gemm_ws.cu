@@ -16,6 +16,8 @@
 #include "gemm.cuh"
 #include "prof.cuh"
 
+#include <stdlib.h>
+
 namespace trid {
 
 namespace ws {
@@ -461,6 +463,24 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 
+// Strip splits of the SYMM: the persistent grid runs >= ~8 waves of units (tail imbalance <~ 6%);
+// env TRID_SYMM_WAVES overrides (tuning).
+int64_t symm_ws_splits(int64_t m, int64_t w) {
+  const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
+  static const char* wv = getenv("TRID_SYMM_WAVES");
+  const int64_t waves = wv ? atoll(wv) : 8;
+  int64_t sp = (waves * kNumSMsB200 + rows - 1) / rows;
+  const int64_t maxs = (m + 511) / 512;
+  if (sp > maxs) sp = maxs;
+  if (sp > 32) sp = 32;
+  if (sp < 1) sp = 1;
+  return sp;
+}
+int64_t symm_ws_part_elems(int64_t m, int64_t w) {
+  const int64_t sp = symm_ws_splits(m, w);
+  return sp > 1 ? sp * m * w : 0;
+}
+
 // X = Asym W on the warp-specialized engine (row strip + transposed column strip per row block).
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
                     int64_t ldx, double* part, int64_t part_elems, cudaStream_t st) {
@@ -470,12 +490,7 @@ cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const do
   a.A[0] = A; a.B[0] = W; a.lda[0] = lda; a.ldb[0] = ldw; a.K[0] = m;
   a.vec16 = ws::al16(A) && ws::al16(W) && !(lda & 1) && !(ldw & 1);
   a.alpha = 1.0; a.beta = 0.0; a.C = X; a.ldc = ldx;
-  // split the strip so that the persistent grid has >= ~3 units per CTA
-  const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
-  int64_t sp = (3 * kNumSMsB200 + rows - 1) / rows;
-  const int64_t maxs = (m + 1023) / 1024;
-  if (sp > maxs) sp = maxs;
-  if (sp > 32) sp = 32;
+  int64_t sp = symm_ws_splits(m, w);
   if (sp * m * w > part_elems) sp = part_elems / (m * w);
   if (sp < 1) sp = 1;
   a.splits = (int)sp;
