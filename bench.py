@@ -7,8 +7,9 @@ Inputs live in HBM before the timed region; the 8.6 GB matrix is far larger than
 explicit flush is needed between steps.
 
 Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--n N --b B ...]
-Multi-GPU (torchrun): every rank runs an independent replica (stage 1 sharding is future work, see
-DESIGN.md); time is the max over ranks; value is the whole-job aggregate.
+Multi-GPU (torchrun): stage 1 is sharded over the ranks (block-cyclic column blocks, per-panel NCCL
+broadcast + all-reduce), the band is gathered to rank 0 and stage 2 runs there; the
+matrix is the same for every N (strong scaling); time is the max over ranks.
 """
 from __future__ import annotations
 
@@ -219,20 +220,52 @@ def main():
     if args.n or args.b or args.k >= 0:
         cfg["desc"] = f"n={n} random symmetric FP64, b={b}, nb={nb}, k={k}"
 
-    A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
-    A = torch.empty_like(A0)
-    nbytes, v2len, t2len = trid.sytrd_2stage_bufsize(n, b, nb, k)
-    work = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
     want = not args.eig_only
-    out = (torch.empty(n, dtype=torch.float64, device=dev), torch.empty(max(n - 1, 1), dtype=torch.float64, device=dev),
-           torch.empty(n, dtype=torch.float64, device=dev),
-           torch.empty(max(v2len, 1), dtype=torch.float64, device=dev) if want else None,
-           torch.empty(max(t2len, 1), dtype=torch.float64, device=dev) if want else None)
     stream = torch.cuda.current_stream()
+    if ws == 1:
+        A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
+        A = torch.empty_like(A0)
+        nbytes, v2len, t2len = trid.sytrd_2stage_bufsize(n, b, nb, k)
+        work = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
+        out = (torch.empty(n, dtype=torch.float64, device=dev),
+               torch.empty(max(n - 1, 1), dtype=torch.float64, device=dev),
+               torch.empty(n, dtype=torch.float64, device=dev),
+               torch.empty(max(v2len, 1), dtype=torch.float64, device=dev) if want else None,
+               torch.empty(max(t2len, 1), dtype=torch.float64, device=dev) if want else None)
+
+        def run(Ain):
+            trid.sytrd_2stage(Ain, b, nb=nb, k=k, want_vectors=want, work=work, out=out)
+            return out[0], out[1], out[2]
+    else:
+        # multi-GPU: stage 1 sharded over the ranks (block-cyclic columns, NCCL per panel), band gathered to
+        # rank 0, stage 2 on rank 0 (one chase is one dependency chain).  Same matrix as N = 1: strong scaling.
+        comm = trid.comm_nccl()
+        cols = trid_gen.block_cyclic_columns(n, b, ws, rank)
+        A0 = trid_gen.random_symmetric_rows(n, cfg["seed"], cols, device=dev)
+        A = torch.empty_like(A0)
+        work = torch.empty(max(trid.sbr_dbbr_mg_bufsize(n, b, nb, k, ws, rank), 256), dtype=torch.uint8, device=dev)
+        tau1 = torch.empty(n, dtype=torch.float64, device=dev)
+        AB = torch.empty((n, b + 1), dtype=torch.float64, device=dev)
+        bc_out = None
+        if rank == 0:
+            bcb, v2len, t2len = trid.bulge_chase_bufsize(n, b)
+            bc_work = torch.empty(max(bcb, 256), dtype=torch.uint8, device=dev)
+            bc_out = (torch.empty(n, dtype=torch.float64, device=dev),
+                      torch.empty(max(n - 1, 1), dtype=torch.float64, device=dev),
+                      torch.empty(max(v2len, 1), dtype=torch.float64, device=dev) if want else None,
+                      torch.empty(max(t2len, 1), dtype=torch.float64, device=dev) if want else None)
+
+        def run(Ain):
+            trid.sbr_dbbr_mg(comm, Ain, n, b, nb=nb, k=k, tau1=tau1, work=work)
+            trid.band_gather(comm, Ain, n, b, root=0, AB=AB)
+            if rank == 0:
+                trid.bulge_chase_band(AB, n, b, want_vectors=want, work=bc_work, out=bc_out)
+                return bc_out[0], bc_out[1], tau1
+            return None
 
     def step():
         A.copy_(A0)
-        trid.sytrd_2stage(A, b, nb=nb, k=k, want_vectors=want, work=work, out=out)
+        run(A)
 
     for _ in range(args.warmup):
         step()
@@ -261,14 +294,14 @@ def main():
         ms = float(t.item())
 
     flop = 4.0 * n ** 3 / 3.0
-    value = ws * flop * args.steps / (ms * 1e-3) / 1e12
+    value = flop * args.steps / (ms * 1e-3) / 1e12   # one matrix per step for every N (strong scaling)
     per = {c: (v[0] / args.steps, v[1] / args.steps) for c, v in stages.items()}
     t_bc = per["bulge_chase"][0]
     t_sbr = sum(v[0] for c, v in per.items() if c != "bulge_chase")
 
     # roofline: the dominant DBBR contraction (largest time share) against the measured FP64 DMMA peak
     fl = dbbr_flops(n, b, k)
-    cand = {"symm": (fl["symm"], stages["symm"]), "syr2k": (fl["syr2k"], stages["syr2k"])}
+    cand = {"symm": (fl["symm"], per["symm"]), "syr2k": (fl["syr2k"], per["syr2k"])}
     dom = max(cand, key=lambda c: cand[c][1][0])
     dflops, (dms, dcalls) = cand[dom]
     achieved = (dflops / max(dcalls, 1)) / ((dms / max(dcalls, 1)) * 1e-3) / 1e12 if dcalls else 0.0
@@ -286,10 +319,10 @@ def main():
     line = {
         "metric": "FP64 TFLOPs (4n^3/3) full tridiag at n=32768, SBR/BC time split, 1/2/4/8 GPU",
         "value": round(value, 4), "unit": "TFLOP/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "strong" if ws > 1 else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": cfg["desc"], "n": n, "b": b, "nb": nb, "k": k, "seed": cfg["seed"],
-                   "parallelism": "replicas" if ws > 1 else "single-gpu",
+                   "parallelism": f"sbr-colblock-cyclic-x{ws}+bc-rank0" if ws > 1 else "single-gpu",
                    "l2": "inputs larger than L2 (n^2*8 B matrix restored from a resident copy each step)",
                    "vectors": "stored (V1 in A, tau1, V2, tau2)" if want else "eigenvalues-only"},
         "t_sbr_ms": round(t_sbr, 3), "t_bc_ms": round(t_bc, 3),
@@ -312,7 +345,7 @@ def main():
 
     # ---- end to end through the public API with host buffers (pinned H2D of A, D2H of d, e, tau1)
     if not args.no_e2e and args.e2e_steps > 0:
-        Ah = torch.empty((n, n), dtype=torch.float64, pin_memory=True)
+        Ah = torch.empty(A0.shape, dtype=torch.float64, pin_memory=True)
         Ah.copy_(A0)
         dh = torch.empty(n, dtype=torch.float64, pin_memory=True)
         eh = torch.empty(max(n - 1, 1), dtype=torch.float64, pin_memory=True)
@@ -324,10 +357,11 @@ def main():
         e0.record(stream)
         for _ in range(args.e2e_steps):
             A.copy_(Ah, non_blocking=True)
-            trid.sytrd_2stage(A, b, nb=nb, k=k, want_vectors=want, work=work, out=out)
-            dh.copy_(out[0], non_blocking=True)
-            eh.copy_(out[1], non_blocking=True)
-            th.copy_(out[2], non_blocking=True)
+            res = run(A)
+            if res is not None:
+                dh.copy_(res[0], non_blocking=True)
+                eh.copy_(res[1][: max(n - 1, 1)], non_blocking=True)
+                th.copy_(res[2], non_blocking=True)
         e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
@@ -335,8 +369,8 @@ def main():
             t = torch.tensor([ems], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
-        line["e2e"] = {"value": round(ws * flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
-                       "h2d_bytes_per_step": 8 * n * n, "d2h_bytes_per_step": 8 * (n + (n - 1) + n),
+        line["e2e"] = {"value": round(flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
+                       "h2d_bytes_per_step": 8 * A0.numel() * ws, "d2h_bytes_per_step": 8 * (n + (n - 1) + n),
                        "note": "V1/V2 reflectors stay device-resident for the back transformation"}
         del Ah
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:

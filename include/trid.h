@@ -39,7 +39,7 @@ extern "C" {
 enum {
   TRID_SUCCESS = 0,
   TRID_ERR_CUDA = 1,        /* a CUDA runtime call or launch failed */
-  TRID_ERR_NCCL = 2,        /* reserved for the multi-GPU stage-1 path */
+  TRID_ERR_NCCL = 2,        /* an NCCL call failed (multi-GPU stage 1); see trid_last_error_string() */
   TRID_ERR_WORKSPACE = 3,   /* dwork_bytes smaller than the *_bufsize result */
   TRID_ERR_UNSUPPORTED = 4  /* a valid but unsupported configuration (e.g. b > TRID_MAX_B) */
 };
@@ -100,6 +100,45 @@ int trid_bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, 
 int trid_sytrd_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* d, double* e,
                       double* tau1, double* V2, double* tau2, void* dwork, size_t dwork_bytes,
                       cudaStream_t stream);
+
+/* ---- stage 2 from LAPACK lower band storage (dsbtrd-style input): AB[(i-j) + j*ldab] = B(i, j) for
+ * 0 <= i-j <= b, ldab >= b+1 (the layout trid_band_gather produces).  Otherwise as trid_bulge_chase. */
+int trid_bulge_chase_band(int64_t n, int b, const double* AB, int64_t ldab, double* d, double* e, double* V2,
+                          double* tau2, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+/* ---- multi-GPU stage 1 ------------------------------------------------
+ * One rank per GPU (one process each, NCCL), or — for testing the sharded arithmetic on one device —
+ * g "local" virtual ranks in one process, each driven from its own host thread with its own stream.
+ * Layout: the n x n matrix is 1D block-cyclic over column blocks of width colblock = b: global column
+ * block B lives on rank B % g; rank q stores its columns contiguously in order (local column x) as
+ * full-height columns, A_local(i, x) = A(i, c(x)), lda_local >= n; only entries with i >= c(x) (the
+ * lower triangle) are referenced.  trid_mg_local_cols gives the local column count.
+ * Communicator calls are collective over the ranks; a failing rank leaves the others waiting (as NCCL). */
+typedef struct trid_comm* trid_comm_t;
+/* 128-byte NCCL unique id (call on one rank, distribute out of band, e.g. torch.distributed.broadcast). */
+int trid_comm_unique_id(unsigned char id[128]);
+/* NCCL communicator (libnccl.so.2 resolved at run time; the current CUDA device is the rank's GPU). */
+int trid_comm_init_nccl(const unsigned char id[128], int nranks, int rank, trid_comm_t* comm);
+/* nranks (<= 16) virtual ranks sharing this process and device: comms[q] is rank q. */
+int trid_comm_init_local(int nranks, trid_comm_t* comms);
+int trid_comm_destroy(trid_comm_t comm);
+int trid_comm_size(trid_comm_t comm);
+int trid_comm_rank(trid_comm_t comm);
+/* number of columns rank `rank` of `nranks` stores (block-cyclic, blocks of colblock); -1 on bad args */
+int64_t trid_mg_local_cols(int64_t n, int colblock, int nranks, int rank);
+int trid_sbr_dbbr_mg_bufsize(int64_t n, int b, int nb, int k, int nranks, int rank, size_t* dwork_bytes);
+/* Alg. 1 with the per-panel exchange of SURVEY 8(e): the panel owner's [Y_p | T | tau] is broadcast,
+ * the partial X = A_blk W_p over each rank's stored entries is all-reduced (sum), the Z builder runs
+ * redundantly, the next-panel update on the next panel's owner, the syr2k on every rank's own columns.
+ * Out: as trid_sbr_dbbr, in the block-cyclic layout (band + SBR vectors in each owner's columns);
+ * tau1[n] complete on every rank.  colblock must equal b. */
+int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A_local, int64_t lda_local, int colblock, int b, int nb,
+                     int k, double* tau1, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+/* Gather the band (diagonal + b sub-diagonals) to `root` in LAPACK lower band storage AB (ldab >= b+1,
+ * ldab x n doubles, a device buffer on EVERY rank — it is the send buffer; only root's holds the band on
+ * return).  Collective (a sum-reduce of disjoint column sets). */
+int trid_band_gather(trid_comm_t comm, int64_t n, int b, const double* A_local, int64_t lda_local, int colblock,
+                     int root, double* AB, int64_t ldab, cudaStream_t stream);
 
 /* ---- profiling (host-side, optional; used by bench.py) ------------------------------------------
  * trid_profile_begin(): from now on every hot-path stage launched by the library is bracketed by a pair

@@ -60,6 +60,22 @@ def lib():
         L.trid_syr2k_lower.argtypes = [_I64, _I64, _P, _I64, _P, _I64, _P, _I64, _P]
         L.trid_zy_bufsize.argtypes = [_I64, _INT, ctypes.POINTER(_SZ)]
         L.trid_zy.argtypes = [_I64, _INT, _P, _I64, _P, _I64, _P, _I64, _P, _I64, _P, _SZ, _P]
+        L.trid_bulge_chase_band.argtypes = [_I64, _INT, _P, _I64, _P, _P, _P, _P, _P, _SZ, _P]
+        L.trid_comm_unique_id.argtypes = [ctypes.c_char_p]
+        L.trid_comm_init_nccl.argtypes = [ctypes.c_char_p, _INT, _INT, ctypes.POINTER(_P)]
+        L.trid_comm_init_local.argtypes = [_INT, ctypes.POINTER(_P)]
+        L.trid_comm_destroy.argtypes = [_P]
+        L.trid_comm_size.argtypes = [_P]
+        L.trid_comm_rank.argtypes = [_P]
+        L.trid_mg_local_cols.restype = _I64
+        L.trid_mg_local_cols.argtypes = [_I64, _INT, _INT, _INT]
+        L.trid_sbr_dbbr_mg_bufsize.argtypes = [_I64, _INT, _INT, _INT, _INT, _INT, ctypes.POINTER(_SZ)]
+        L.trid_sbr_dbbr_mg.argtypes = [_P, _I64, _P, _I64, _INT, _INT, _INT, _INT, _P, _P, _SZ, _P]
+        L.trid_band_gather.argtypes = [_P, _I64, _INT, _P, _I64, _INT, _INT, _P, _I64, _P]
+        for name in ("trid_bulge_chase_band", "trid_comm_unique_id", "trid_comm_init_nccl", "trid_comm_init_local",
+                     "trid_comm_destroy", "trid_comm_size", "trid_comm_rank", "trid_sbr_dbbr_mg_bufsize",
+                     "trid_sbr_dbbr_mg", "trid_band_gather"):
+            getattr(L, name).restype = _INT
         L.trid_profile_begin.restype = _INT
         L.trid_profile_end.restype = _INT
         L.trid_profile_end.argtypes = [_P, _P, _INT]
@@ -75,7 +91,9 @@ def lib():
 EXPORTS = ("trid_status_string", "trid_last_error_string", "trid_version", "trid_default_k", "trid_bc_total_steps", "trid_sbr_dbbr_bufsize",
            "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize", "trid_sbr_dbbr", "trid_bulge_chase",
            "trid_sytrd_2stage", "trid_panel_qr_bufsize", "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize",
-           "trid_zy", "trid_profile_begin", "trid_profile_end", "trid_kernel_launches")
+           "trid_zy", "trid_profile_begin", "trid_profile_end", "trid_kernel_launches", "trid_bulge_chase_band",
+           "trid_comm_unique_id", "trid_comm_init_nccl", "trid_comm_init_local", "trid_comm_destroy", "trid_comm_size",
+           "trid_comm_rank", "trid_mg_local_cols", "trid_sbr_dbbr_mg_bufsize", "trid_sbr_dbbr_mg", "trid_band_gather")
 
 PROF_CLASSES = ("panel_qr", "wy", "symm", "zy", "next_panel", "syr2k", "bulge_chase")
 
@@ -254,3 +272,105 @@ def zy(A: torch.Tensor, W: torch.Tensor, Y: torch.Tensor):
     _check(lib().trid_zy(m, w, _dev(A, "A"), _ld(A, m), _dev(W, "W"), _ld(W, m), _dev(Y, "Y"), _ld(Y, m),
                          _dev(Z, "Z"), m, work.data_ptr(), work.numel(), _stream()), "trid_zy")
     return Z
+
+
+def bulge_chase_band(AB: torch.Tensor, n: int, b: int, want_vectors: bool = True, work=None, out=None):
+    """Stage 2 from LAPACK lower band storage: AB storage tensor of shape (n, ldab) (column-major ldab x n,
+    AB[j, i-j] = B(i, j)).  Returns (d, e, V2, tau2)."""
+    ldab = _ld(AB, b + 1)
+    nbytes, v2len, t2len = bulge_chase_bufsize(n, b)
+    dev = AB.device
+    if out is None:
+        d = torch.empty(max(n, 1), dtype=torch.float64, device=dev)
+        e = torch.empty(max(n - 1, 1), dtype=torch.float64, device=dev)
+        V2 = torch.empty(max(v2len, 1), dtype=torch.float64, device=dev) if want_vectors else None
+        tau2 = torch.empty(max(t2len, 1), dtype=torch.float64, device=dev) if want_vectors else None
+    else:
+        d, e, V2, tau2 = out
+    work = work if work is not None else _workspace(nbytes, dev)
+    _check(lib().trid_bulge_chase_band(n, b, _dev(AB, "AB"), ldab, _dev(d, "d"), _dev(e, "e"),
+                                       V2.data_ptr() if V2 is not None else None,
+                                       tau2.data_ptr() if tau2 is not None else None,
+                                       work.data_ptr(), work.numel(), _stream()), "trid_bulge_chase_band")
+    return d[:n], e[: max(n - 1, 0)], (V2[:v2len] if V2 is not None else None), (tau2[:t2len] if tau2 is not None else None)
+
+
+# ------------------------------------------------------------------ multi-GPU stage 1 (DESIGN.md sec. 8)
+class Comm:
+    """A libtrid communicator handle (NCCL rank or local virtual rank)."""
+
+    def __init__(self, handle: int):
+        self.handle = ctypes.c_void_p(handle)
+
+    @property
+    def size(self) -> int:
+        return lib().trid_comm_size(self.handle)
+
+    @property
+    def rank(self) -> int:
+        return lib().trid_comm_rank(self.handle)
+
+    def destroy(self):
+        if self.handle:
+            _check(lib().trid_comm_destroy(self.handle), "trid_comm_destroy")
+            self.handle = ctypes.c_void_p(0)
+
+
+def comm_local(nranks: int):
+    """nranks virtual ranks sharing this process and the current device (drive each from its own thread)."""
+    arr = (_P * nranks)()
+    _check(lib().trid_comm_init_local(nranks, arr), "trid_comm_init_local")
+    return [Comm(arr[q]) for q in range(nranks)]
+
+
+def comm_nccl(group=None) -> Comm:
+    """NCCL communicator over the ranks of a torch.distributed process group (one GPU per rank, the current
+    CUDA device); the 128-byte unique id is created on rank 0 and broadcast through the group."""
+    import torch.distributed as dist
+    rank, size = dist.get_rank(group), dist.get_world_size(group)
+    dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+    buf = torch.zeros(128, dtype=torch.uint8, device=dev)
+    if rank == 0:
+        idb = ctypes.create_string_buffer(128)
+        _check(lib().trid_comm_unique_id(idb), "trid_comm_unique_id")
+        buf.copy_(torch.frombuffer(bytearray(idb.raw), dtype=torch.uint8))
+    dist.broadcast(buf, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    idb = ctypes.create_string_buffer(bytes(buf.cpu().numpy().tobytes()), 128)
+    h = _P()
+    _check(lib().trid_comm_init_nccl(idb, size, rank, ctypes.byref(h)), "trid_comm_init_nccl")
+    return Comm(h.value)
+
+
+def mg_local_cols(n: int, colblock: int, nranks: int, rank: int) -> int:
+    return int(lib().trid_mg_local_cols(n, colblock, nranks, rank))
+
+
+def sbr_dbbr_mg_bufsize(n, b, nb, k, nranks, rank):
+    out = _SZ()
+    _check(lib().trid_sbr_dbbr_mg_bufsize(n, b, nb, k, nranks, rank, ctypes.byref(out)), "trid_sbr_dbbr_mg_bufsize")
+    return out.value
+
+
+def sbr_dbbr_mg(comm: Comm, A_local: torch.Tensor, n: int, b: int, nb: int | None = None, k: int = 0, tau1=None,
+                work=None):
+    """Stage 1 on this rank's block-cyclic columns (storage tensor of shape (nq, >= n): local column x is row
+    x).  Collective over the communicator.  Returns tau1 (n)."""
+    nb = nb or b
+    g, q = comm.size, comm.rank
+    tau1 = tau1 if tau1 is not None else torch.empty(max(n, 1), dtype=torch.float64, device=A_local.device)
+    nbytes = sbr_dbbr_mg_bufsize(n, b, nb, k, g, q)
+    work = work if work is not None else _workspace(nbytes, A_local.device)
+    ldA = _ld(A_local, n) if A_local.numel() else max(n, 1)
+    _check(lib().trid_sbr_dbbr_mg(comm.handle, n, A_local.data_ptr() if A_local.numel() else None, ldA, b, b, nb, k,
+                                  _dev(tau1, "tau1"), work.data_ptr(), work.numel(), _stream()), "trid_sbr_dbbr_mg")
+    return tau1[:n]
+
+
+def band_gather(comm: Comm, A_local: torch.Tensor, n: int, b: int, root: int = 0, AB=None):
+    """Band of the block-cyclic matrix to `root` in LAPACK lower band storage (returned as a storage tensor
+    of shape (n, b+1)); collective.  Only root's result holds the band."""
+    AB = AB if AB is not None else torch.empty((max(n, 1), b + 1), dtype=torch.float64, device=A_local.device)
+    ldA = _ld(A_local, n) if A_local.numel() else max(n, 1)
+    _check(lib().trid_band_gather(comm.handle, n, b, A_local.data_ptr() if A_local.numel() else None, ldA, b, root,
+                                  _dev(AB, "AB"), _ld(AB, b + 1), _stream()), "trid_band_gather")
+    return AB

@@ -22,6 +22,7 @@
 #include "gemm.cuh"
 #include "panel.cuh"
 #include "prof.cuh"
+#include "driver.cuh"
 
 using namespace trid;
 
@@ -111,17 +112,16 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
   return w;
 }
 
-// ---- the Z builder for one panel (a3): X = A W; corrections; Z_p = X - 1/2 Y_p (W^T X) ----------
-cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const double* Wp, int64_t ldw,
-                     const double* Yp, const double* Yprev, const double* Zprev, int64_t ldyz, int64_t nprev,
-                     double* Zp, double* X, int64_t ldx, double* U1, double* U2, int64_t ldu, double* S, int64_t lds,
-                     double* part, int64_t part_elems, cudaStream_t st) {
+}  // namespace
+
+namespace trid {
+// ---- the Z builder after the SYMM (a3): corrections for the block's earlier panels (R4e), S = W^T X,
+// Z_p = X - 1/2 Y_p S (Eq. (1)).  X (m x kk, ld ldx) holds A_blk W_p on entry and is updated.
+cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
+                    const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U1,
+                    double* U2, int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems,
+                    cudaStream_t st) {
   cudaError_t e;
-  {
-    ProfScope ps(PROF_SYMM, st);
-    e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
-  }
-  if (e != cudaSuccess) return e;
   ProfScope ps(PROF_ZY, st);
   if (nprev > 0) {
     // U1 = Z_<^T W, U2 = Y_<^T W   (TN, K = m, deterministic split-K)
@@ -153,6 +153,22 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
   z.M = m; z.N = kk; z.K[0] = kk; z.A[0] = Yp; z.lda[0] = ldyz; z.B[0] = S; z.ldb[0] = lds;
   z.alpha = -0.5; z.beta = 1.0; z.Cin = X; z.ldcin = ldx; z.C = Zp; z.ldc = ldyz;
   return gemm_ws(z, OP_N, st);
+}
+}  // namespace trid
+
+namespace {
+// ---- the Z builder for one panel (a3): X = A W (SYMM); then zy_tail
+cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const double* Wp, int64_t ldw,
+                     const double* Yp, const double* Yprev, const double* Zprev, int64_t ldyz, int64_t nprev,
+                     double* Zp, double* X, int64_t ldx, double* U1, double* U2, int64_t ldu, double* S, int64_t lds,
+                     double* part, int64_t part_elems, cudaStream_t st) {
+  cudaError_t e;
+  {
+    ProfScope ps(PROF_SYMM, st);
+    e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
+  }
+  if (e != cudaSuccess) return e;
+  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U1, U2, ldu, S, lds, part, part_elems, st);
 }
 
 int check_common(int64_t n, const void* A, int64_t lda, int b) {

@@ -17,6 +17,7 @@
 #include "common.cuh"
 #include "panel.cuh"
 #include "prof.cuh"
+#include "driver.cuh"
 
 #include <stdlib.h>
 
@@ -74,11 +75,13 @@ int bc_ldab(int64_t n, int b) {
 }
 int64_t bc_total_steps(int64_t n, int b) { return n >= 3 ? bc_offset(n, b, n - 2) : 0; }
 
-__global__ void band_pack_kernel(int64_t n, int b, int ldab, const double* A, int64_t lda, double* band) {
+// element (c+o, c) of the input band lives at X[o + c*cs] (full column-major A: X = A, cs = lda+1;
+// LAPACK lower band storage AB: cs = ldab)
+__global__ void band_pack_kernel(int64_t n, int b, int ldab, const double* X, int64_t cs, double* band) {
   const int64_t total = n * ldab;
   for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total; idx += (int64_t)gridDim.x * blockDim.x) {
     const int64_t c = idx / ldab, o = idx - c * ldab;
-    band[idx] = (o <= b && c + o < n) ? A[(c + o) + c * lda] : 0.0;
+    band[idx] = (o <= b && c + o < n) ? X[o + c * cs] : 0.0;
   }
 }
 
@@ -583,6 +586,11 @@ size_t bc_work_bytes(int64_t n, int b) {
 
 cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
                         double* tau2, void* work, cudaStream_t st) {
+  return bulge_chase_cs(n, b, A, lda + 1, d, e, V2, tau2, work, st);
+}
+
+cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double* d, double* e, double* V2,
+                           double* tau2, void* work, cudaStream_t st) {
   if (n <= 0) return cudaSuccess;
   const int beff = (int)((b < n - 1) ? b : (n - 1 > 0 ? n - 1 : 1));
   const int ldab = bc_ldab(n, beff);
@@ -598,7 +606,7 @@ cudaError_t bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* 
     int64_t total = n * (int64_t)ldab;
     int blocks = (int)((total + 255) / 256);
     if (blocks > 8 * kNumSMsB200 * 4) blocks = 8 * kNumSMsB200 * 4;
-    band_pack_kernel<<<blocks, 256, 0, st>>>(n, beff, ldab, A, lda, band);
+    band_pack_kernel<<<blocks, 256, 0, st>>>(n, beff, ldab, X, cs, band);
     count_launches(1);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess) return err;

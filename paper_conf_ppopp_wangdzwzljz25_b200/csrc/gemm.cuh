@@ -36,6 +36,16 @@ struct GemmArgs {
   int splits = 1;
   double* part = nullptr;
   int64_t part_ld = 1, part_stride = 0;
+  // multi-GPU column map for the lower epilogue mask (gemm_ws only): C's column x is global column
+  // cmap(x) = ((x+mg_lofs)/mg_cb*mg_g + mg_q)*mg_cb + (x+mg_lofs)%mg_cb - mg_gofs; mg_g <= 1: identity.
+  int mg_g = 1, mg_q = 0, mg_cb = 1;
+  int64_t mg_lofs = 0, mg_gofs = 0;
+};
+
+// 1D block-cyclic column map of one rank
+struct MgMap {
+  int g = 1, q = 0, cb = 1;
+  int64_t lofs = 0, gofs = 0;
 };
 
 // Launch; when a.splits > 1 also launches the reduction.  Returns the first CUDA error.
@@ -56,5 +66,14 @@ int64_t symm_ws_splits(int64_t m, int64_t w);
 int64_t symm_ws_part_elems(int64_t m, int64_t w);
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
                     int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);
+
+// Multi-GPU SYMM partials over a rank's local trailing columns (nqt of them, A_loc rows = global rows).
+int64_t symm_mg_part_elems(int64_t m, int64_t w, int64_t nqt);
+cudaError_t symm_mg_rows(int64_t m, int64_t w, int64_t nqt, const double* Aloc, int64_t lda, const double* Wloc,
+                         int64_t ldwl, double* X, int64_t ldx, const MgMap& mp, double* part, int64_t part_elems,
+                         cudaStream_t st);
+cudaError_t symm_mg_cols(int64_t m, int64_t w, int64_t nqt, const double* Aloc, int64_t lda, const double* W,
+                         int64_t ldw, double* Xl, int64_t ldxl, const MgMap& mp, double* part, int64_t part_elems,
+                         cudaStream_t st);
 
 }  // namespace trid

@@ -44,6 +44,7 @@ struct Seg {
   int64_t kb, ke;   // K range [kb, ke)
   int opa;          // OP_N / OP_T
   int mask;         // 0 none, 1 keep k <= row, 2 keep k > row (global row = m0 + r)
+  int mapk, mapr;   // multi-GPU: compare cmap(k) / cmap(row) instead of k / row (block-cyclic local columns)
 };
 
 struct WsArgs {
@@ -67,7 +68,31 @@ struct WsArgs {
   double* part;             // split partials: part + z*part_stride, ld part_ld
   int64_t part_ld, part_stride;
   int vec16;                // operands 16-byte aligned (base pointers and leading dimensions even)
+  // multi-GPU column map (1D block-cyclic, mg_g ranks, blocks of mg_cb columns, this rank mg_q): local
+  // column x (relative to local column mg_lofs) is global column cmap(x) (relative to global mg_gofs).
+  // mg_g <= 1: identity.  Used by the lower epilogue mask (C's columns are local) and the SYMM modes 2/3.
+  int mg_g, mg_q, mg_cb;
+  int64_t mg_lofs, mg_gofs;
 };
+
+__device__ __forceinline__ int64_t cmap(const WsArgs& a, int64_t x) {
+  if (a.mg_g <= 1) return x;
+  const int64_t X = x + a.mg_lofs, blk = X / a.mg_cb;
+  return (blk * a.mg_g + a.mg_q) * a.mg_cb + (X - blk * a.mg_cb) - a.mg_gofs;
+}
+// number of local columns x in [0, kt) with cmap(x) <= r
+__device__ __forceinline__ int64_t kcount(const WsArgs& a, int64_t r, int64_t kt) {
+  if (r < 0) return 0;
+  int64_t c;
+  if (a.mg_g <= 1) {
+    c = r + 1;
+  } else {
+    const int64_t G = r + a.mg_gofs, B = G / a.mg_cb, w = G - B * a.mg_cb;
+    const int64_t nbl = B > a.mg_q ? (B - a.mg_q + a.mg_g - 1) / a.mg_g : 0;
+    c = nbl * a.mg_cb + ((B % a.mg_g) == a.mg_q ? w + 1 : 0) - a.mg_lofs;
+  }
+  return c < 0 ? 0 : (c > kt ? kt : c);
+}
 
 __device__ __forceinline__ void tri_unit(int64_t t, int& tm, int& tn) {
   int64_t r = (int64_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
@@ -96,6 +121,27 @@ __device__ __forceinline__ void unit_geom(const WsArgs& a, int64_t u, int64_t& m
 // Segments of unit u (identical in producer and consumers).
 template <int BM, int BN>
 __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg& s0, Seg& s1) {
+  if (a.symm >= 2) {
+    // multi-GPU SYMM partial over this rank's local columns (mode 2: rows = global, K = local columns,
+    // keep cmap(k) <= row; mode 3: rows = local columns, K = global rows, keep k > cmap(row))
+    const int64_t rl = (m0 + BM < a.M ? m0 + BM : a.M) - 1;
+    int64_t lo, hi;
+    if (a.symm == 2) {
+      lo = 0;
+      hi = kcount(a, rl, a.K[0]);
+    } else {
+      lo = (cmap(a, m0) + 1) / BK * BK;
+      hi = a.K[0];
+    }
+    if (hi <= lo) return 0;
+    const int64_t chunk = (hi - lo + a.splits - 1) / a.splits;
+    const int64_t cz = (chunk + BK - 1) / BK * BK;
+    const int64_t k0 = lo + (int64_t)z * cz, k1 = (k0 + cz < hi) ? k0 + cz : hi;
+    if (k1 <= k0) return 0;
+    s0 = a.symm == 2 ? Seg{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, k1, OP_N, 1, 1, 0}
+                     : Seg{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, k1, OP_T, 2, 0, 1};
+    return 1;
+  }
   if (a.symm) {
     // K chunk z of the strip: [k0, k1); row strip (k <= row) then column strip (k > row)
     const int64_t chunk = (a.K[0] + a.splits - 1) / a.splits;
@@ -103,8 +149,8 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
     const int64_t k0 = (int64_t)z * cz, k1 = (k0 + cz < a.K[0]) ? k0 + cz : a.K[0];
     const int64_t e1 = (k1 < m0 + BM) ? k1 : m0 + BM;
     const int64_t s2 = (k0 > m0) ? k0 : m0;
-    const Seg row{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, e1, OP_N, 1};
-    const Seg col{a.A[0], a.B[0], a.lda[0], a.ldb[0], s2, k1, OP_T, 2};
+    const Seg row{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, e1, OP_N, 1, 0, 0};
+    const Seg col{a.A[0], a.B[0], a.lda[0], a.ldb[0], s2, k1, OP_T, 2, 0, 0};
     if (e1 > k0) {
       s0 = row;
       s1 = col;
@@ -128,8 +174,8 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
     kb1 = b0 * BK;
     ke1 = (e * BK < a.K[1]) ? e * BK : a.K[1];
   }
-  const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, OP_N, 0};
-  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, OP_N, 0};
+  const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, OP_N, 0, 0, 0};
+  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, OP_N, 0, 0, 0};
   if (ke0 > kb0) {
     s0 = g0;
     s1 = g1;
@@ -206,7 +252,11 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
   using C = Cfg<BM, BN>;
   const int64_t kend = s.ke;
   // the triangle masks only bite on K-tiles that overlap the diagonal block [m0, m0 + BM)
-  const bool unmasked = s.mask == 0 || (s.mask == 1 && k0 + BK <= m0) || (s.mask == 2 && k0 >= m0 + BM);
+  // (with the multi-GPU map: compare cmap(k) / cmap(row); cmap is monotone)
+  auto km = [&](int64_t k) { return s.mapk ? cmap(a, k) : k; };
+  auto rm = [&](int64_t r) { return s.mapr ? cmap(a, r) : r; };
+  const bool unmasked = s.mask == 0 || (s.mask == 1 && km(k0 + BK - 1) <= rm(m0)) ||
+                        (s.mask == 2 && km(k0) > rm(m0 + BM - 1));
   const bool v16 = a.vec16 && unmasked;
   // ---- A
   if (v16) {
@@ -217,8 +267,8 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
       const int r = e % BM, kk = e / BM;
       const int64_t row = m0 + r, k = k0 + kk;
       bool p = row < a.M && k < kend;
-      if (s.mask == 1) p = p && (k <= row);
-      if (s.mask == 2) p = p && (k > row);
+      if (s.mask == 1) p = p && (km(k) <= rm(row));
+      if (s.mask == 2) p = p && (km(k) > rm(row));
       cp8(As + kk * C::A_LD_N + r, p ? s.A + row + k * s.lda : s.A, p ? 8 : 0);
     }
   } else {                      // op(A)(m, k) = A[k + m*lda], tile As[m][k]
@@ -226,8 +276,8 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
       const int kk = e % BK, r = e / BK;
       const int64_t row = m0 + r, k = k0 + kk;
       bool p = row < a.M && k < kend;
-      if (s.mask == 1) p = p && (k <= row);
-      if (s.mask == 2) p = p && (k > row);
+      if (s.mask == 1) p = p && (km(k) <= rm(row));
+      if (s.mask == 2) p = p && (km(k) > rm(row));
       cp8(As + r * C::A_LD_T + kk, p ? s.A + k + row * s.lda : s.A, p ? 8 : 0);
     }
   }
@@ -318,7 +368,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
       int64_t m0, n0;
       int z;
       unit_geom<BM, BN>(a, u, m0, n0, z);
-      if (a.lower && m0 + BM - 1 + a.diag_off < n0) continue;
+      if (a.lower && m0 + BM - 1 + a.diag_off < cmap(a, n0)) continue;
       Seg s0, s1;
       const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
       auto run = [&](const Seg& sgm) {
@@ -345,7 +395,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
     int64_t m0, n0;
     int z;
     unit_geom<BM, BN>(a, u, m0, n0, z);
-    if (a.lower && m0 + BM - 1 + a.diag_off < n0) continue;
+    if (a.lower && m0 + BM - 1 + a.diag_off < cmap(a, n0)) continue;
     Seg s0, s1;
     const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
     double acc[MT][NT][4];
@@ -377,7 +427,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
         for (int i = 0; i < 4; ++i) {
           const int64_t r = m0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
           const int64_t c = n0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
-          if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= c)) {
+          if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= cmap(a, c))) {
             if (a.splits > 1) {
               a.part[z * a.part_stride + r + c * a.part_ld] = acc[mt][nt][i];
             } else {
@@ -456,6 +506,8 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
   a.alpha = g.alpha; a.beta = g.beta; a.Cin = g.Cin; a.ldcin = g.ldcin; a.C = g.C; a.ldc = g.ldc;
   a.lower = g.lower; a.diag_off = g.diag_off; a.tri = g.tri;
   a.splits = g.splits < 1 ? 1 : g.splits;
+  a.mg_g = g.mg_g; a.mg_q = g.mg_q; a.mg_cb = g.mg_cb; a.mg_lofs = g.mg_lofs; a.mg_gofs = g.mg_gofs;
+  if (a.mg_g > 1 && (a.tri || (a.lower && a.splits > 1) || a.mg_cb < 1)) return cudaErrorInvalidValue;
   a.part = g.part; a.part_ld = g.part_ld; a.part_stride = g.part_stride;
   if (g.N <= 64) {
     return opB == OP_T ? ws::launch<128, 64, 4, 2, OP_T>(a, st) : ws::launch<128, 64, 4, 2, OP_N>(a, st);
@@ -496,6 +548,50 @@ cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const do
   a.splits = (int)sp;
   a.part = part; a.part_ld = m; a.part_stride = m * w;
   return ws::launch<128, 64, 4, 2, OP_N>(a, st);
+}
+
+// ---- multi-GPU SYMM partials (block-cyclic local columns) ------------------------
+static int64_t mg_splits(int64_t tiles, int64_t K) {
+  int64_t sp = (8 * kNumSMsB200 + tiles - 1) / tiles;
+  const int64_t maxs = (K + 511) / 512;
+  if (sp > maxs) sp = maxs;
+  if (sp > 32) sp = 32;
+  return sp < 1 ? 1 : sp;
+}
+int64_t symm_mg_part_elems(int64_t m, int64_t w, int64_t nqt) {
+  const int64_t tn = (w + 63) / 64;
+  const int64_t s2 = mg_splits((m + 127) / 128 * tn, nqt), s3 = mg_splits((nqt + 127) / 128 * tn, m);
+  const int64_t e2 = s2 > 1 ? s2 * m * w : 0, e3 = s3 > 1 ? s3 * nqt * w : 0;
+  return e2 > e3 ? e2 : e3;
+}
+static cudaError_t symm_mg(int mode, int64_t M, int64_t w, int64_t K, const double* A, int64_t lda, const double* B,
+                           int64_t ldb, double* C, int64_t ldc, const MgMap& mp, double* part, int64_t part_elems,
+                           cudaStream_t st) {
+  if (M <= 0 || w <= 0) return cudaSuccess;
+  ws::WsArgs a{};
+  a.M = M; a.N = w; a.opb = OP_N; a.nseg = 1; a.symm = mode;
+  a.A[0] = A; a.B[0] = B; a.lda[0] = lda; a.ldb[0] = ldb; a.K[0] = K;
+  a.vec16 = ws::al16(A) && ws::al16(B) && !(lda & 1) && !(ldb & 1);
+  a.alpha = 1.0; a.beta = 0.0; a.C = C; a.ldc = ldc;
+  a.mg_g = mp.g; a.mg_q = mp.q; a.mg_cb = mp.cb; a.mg_lofs = mp.lofs; a.mg_gofs = mp.gofs;
+  int64_t sp = mg_splits((M + 127) / 128 * ((w + 63) / 64), K);
+  if (sp * M * w > part_elems) sp = part_elems / (M * w);
+  if (sp < 1) sp = 1;
+  a.splits = (int)sp;
+  a.part = part; a.part_ld = M; a.part_stride = M * w;
+  return w <= 64 ? ws::launch<128, 64, 4, 2, OP_N>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
+}
+// X (m x w) = sum over local columns x with cmap(x) <= row of A_loc(row, x) W_loc(x, :)
+cudaError_t symm_mg_rows(int64_t m, int64_t w, int64_t nqt, const double* Aloc, int64_t lda, const double* Wloc,
+                         int64_t ldwl, double* X, int64_t ldx, const MgMap& mp, double* part, int64_t part_elems,
+                         cudaStream_t st) {
+  return symm_mg(2, m, w, nqt, Aloc, lda, Wloc, ldwl, X, ldx, mp, part, part_elems, st);
+}
+// Xl (nqt x w) = sum over global rows k > cmap(x) of A_loc(k, x) W(k, :)
+cudaError_t symm_mg_cols(int64_t m, int64_t w, int64_t nqt, const double* Aloc, int64_t lda, const double* W,
+                         int64_t ldw, double* Xl, int64_t ldxl, const MgMap& mp, double* part, int64_t part_elems,
+                         cudaStream_t st) {
+  return symm_mg(3, nqt, w, m, Aloc, lda, W, ldw, Xl, ldxl, mp, part, part_elems, st);
 }
 
 }  // namespace trid

@@ -17,6 +17,8 @@
 #include "panel.cuh"
 #include "prof.cuh"
 
+#include <stdlib.h>
+
 namespace trid {
 
 namespace cg = cooperative_groups;
@@ -292,7 +294,11 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   attr[1].id = cudaLaunchAttributeCooperative;
   attr[1].val.cooperative = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 2;
+  // The cooperative attribute guarantees co-residency for the grid barrier.  ncu cannot replay a
+  // cooperative cluster launch, so profiling runs set TRID_PANEL_NOCOOP=1 (the grid fits in one wave:
+  // G <= 4 x max co-resident clusters, so on an otherwise idle GPU every CTA is resident anyway).
+  static const bool nocoop = getenv("TRID_PANEL_NOCOOP") != nullptr;
+  cfg.numAttrs = nocoop ? 1 : 2;
   count_launches(1);
   switch (w) {
     case 16: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<2>, a);

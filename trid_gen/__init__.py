@@ -89,6 +89,29 @@ def random_symmetric(n: int, seed: int, device="cpu", out: torch.Tensor | None =
     return A
 
 
+def random_symmetric_rows(n: int, seed: int, rows, device="cpu", chunk: int = 2048) -> torch.Tensor:
+    """Rows `rows` (global indices) of random_symmetric(n, seed), as a (len(rows), n) tensor.  For the
+    symmetric matrix row c equals column c, so this is also the column-major storage of the columns
+    `rows` (the multi-GPU block-cyclic local matrix)."""
+    rows = torch.as_tensor(rows, dtype=torch.int64, device=device)
+    A = torch.empty((rows.numel(), n), dtype=torch.float64, device=device)
+    cols = torch.arange(n, dtype=torch.int64, device=device)
+    for r0 in range(0, rows.numel(), chunk):
+        r = rows[r0:r0 + chunk, None]
+        lo = torch.minimum(r, cols[None, :])
+        hi = torch.maximum(r, cols[None, :])
+        A[r0:r0 + chunk] = 2.0 * uniform_t(seed, lo * n + hi) - 1.0
+    return A
+
+
+def block_cyclic_columns(n: int, colblock: int, nranks: int, rank: int) -> np.ndarray:
+    """Global column indices stored by `rank` in the 1D block-cyclic layout (blocks of colblock columns,
+    block B on rank B % nranks), in local order.  Pure index bookkeeping."""
+    blocks = np.arange(rank, (n + colblock - 1) // colblock, nranks, dtype=np.int64)
+    cols = (blocks[:, None] * colblock + np.arange(colblock, dtype=np.int64)[None, :]).ravel()
+    return cols[cols < n]
+
+
 def _vec_idx(t: int, n: int, device) -> torch.Tensor:
     return (1 << 62) + t * (1 << 32) + torch.arange(n, dtype=torch.int64, device=device)
 
