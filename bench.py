@@ -309,7 +309,7 @@ def main():
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tpath):
         try:
-            traffic = json.load(open(tpath)).get(f"{cfg.get('name', args.config)}:{dom}")
+            traffic = json.load(open(tpath)).get(f"{args.config}:{dom}")
         except Exception:
             traffic = None
     hbm, hbm_kind = peaks()

@@ -577,6 +577,279 @@ __global__ void __launch_bounds__(NTH, 3 - NBUF) bc_fast_kernel(BcArgs a) {
   }
 }
 
+// ---- warp-specialized chase (default for b <= 64) -----------------------------------------------------
+// Same step arithmetic and register-resident window as bc_fast_kernel, but no compute warp ever waits on
+// global memory: NTH compute threads (named barrier 1) + a LOAD warp + a STORE warp.
+//   LOAD  (lane 0): claims sweeps (atomic ticket), and for every step fills a window buffer by bulk copies
+//         completing on full[buf] (mbarrier, expect_tx): columns 0..L-2 once the predecessor sweep's
+//         prog_full reached m+1, the last column once its prog reached min(m+2, nprev) (R9, lag 2), plus
+//         column s at a sweep's step 0.  It runs one step ahead (prefetch) and only waits on the
+//         predecessor sweep and on empty[buf] (the STORE warp finished with that buffer).
+//   STORE (lane 0): waits col0[] (compute finalized column 0) -> bulk store, completion, st.release prog;
+//         waits cols[] (left-apply done) -> bulk store of columns 1..L-1, completion, release prog_full,
+//         then frees the buffer (empty[buf]).  It never waits on another CTA, so publication cannot be
+//         held up by this CTA's own prefetch (no cycle through the predecessor chain).
+// Step/sweep ids travel with the buffer (info[buf]); s < 0 terminates all roles.
+template <int B, int NTH>
+__global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
+  constexpr int TPR = NTH / (2 * B);
+  constexpr int CPT = B / TPR;
+  constexpr int RW = (2 * B) / 32;
+  constexpr int NW = NTH / 32;
+  constexpr int CPW = B / NW;
+  static_assert(CPW == 4 || CPW == 8, "z-pass butterfly assumes 4 or 8 columns per warp");
+  extern __shared__ __align__(16) double sm[];
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int lda1 = ldab - 1;
+  const int64_t n = a.n;
+  const int wsz = B * ldab;
+  double* colb = sm + 2 * wsz;               // 2 x ldab: column s of a sweep's step 0, per buffer
+  double* vb = colb + 2 * ldab;              // 2 x B   (v / vn)
+  double* pyv = vb + 2 * B;                  // 2B
+  double* zv = pyv + 2 * B;                  // B
+  double* part = zv + B;                     // TPR x 2B
+  __shared__ __align__(8) uint64_t full[2], empty[2], col0b[2], colsb[2];
+  __shared__ int64_t info_s[2];
+  __shared__ int info_m[2];
+  if (tid == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+      mbar_init(&col0b[i], 1);
+      mbar_init(&colsb[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == NW) {
+    // ============================== LOAD warp ==============================
+    if (lane != 0) return;
+    uint32_t it = 0;
+    for (;;) {
+      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
+      const bool done = s > n - 3;
+      const int64_t nst = done ? 1 : bc_steps(n, b, s);
+      const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+      for (int64_t m = 0; m < nst; ++m, ++it) {
+        const int bi = it & 1;
+        if (it >= 2) mbar_wait(&empty[bi], ((it >> 1) - 1) & 1u);
+        if (done) {
+          info_s[bi] = -1;
+          mbar_arrive(&full[bi]);
+          return;
+        }
+        info_s[bi] = s;
+        info_m[bi] = (int)m;
+        const int64_t r0 = s + 1 + m * b;
+        const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+        const int L = (int)(r1 - r0 + 1);
+        double* win = sm + bi * wsz;
+        mbar_arrive_expect_tx(&full[bi], (unsigned)((L + (m == 0 ? 1 : 0)) * ldab * 8));
+        if (s > 0) {
+          if (m == 0) wait_geq(a.prog + (s - 1), 1);
+          wait_geq(a.prog_full + (s - 1), (int)(m + 1));
+        }
+        fence_proxy_async_global();
+        if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
+        if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
+        if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        fence_proxy_async_global();
+        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &full[bi]);
+      }
+    }
+  }
+  if (warp == NW + 1) {
+    // ============================== STORE warp ==============================
+    if (lane != 0) return;
+    for (uint32_t it = 0;; ++it) {
+      const int bi = it & 1;
+      const unsigned ph = (it >> 1) & 1u;
+      mbar_wait(&col0b[bi], ph);
+      const int64_t s = info_s[bi];
+      if (s < 0) return;
+      const int m = info_m[bi];
+      const int64_t r0 = s + 1 + (int64_t)m * b;
+      const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
+      const int L = (int)(r1 - r0 + 1);
+      double* win = sm + bi * wsz;
+      bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
+      bulk_commit();
+      bulk_wait_all();
+      fence_proxy_async_global();
+      st_release_s32(a.prog + s, m + 1);
+      mbar_wait(&colsb[bi], ph);
+      if (L > 1) {
+        bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
+        bulk_commit();
+        bulk_wait_all();
+        fence_proxy_async_global();
+      }
+      st_release_s32(a.prog_full + s, m + 1);
+      mbar_arrive(&empty[bi]);
+    }
+  }
+  // ============================== compute warps ==============================
+  const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
+  auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NTH) : "memory"); };
+  double tau = 0.0;
+  for (uint32_t it = 0;; ++it) {
+    const int bi = it & 1;
+    const unsigned ph = (it >> 1) & 1u;
+    mbar_wait(&full[bi], ph);
+    const int64_t s = info_s[bi];
+    if (s < 0) {
+      if (tid == 0) mbar_arrive(&col0b[bi]);   // wake the STORE warp so it can see the end
+      return;
+    }
+    const int64_t m = info_m[bi];
+    const int64_t off = bc_offset(n, b, s);
+    const int64_t r0 = s + 1 + m * b;
+    const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+    const int L = (int)(r1 - r0 + 1);
+    const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
+    const int L2 = (int)(r2 - r1);
+    double* win = sm + bi * wsz;
+    double* v = vb + (m & 1) * B;
+    double* vn = vb + ((m & 1) ^ 1) * B;
+    if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
+      const double* col = colb + bi * ldab + 1;
+      double sig = 0.0;
+      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
+      sig = warp_sum(sig);
+      const House hh = make_house(col[0], sig);
+      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
+      if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
+      tau = hh.tau;
+      cbar();
+    }
+    const bool active = r < L + L2;
+    const bool isO = r >= L && active;
+    const int lo_base = j0 * lda1 + r;
+    const int hi_base = r * lda1 + j0;
+    double e[CPT];
+#pragma unroll
+    for (int jj = 0; jj < CPT; ++jj) {
+      const int j = j0 + jj;
+      e[jj] = win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
+    }
+    if (tau != 0.0) {
+      double acc0 = 0.0, acc1 = 0.0;
+#pragma unroll
+      for (int jj = 0; jj < CPT; jj += 2) {
+        acc0 = fma(e[jj], v[j0 + jj], acc0);
+        acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
+      }
+      part[hg * 2 * B + r] = acc0 + acc1;
+      cbar();
+      if (tid < 2 * B) {
+        double acc = 0.0;
+#pragma unroll
+        for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + tid];
+        pyv[tid] = (tid >= L) ? acc : tau * acc;
+      }
+      cbar();
+      double pv = 0.0;
+      for (int i = lane; i < L; i += 32) pv += pyv[i] * v[i];
+      pv = warp_sum(pv);
+      const double hp = 0.5 * tau * pv;
+      if (isO) {
+        const double ty = tau * pyv[r];
+#pragma unroll
+        for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
+      } else {
+        const double vr = r < L ? v[r] : 0.0;
+        const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
+#pragma unroll
+        for (int jj = 0; jj < CPT; ++jj) {
+          const double vj = v[j0 + jj];
+          const double wj = fma(-hp, vj, pyv[j0 + jj]);
+          e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
+        }
+      }
+    }
+#pragma unroll
+    for (int jj = 0; jj < CPT; ++jj) {
+      const int j = j0 + jj;
+      if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
+    }
+    cbar();
+    double tau_next = 0.0;
+    House h2;
+    h2.beta = 0.0;
+    h2.tau = 0.0;
+    h2.scale = 0.0;
+    if (L2 > 0) {
+      double sg = 0.0;
+      for (int i = 1 + lane; i < L2; i += 32) sg = fma(win[L + i], win[L + i], sg);
+      sg = warp_sum(sg);
+      h2 = make_house(win[L], sg);
+      tau_next = h2.tau;
+      if (tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : h2.scale * win[L + tid]) : 0.0;
+    }
+    if (L2 > 0 && h2.tau != 0.0 && L > 1) {
+      const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
+      const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
+      double c[CPW];
+#pragma unroll
+      for (int q = 0; q < CPW; ++q) {
+        const int j = warp + q * NW;
+        double acc = 0.0;
+        if (j >= 1 && j < L) {
+          const int ob = j * lda1 + L;
+          if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
+          if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
+        }
+        c[q] = acc;
+      }
+      {
+        int qbase = 0;
+#pragma unroll
+        for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
+          const bool up = (lane & o) != 0;
+#pragma unroll
+          for (int i = 0; i < K / 2; ++i) {
+            const double send = up ? c[i] : c[i + K / 2];
+            const double keep = up ? c[i + K / 2] : c[i];
+            c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+          }
+          if (up) qbase += K / 2;
+        }
+        constexpr int LV = CPW == 4 ? 2 : 3;
+        double f = c[0];
+#pragma unroll
+        for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+        if ((lane & ((32 >> LV) - 1)) == 0) {
+          const int j = warp + qbase * NW;
+          if (j >= 1 && j < L) zv[j] = fma(h2.scale, f, win[j * lda1 + L]);
+        }
+      }
+    }
+    cbar();   // all reads of the raw O(:, 0) done; zv ready
+    if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
+    fence_proxy_async_smem();
+    cbar();
+    if (tid == 0) mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
+    if (L2 > 0 && h2.tau != 0.0 && isO) {
+      const double vni = vn[r - L];
+      const double tv = h2.tau * vni;
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
+      }
+    }
+    fence_proxy_async_smem();
+    if (a.V2) {
+      double* vd = a.V2 + (off + m) * a.vs;
+      for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
+      if (tid == 0) a.tau2[off + m] = tau;
+    }
+    cbar();
+    if (tid == 0) mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
+    tau = tau_next;
+  }
+}
+
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
   const size_t flags = sizeof(int) * (size_t)(2 * n + 128);
@@ -624,25 +897,37 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
     a.trace_sweep = tr ? atoll(tr) : -1;
     int occ = 1;
     if (beff <= 64) {
-      // B = 64: 1 CTA/SM x 512 threads with a double-buffered window (default; n=32768: 458 ms) or, forced,
-      // 2 CTAs/SM x 256 threads with a single buffer (580 ms: the chase is dependency-chain bound).
+      // default: warp-specialized chase (bc_ws_kernel, 1 CTA/SM).  TRID_BC_FORCE (debug/tests): "1" the
+      // single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel.
       const int B = beff <= 32 ? 32 : 64;
-      bool two = false;   // measured: the chase is chain bound at every n in configs (1 CTA/SM, 512 thr wins)
-      const char* force = getenv("TRID_BC_FORCE");   // debug/test: "1" single-buffer 2 CTAs/SM, "2" double
-      if (force && B == 64) two = force[0] == '1';
-      const int nbuf = (B == 64 && two) ? 1 : 2;
-      const int nth = B == 32 ? 256 : (two ? 256 : 512);
-      const size_t smem = sizeof(double) * (nbuf * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
-      const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256, 2>
-                               : (two ? (const void*)bc_fast_kernel<64, 256, 1> : (const void*)bc_fast_kernel<64, 512, 2>);
-      cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, nth, smem);
-      if (occ < 1) occ = 1;
-      int64_t grid = (int64_t)kNumSMsB200 * occ;
-      if (grid > n - 2) grid = n - 2;
-      if (B == 32) bc_fast_kernel<32, 256, 2><<<(unsigned)grid, 256, smem, st>>>(a);
-      else if (two) bc_fast_kernel<64, 256, 1><<<(unsigned)grid, 256, smem, st>>>(a);
-      else bc_fast_kernel<64, 512, 2><<<(unsigned)grid, 512, smem, st>>>(a);
+      const char* force = getenv("TRID_BC_FORCE");
+      const int variant = force ? force[0] - '0' : 3;
+      if (variant == 3) {
+        const int nth = B == 32 ? 256 : 512;
+        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B + B +
+                                              (size_t)(nth / (2 * B)) * 2 * B + 8);
+        const void* fn = B == 32 ? (const void*)bc_ws_kernel<32, 256> : (const void*)bc_ws_kernel<64, 512>;
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int64_t grid = kNumSMsB200;
+        if (grid > n - 2) grid = n - 2;
+        if (B == 32) bc_ws_kernel<32, 256><<<(unsigned)grid, 256 + 64, smem, st>>>(a);
+        else bc_ws_kernel<64, 512><<<(unsigned)grid, 512 + 64, smem, st>>>(a);
+      } else {
+        const bool two = B == 64 && variant == 1;
+        const int nbuf = two ? 1 : 2;
+        const int nth = B == 32 ? 256 : (two ? 256 : 512);
+        const size_t smem = sizeof(double) * (nbuf * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
+        const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256, 2>
+                                 : (two ? (const void*)bc_fast_kernel<64, 256, 1> : (const void*)bc_fast_kernel<64, 512, 2>);
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, nth, smem);
+        if (occ < 1) occ = 1;
+        int64_t grid = (int64_t)kNumSMsB200 * occ;
+        if (grid > n - 2) grid = n - 2;
+        if (B == 32) bc_fast_kernel<32, 256, 2><<<(unsigned)grid, 256, smem, st>>>(a);
+        else if (two) bc_fast_kernel<64, 256, 1><<<(unsigned)grid, 256, smem, st>>>(a);
+        else bc_fast_kernel<64, 512, 2><<<(unsigned)grid, 512, smem, st>>>(a);
+      }
     } else {
       const size_t vec = sizeof(double) * (size_t)(5 * beff + 2 * BC_NT + 8);
       const size_t winb = sizeof(double) * (size_t)beff * ldab;

@@ -75,16 +75,18 @@ struct WsArgs {
   int64_t mg_lofs, mg_gofs;
 };
 
+template <bool MG>
 __device__ __forceinline__ int64_t cmap(const WsArgs& a, int64_t x) {
-  if (a.mg_g <= 1) return x;
+  if (!MG) return x;
   const int64_t X = x + a.mg_lofs, blk = X / a.mg_cb;
   return (blk * a.mg_g + a.mg_q) * a.mg_cb + (X - blk * a.mg_cb) - a.mg_gofs;
 }
 // number of local columns x in [0, kt) with cmap(x) <= r
+template <bool MG>
 __device__ __forceinline__ int64_t kcount(const WsArgs& a, int64_t r, int64_t kt) {
   if (r < 0) return 0;
   int64_t c;
-  if (a.mg_g <= 1) {
+  if (!MG) {
     c = r + 1;
   } else {
     const int64_t G = r + a.mg_gofs, B = G / a.mg_cb, w = G - B * a.mg_cb;
@@ -119,18 +121,18 @@ __device__ __forceinline__ void unit_geom(const WsArgs& a, int64_t u, int64_t& m
 }
 
 // Segments of unit u (identical in producer and consumers).
-template <int BM, int BN>
+template <int BM, int BN, bool MG>
 __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg& s0, Seg& s1) {
-  if (a.symm >= 2) {
+  if (MG && a.symm >= 2) {
     // multi-GPU SYMM partial over this rank's local columns (mode 2: rows = global, K = local columns,
     // keep cmap(k) <= row; mode 3: rows = local columns, K = global rows, keep k > cmap(row))
     const int64_t rl = (m0 + BM < a.M ? m0 + BM : a.M) - 1;
     int64_t lo, hi;
     if (a.symm == 2) {
       lo = 0;
-      hi = kcount(a, rl, a.K[0]);
+      hi = kcount<MG>(a, rl, a.K[0]);
     } else {
-      lo = (cmap(a, m0) + 1) / BK * BK;
+      lo = (cmap<MG>(a, m0) + 1) / BK * BK;
       hi = a.K[0];
     }
     if (hi <= lo) return 0;
@@ -246,15 +248,15 @@ __device__ __forceinline__ void load_kinner16(double* T, const double* base, int
 }
 
 // Producer: one K-tile of A and B into stage buffers (NP threads).
-template <int BM, int BN, int NP>
+template <int BM, int BN, int NP, bool MG>
 __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t k0, int64_t m0, int64_t n0,
                                           double* As, double* Bs, int pt) {
   using C = Cfg<BM, BN>;
   const int64_t kend = s.ke;
   // the triangle masks only bite on K-tiles that overlap the diagonal block [m0, m0 + BM)
   // (with the multi-GPU map: compare cmap(k) / cmap(row); cmap is monotone)
-  auto km = [&](int64_t k) { return s.mapk ? cmap(a, k) : k; };
-  auto rm = [&](int64_t r) { return s.mapr ? cmap(a, r) : r; };
+  auto km = [&](int64_t k) { return MG && s.mapk ? cmap<MG>(a, k) : k; };
+  auto rm = [&](int64_t r) { return MG && s.mapr ? cmap<MG>(a, r) : r; };
   const bool unmasked = s.mask == 0 || (s.mask == 1 && km(k0 + BK - 1) <= rm(m0)) ||
                         (s.mask == 2 && km(k0) > rm(m0 + BM - 1));
   const bool v16 = a.vec16 && unmasked;
@@ -339,7 +341,7 @@ constexpr int NPW = 4;   // producer warps (one warpgroup, so setmaxnreg can shr
 // warpgroup drops to 96 and the two consumer warpgroups rise to 200: 128*96 + 256*200 = 63488 <= 64512
 // (an increase the freed registers cannot cover blocks setmaxnreg.inc forever).
 
-template <int BM, int BN, int CWM, int CWN, int OPB>
+template <int BM, int BN, int CWM, int CWN, int OPB, bool MG>
 __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __grid_constant__ WsArgs a) {
   using C = Cfg<BM, BN>;
   constexpr int NCW = CWM * CWN;
@@ -368,16 +370,16 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
       int64_t m0, n0;
       int z;
       unit_geom<BM, BN>(a, u, m0, n0, z);
-      if (a.lower && m0 + BM - 1 + a.diag_off < cmap(a, n0)) continue;
+      if (a.lower && m0 + BM - 1 + a.diag_off < cmap<MG>(a, n0)) continue;
       Seg s0, s1;
-      const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
+      const int ns = unit_segs<BM, BN, MG>(a, m0, z, s0, s1);
       auto run = [&](const Seg& sgm) {
         for (int64_t k0 = sgm.kb; k0 < sgm.ke; k0 += BK, ++kt) {
           const int slot = kt % STAGES;
           const uint32_t use = kt / STAGES;
           if (use > 0) mbar_wait(&empty[slot], (use - 1) & 1u);
           double* As = smem + (size_t)slot * C::STAGE;
-          load_tile<BM, BN, NPW * 32>(a, sgm, k0, m0, n0, As, As + C::A_ELEMS, pt);
+          load_tile<BM, BN, NPW * 32, MG>(a, sgm, k0, m0, n0, As, As + C::A_ELEMS, pt);
           cp_arrive_noinc(&full[slot]);
         }
       };
@@ -395,9 +397,9 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
     int64_t m0, n0;
     int z;
     unit_geom<BM, BN>(a, u, m0, n0, z);
-    if (a.lower && m0 + BM - 1 + a.diag_off < cmap(a, n0)) continue;
+    if (a.lower && m0 + BM - 1 + a.diag_off < cmap<MG>(a, n0)) continue;
     Seg s0, s1;
-    const int ns = unit_segs<BM, BN>(a, m0, z, s0, s1);
+    const int ns = unit_segs<BM, BN, MG>(a, m0, z, s0, s1);
     double acc[MT][NT][4];
 #pragma unroll
     for (int i = 0; i < MT; ++i)
@@ -427,7 +429,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
         for (int i = 0; i < 4; ++i) {
           const int64_t r = m0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
           const int64_t c = n0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
-          if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= cmap(a, c))) {
+          if (r < a.M && c < a.N && (!a.lower || r + a.diag_off >= cmap<MG>(a, c))) {
             if (a.splits > 1) {
               a.part[z * a.part_stride + r + c * a.part_ld] = acc[mt][nt][i];
             } else {
@@ -456,12 +458,12 @@ __global__ void ws_reduce_kernel(int64_t M, int64_t N, int splits, const double*
   }
 }
 
-template <int BM, int BN, int CWM, int CWN, int OPB>
+template <int BM, int BN, int CWM, int CWN, int OPB, bool MG = false>
 static cudaError_t launch(WsArgs& a, cudaStream_t st) {
   using C = Cfg<BM, BN>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(ws_kernel<BM, BN, CWM, CWN, OPB>,
+    cudaError_t e = cudaFuncSetAttribute(ws_kernel<BM, BN, CWM, CWN, OPB, MG>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
@@ -473,7 +475,7 @@ static cudaError_t launch(WsArgs& a, cudaStream_t st) {
   a.units = tiles * a.splits;
   int64_t grid = a.units < kNumSMsB200 ? a.units : kNumSMsB200;
   if (grid < 1) return cudaSuccess;
-  ws_kernel<BM, BN, CWM, CWN, OPB><<<(unsigned)grid, (CWM * CWN + NPW) * 32, C::SMEM, st>>>(a);
+  ws_kernel<BM, BN, CWM, CWN, OPB, MG><<<(unsigned)grid, (CWM * CWN + NPW) * 32, C::SMEM, st>>>(a);
   count_launches(1);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess || a.splits == 1) return e;
@@ -509,6 +511,10 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
   a.mg_g = g.mg_g; a.mg_q = g.mg_q; a.mg_cb = g.mg_cb; a.mg_lofs = g.mg_lofs; a.mg_gofs = g.mg_gofs;
   if (a.mg_g > 1 && (a.tri || (a.lower && a.splits > 1) || a.mg_cb < 1)) return cudaErrorInvalidValue;
   a.part = g.part; a.part_ld = g.part_ld; a.part_stride = g.part_stride;
+  if (a.mg_g > 1) {   // multi-GPU column map (only the lower-masked syr2k of mg.cu uses it)
+    if (opB != OP_T) return cudaErrorInvalidValue;
+    return g.N <= 64 ? ws::launch<128, 64, 4, 2, OP_T, true>(a, st) : ws::launch<128, 128, 4, 2, OP_T, true>(a, st);
+  }
   if (g.N <= 64) {
     return opB == OP_T ? ws::launch<128, 64, 4, 2, OP_T>(a, st) : ws::launch<128, 64, 4, 2, OP_N>(a, st);
   }
@@ -579,7 +585,7 @@ static cudaError_t symm_mg(int mode, int64_t M, int64_t w, int64_t K, const doub
   if (sp < 1) sp = 1;
   a.splits = (int)sp;
   a.part = part; a.part_ld = M; a.part_stride = M * w;
-  return w <= 64 ? ws::launch<128, 64, 4, 2, OP_N>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
+  return w <= 64 ? ws::launch<128, 64, 4, 2, OP_N, true>(a, st) : ws::launch<128, 128, 4, 2, OP_N, true>(a, st);
 }
 // X (m x w) = sum over local columns x with cmap(x) <= row of A_loc(row, x) W_loc(x, :)
 cudaError_t symm_mg_rows(int64_t m, int64_t w, int64_t nqt, const double* Aloc, int64_t lda, const double* Wloc,

@@ -1,0 +1,87 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times (-m gpu).
+
+Q cannot be formed at n >= 8192, so:
+  * G3 on prescribed-spectrum inputs (trid_gen.clustered_symmetric: the 1-2-1 Toeplitz spectrum in closed
+    form, or 32 tight clusters), eigenvalues of T sampled one by one with the oracle's Sturm count
+    (bisection to full precision), against the known eigenvalues: within 1e-12 ||A||_2;
+  * G1/G2 with Hutchinson probes through the returned reflectors (tests/qapply.py): <= 1e-14;
+  * the stage split is checked too: the band after stage 1 has the input's spectrum (sampled)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_ppopp_wangdzwzljz25_b200 as trid
+import trid_gen
+from tests.qapply import probe_gates
+
+pytestmark = pytest.mark.gpu
+
+
+def sampled_eigs(d, e, idx):
+    """k-th smallest eigenvalues of tridiag(e, d, e) for k in idx, each by bisection on the oracle's Sturm
+    count (Gershgorin start, stop at width <= 2 eps max(|lo|, |hi|))."""
+    g = np.abs(np.concatenate([[0.0], e])) + np.abs(np.concatenate([e, [0.0]]))
+    lo0, hi0 = float(np.min(d - g)), float(np.max(d + g))
+    out = []
+    for k in idx:
+        lo, hi = lo0, hi0
+        while hi - lo > 2 * np.finfo(float).eps * max(abs(lo), abs(hi), 1e-300):
+            mid = 0.5 * (lo + hi)
+            if mid <= lo or mid >= hi:
+                break
+            if oracle.sturm_count(d, e, mid) > k:
+                hi = mid
+            else:
+                lo = mid
+        out.append(0.5 * (lo + hi))
+    return np.array(out)
+
+
+@pytest.mark.parametrize("n,b,nb,k,kind,seed", [
+    (8192, 64, 16, 1024, "toeplitz", 2001),       # configs[1]
+    (32768, 64, 16, 1024, "toeplitz", 3001),      # configs[2], the bench headline launch configuration
+    (16384, 128, 16, 1024, "clusters", 5001),     # configs[4] (b sweep, widest default-path band)
+])
+def test_fullsize_gates(n, b, nb, k, kind, seed, dev):
+    A, lam = trid_gen.clustered_symmetric(n, seed, kind=kind, device="cuda:0")
+    A0 = A.clone()
+    d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=nb, k=k)
+    torch.cuda.synchronize()
+    norm2 = float(np.max(np.abs(lam)))
+    dn, en = d.cpu().numpy(), e.cpu().numpy()
+    rng = np.random.default_rng(seed)
+    idx = np.unique(np.concatenate([[0, n - 1], rng.integers(0, n, 62)]))
+    w = sampled_eigs(dn, en, idx)
+    assert np.max(np.abs(w - lam[idx])) <= 1e-12 * norm2
+    g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b, p=4)
+    assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
+
+
+def test_fullsize_random_b_sweep_spectrum(dev):
+    """configs[4]: n = 16384 random symmetric, b in {32, 64, 256}: eigenvalues of T (sampled) equal those of
+    the input (cuSOLVER syevd through torch as the independent reference for a random matrix)."""
+    n = 16384
+    A = trid_gen.random_symmetric(n, 5001, device="cuda:0")
+    lam = torch.linalg.eigvalsh(A).cpu().numpy()
+    norm2 = float(np.max(np.abs(lam)))
+    rng = np.random.default_rng(5)
+    idx = np.unique(np.concatenate([[0, n - 1], rng.integers(0, n, 30)]))
+    for b in (32, 64, 256):
+        Ab = A.clone()
+        d, e, *_ = trid.sytrd_2stage(Ab, b, nb=min(16, b), k=1024, want_vectors=False)
+        w = sampled_eigs(d.cpu().numpy(), e.cpu().numpy(), idx)
+        assert np.max(np.abs(w - lam[idx])) <= 1e-12 * norm2, b
+
+
+def test_probe_gates_detect_a_wrong_reflector(dev):
+    """The probe estimator is sensitive: flipping one BC scalar breaks G1 by orders of magnitude."""
+    n, b = 2048, 64
+    A = trid_gen.random_symmetric(n, 7, device="cuda:0")
+    A0 = A.clone()
+    d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=16, k=256)
+    g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b)
+    assert g1 <= 1e-14 and g2 <= 1e-14
+    tau2[len(tau2) // 2] *= -1.0
+    g1b, g2b = probe_gates(A0, A, d, e, tau1, V2, tau2, b)
+    assert g1b > 1e-10
