@@ -83,9 +83,20 @@ int64_t max_symm_part(int64_t n, int b) {
   return best;
 }
 
+// largest split-K partial footprint of the skinny engine GEMMs (M = m, N = b, K <= 2k)
+int64_t max_skinny_part(int64_t n, int b, int k) {
+  int64_t best = 0;
+  for (int64_t j = 0; j + b + 1 < n; j += b) {
+    const int64_t m = n - j - b;
+    const int64_t e = (int64_t)ws_skinny_splits(m, b, 2 * (int64_t)k) * m * b;
+    if (e > best) best = e;
+  }
+  return best;
+}
+
 struct DbbrWork {
   double *Y, *Z, *W, *X, *T, *U1, *U2, *S, *part, *red;
-  unsigned* bar;
+  unsigned *bar, *sem;
   int64_t part_elems;
   size_t bytes;
 };
@@ -104,10 +115,13 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
   int64_t pe = max_symm_part(n, b);
   const int64_t tn = (int64_t)32 * k * b;  // split-K partials of the tall reductions
   if (pe < tn) pe = tn;
+  const int64_t sk = max_skinny_part(n, b, k);   // next-panel update / corrections split-K
+  if (pe < sk) pe = sk;
   w.part_elems = pe;
   w.part = c.take<double>((size_t)pe);
   w.red = (double*)c.take<char>(panel_red_bytes(b));
   w.bar = c.take<unsigned>(64);
+  w.sem = c.take<unsigned>(1024);
   w.bytes = c.off;
   return w;
 }
@@ -120,7 +134,7 @@ namespace trid {
 cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
                     const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U1,
                     double* U2, int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems,
-                    cudaStream_t st) {
+                    unsigned* sem, cudaStream_t st) {
   cudaError_t e;
   ProfScope ps(PROF_ZY, st);
   if (nprev > 0) {
@@ -129,7 +143,7 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
     g.M = nprev; g.N = kk; g.K[0] = m; g.A[0] = Zprev; g.lda[0] = ldyz; g.B[0] = Wp; g.ldb[0] = ldw;
     g.C = U1; g.ldc = ldu; g.alpha = 1.0; g.beta = 0.0;
     g.splits = pick_splits(nprev, kk, m, TILE_64x64, part_elems);
-    g.part = part; g.part_ld = nprev; g.part_stride = nprev * kk;
+    g.part = part; g.part_ld = nprev; g.part_stride = nprev * kk; g.sem = sem;
     if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
     g.A[0] = Yprev; g.C = U2;
     if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
@@ -139,6 +153,9 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
     h.A[0] = Yprev; h.lda[0] = ldyz; h.B[0] = U1; h.ldb[0] = ldu; h.K[0] = nprev;
     h.A[1] = Zprev; h.lda[1] = ldyz; h.B[1] = U2; h.ldb[1] = ldu; h.K[1] = nprev;
     h.alpha = -1.0; h.beta = 1.0; h.Cin = X; h.ldcin = ldx; h.C = X; h.ldc = ldx;
+    h.splits = ws_skinny_splits(m, kk, 2 * nprev);
+    if ((int64_t)h.splits * m * kk > part_elems) h.splits = 1;
+    h.part = part; h.part_ld = m; h.part_stride = m * kk;
     if ((e = gemm_ws(h, OP_N, st)) != cudaSuccess) return e;
   }
   // S = W^T X
@@ -146,7 +163,7 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
   s.M = kk; s.N = kk; s.K[0] = m; s.A[0] = Wp; s.lda[0] = ldw; s.B[0] = X; s.ldb[0] = ldx;
   s.C = S; s.ldc = lds; s.alpha = 1.0; s.beta = 0.0;
   s.splits = pick_splits(kk, kk, m, TILE_64x64, part_elems);
-  s.part = part; s.part_ld = kk; s.part_stride = (int64_t)kk * kk;
+  s.part = part; s.part_ld = kk; s.part_stride = (int64_t)kk * kk; s.sem = sem;
   if ((e = gemm(s, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
   // Z_p = X - 1/2 Y_p S
   GemmArgs z;
@@ -161,14 +178,15 @@ namespace {
 cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const double* Wp, int64_t ldw,
                      const double* Yp, const double* Yprev, const double* Zprev, int64_t ldyz, int64_t nprev,
                      double* Zp, double* X, int64_t ldx, double* U1, double* U2, int64_t ldu, double* S, int64_t lds,
-                     double* part, int64_t part_elems, cudaStream_t st) {
+                     double* part, int64_t part_elems, unsigned* sem, cudaStream_t st) {
   cudaError_t e;
   {
     ProfScope ps(PROF_SYMM, st);
     e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
   }
   if (e != cudaSuccess) return e;
-  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U1, U2, ldu, S, lds, part, part_elems, st);
+  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U1, U2, ldu, S, lds, part, part_elems, sem,
+                 st);
 }
 
 int check_common(int64_t n, const void* A, int64_t lda, int b) {
@@ -322,6 +340,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
   if (!dwork) return -8;
   DbbrWork w = carve_dbbr(dwork, n, b, k);
   if (dwork_bytes < w.bytes) return TRID_ERR_WORKSPACE;
+  TRID_CUDA_TRY(cudaMemsetAsync(w.sem, 0, sizeof(unsigned) * 1024, stream));
   const int64_t ld = n;  // Y, Z, W, X leading dimension
   for (int64_t i = 0; i + b + 1 < n; i += k) {                     // l.1
     int64_t ncols = 0, jlast = i;
@@ -345,7 +364,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
       }
       // Z builder against the implicitly updated trailing matrix (R4e)
       TRID_CUDA_TRY(zy_panel(m, kk, A + o + o * lda, lda, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ld,
-                             w.U1, w.U2, k, w.S, b, w.part, w.part_elems, stream));
+                             w.U1, w.U2, k, w.S, b, w.part, w.part_elems, w.sem, stream));
       ncols += kk;                                                  // l.6
       jlast = j;
       const int64_t jn = j + b;
@@ -358,6 +377,9 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
         g.alpha = -1.0; g.beta = 1.0;
         g.C = A + o + o * lda; g.ldc = lda; g.Cin = g.C; g.ldcin = lda;
         g.lower = 1; g.diag_off = 0;
+        g.splits = ws_skinny_splits(m, b, 2 * ncols);
+        if ((int64_t)g.splits * m * b > w.part_elems) g.splits = 1;
+        g.part = w.part; g.part_ld = m; g.part_stride = m * b;
         ProfScope ps(PROF_NEXT, stream);
         TRID_CUDA_TRY(gemm_ws(g, OP_T, stream));
       }

@@ -590,6 +590,13 @@ __global__ void __launch_bounds__(NTH, 3 - NBUF) bc_fast_kernel(BcArgs a) {
 //         then frees the buffer (empty[buf]).  It never waits on another CTA, so publication cannot be
 //         held up by this CTA's own prefetch (no cycle through the predecessor chain).
 // Step/sweep ids travel with the buffer (info[buf]); s < 0 terminates all roles.
+// debug trace (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1, slot k of 16
+#define BCW_TRACE(S, M, K)                                                                          \
+  do {                                                                                              \
+    if (a.trace && ((S) == a.trace_sweep || (S) == a.trace_sweep + 1) && (M) < 1024)                \
+      a.trace[(((S)-a.trace_sweep) * 1024 + (M)) * 16 + (K)] = gtimer();                            \
+  } while (0)
+
 template <int B, int NTH>
 __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
   constexpr int TPR = NTH / (2 * B);
@@ -640,6 +647,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         }
         info_s[bi] = s;
         info_m[bi] = (int)m;
+        BCW_TRACE(s, m, 7);
         const int64_t r0 = s + 1 + m * b;
         const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
         const int L = (int)(r1 - r0 + 1);
@@ -649,10 +657,12 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
           if (m == 0) wait_geq(a.prog + (s - 1), 1);
           wait_geq(a.prog_full + (s - 1), (int)(m + 1));
         }
+        BCW_TRACE(s, m, 8);
         fence_proxy_async_global();
         if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
         if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
         if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        BCW_TRACE(s, m, 9);
         fence_proxy_async_global();
         bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &full[bi]);
       }
@@ -672,11 +682,14 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
       const int L = (int)(r1 - r0 + 1);
       double* win = sm + bi * wsz;
+      BCW_TRACE(s, m, 3);
       bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
       bulk_commit();
       bulk_wait_all();
+      BCW_TRACE(s, m, 4);
       fence_proxy_async_global();
       st_release_s32(a.prog + s, m + 1);
+      BCW_TRACE(s, m, 5);
       mbar_wait(&colsb[bi], ph);
       if (L > 1) {
         bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
@@ -685,6 +698,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         fence_proxy_async_global();
       }
       st_release_s32(a.prog_full + s, m + 1);
+      BCW_TRACE(s, m, 6);
       mbar_arrive(&empty[bi]);
     }
   }
@@ -702,6 +716,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       return;
     }
     const int64_t m = info_m[bi];
+    if (tid == 0) BCW_TRACE(s, m, 0);
     const int64_t off = bc_offset(n, b, s);
     const int64_t r0 = s + 1 + m * b;
     const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
@@ -828,7 +843,10 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
     if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
     fence_proxy_async_smem();
     cbar();
-    if (tid == 0) mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
+    if (tid == 0) {
+      BCW_TRACE(s, m, 1);
+      mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
+    }
     if (L2 > 0 && h2.tau != 0.0 && isO) {
       const double vni = vn[r - L];
       const double tv = h2.tau * vni;
@@ -845,7 +863,10 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       if (tid == 0) a.tau2[off + m] = tau;
     }
     cbar();
-    if (tid == 0) mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
+    if (tid == 0) {
+      BCW_TRACE(s, m, 2);
+      mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
+    }
     tau = tau_next;
   }
 }

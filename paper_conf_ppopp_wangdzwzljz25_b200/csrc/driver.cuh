@@ -10,7 +10,7 @@ namespace trid {
 cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
                     const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U1,
                     double* U2, int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems,
-                    cudaStream_t st);
+                    unsigned* sem, cudaStream_t st);
 
 // Band pack into compact BC storage from "element (c+o, c) at X[o + c*cs]" (full A: cs = lda+1; LAPACK lower
 // band storage: cs = ldab).

@@ -195,6 +195,32 @@ __global__ void __launch_bounds__(WGM* WGN * 32, (BM * BN <= 4096 ? 3 : 2)) gemm
           }
         }
       }
+  if (a.splits > 1 && a.sem) {
+    // the last split to finish this tile reduces all partials in fixed order z = 0..splits-1 (deterministic;
+    // saves the separate reduction launch).  The counter is reset for the next launch.
+    __shared__ int s_last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned* cnt = a.sem + (a.tri ? (int64_t)blockIdx.x : (int64_t)blockIdx.y * gridDim.x + blockIdx.x);
+      const unsigned prev = atomicAdd(cnt, 1u);
+      s_last = prev == (unsigned)a.splits - 1u;
+      if (s_last) *cnt = 0u;
+    }
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      for (int e = threadIdx.x; e < BM * BN; e += WGM * WGN * 32) {
+        const int64_t r = m0 + e % BM, c = n0 + e / BM;
+        if (r >= a.M || c >= a.N || (a.lower && r + a.diag_off < c)) continue;
+        double sum = 0.0;
+        for (int q = 0; q < a.splits; ++q) sum += __ldcg(a.part + q * a.part_stride + r + c * a.part_ld);
+        double v = a.alpha * sum;
+        if (a.beta != 0.0) v += a.beta * a.Cin[r + c * a.ldcin];
+        a.C[r + c * a.ldc] = v;
+      }
+    }
+  }
 }
 
 __global__ void reduce_partials_kernel(GemmArgs a) {
@@ -263,7 +289,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
   else if (opA == OP_N && opB == OP_T) e = launch_ops<OP_N, OP_T>(a, tile, st);
   else if (opA == OP_T && opB == OP_N) e = launch_ops<OP_T, OP_N>(a, tile, st);
   else e = launch_ops<OP_T, OP_T>(a, tile, st);
-  if (e != cudaSuccess || a.splits == 1) return e;
+  if (e != cudaSuccess || a.splits == 1 || a.sem) return e;
   int64_t total = a.M * a.N;
   int blocks = (int)((total + 255) / 256);
   if (blocks > 4 * kNumSMsB200 * 4) blocks = 4 * kNumSMsB200 * 4;

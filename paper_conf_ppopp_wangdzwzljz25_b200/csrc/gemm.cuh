@@ -36,6 +36,9 @@ struct GemmArgs {
   int splits = 1;
   double* part = nullptr;
   int64_t part_ld = 1, part_stride = 0;
+  // gemm() only: per-tile arrival counters (zero on entry, left zero on exit, >= tiles entries); when set, the
+  // last split of each tile reduces the partials in fixed order (no separate reduction launch)
+  unsigned* sem = nullptr;
   // multi-GPU column map for the lower epilogue mask (gemm_ws only): C's column x is global column
   // cmap(x) = ((x+mg_lofs)/mg_cb*mg_g + mg_q)*mg_cb + (x+mg_lofs)%mg_cb - mg_gofs; mg_g <= 1: identity.
   int mg_g = 1, mg_q = 0, mg_cb = 1;
@@ -63,6 +66,7 @@ int64_t symm_part_elems(int64_t m, int64_t w);
 // Warp-specialized persistent engine (gemm_ws.cu): op(A) = A only; tiles 128x128 (N > 64) / 128x64.
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
 int64_t symm_ws_splits(int64_t m, int64_t w);
+int ws_skinny_splits(int64_t M, int64_t N, int64_t K);
 int64_t symm_ws_part_elems(int64_t m, int64_t w);
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
                     int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);

@@ -521,6 +521,17 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 
+// Split-K for the skinny engine GEMMs (M = trailing rows, N = b, K = 2 x block columns): enough units for
+// ~3 waves of the persistent grid, >= 256 of K per split, <= 16 splits.  Partials: splits * M * N doubles.
+int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {
+  const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
+  int64_t sp = (3 * kNumSMsB200 + tiles - 1) / tiles;
+  const int64_t maxs = K / 256;
+  if (sp > maxs) sp = maxs;
+  if (sp > 16) sp = 16;
+  return sp < 1 ? 1 : (int)sp;
+}
+
 // Strip splits of the SYMM: the persistent grid runs >= ~8 waves of units (tail imbalance <~ 6%);
 // env TRID_SYMM_WAVES overrides (tuning).
 int64_t symm_ws_splits(int64_t m, int64_t w) {

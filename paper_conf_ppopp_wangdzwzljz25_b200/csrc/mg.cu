@@ -282,7 +282,7 @@ struct Carver {
 
 struct MgWork {
   double *Y, *Z, *W, *X, *Xl, *Wl, *Yl, *Zl, *T, *U1, *U2, *S, *pk, *part, *red;
-  unsigned* bar;
+  unsigned *bar, *sem;
   int64_t part_elems;
   size_t bytes;
 };
@@ -290,6 +290,11 @@ struct MgWork {
 MgWork carve_mg(void* base, int64_t n, int b, int k, int g, int q) {
   const int64_t nq = local_cols(n, b, g, q);
   int64_t pe = (int64_t)32 * k * b;
+  for (int64_t j = 0; j + b + 1 < n; j += b) {
+    const int64_t m = n - j - b;
+    const int64_t e = (int64_t)ws_skinny_splits(m, b, 2 * (int64_t)k) * m * b;
+    if (e > pe) pe = e;
+  }
   for (int64_t j = 0; j + b + 1 < n; j += b) {
     const int64_t o = j + b, m = n - o, kk = m < b ? m : b;
     const int64_t nqt = nq - local_before(o, b, g, q);
@@ -318,6 +323,7 @@ MgWork carve_mg(void* base, int64_t n, int b, int k, int g, int q) {
   w.part = c.take<double>((size_t)pe);
   w.red = (double*)c.take<char>(panel_red_bytes(b));
   w.bar = c.take<unsigned>(64);
+  w.sem = c.take<unsigned>(1024);
   w.bytes = c.off;
   return w;
 }
@@ -448,6 +454,7 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
   if (!dwork) return -10;
   MgWork w = carve_mg(dwork, n, b, k, g, q);
   if (dwork_bytes < w.bytes) return TRID_ERR_WORKSPACE;
+  TRID_CUDA_TRY(cudaMemsetAsync(w.sem, 0, sizeof(unsigned) * 1024, st));
   const int64_t ld = n;   // Y, Z, W leading dimension
   int r;
   for (int64_t i = 0; i + b + 1 < n; i += k) {                       // l.1
@@ -498,7 +505,7 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
         if ((r = comm_sum(comm, w.X, ldx * kk, true, 0, st))) return r;   // padding rows ride along unread
       }
       TRID_CUDA_TRY(zy_tail(m, kk, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ldx, w.U1, w.U2, k, w.S, b,
-                            w.part, w.part_elems, st));
+                            w.part, w.part_elems, w.sem, st));
       ncols += kk;                                                  // l.6
       jlast = j;
       const int64_t jn = j + b;
@@ -511,6 +518,9 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
         gn.alpha = -1.0; gn.beta = 1.0;
         gn.C = A + o + local_col(o, b, g) * lda; gn.ldc = lda; gn.Cin = gn.C; gn.ldcin = lda;
         gn.lower = 1; gn.diag_off = 0;
+        gn.splits = ws_skinny_splits(m, b, 2 * ncols);
+        if ((int64_t)gn.splits * m * b > w.part_elems) gn.splits = 1;
+        gn.part = w.part; gn.part_ld = m; gn.part_stride = m * b;
         ProfScope ps(PROF_NEXT, st);
         TRID_CUDA_TRY(gemm_ws(gn, OP_T, st));
       }
