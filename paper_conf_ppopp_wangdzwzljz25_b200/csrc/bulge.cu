@@ -755,7 +755,9 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
       }
       part[hg * 2 * B + r] = acc0 + acc1;
+      if (tid == 0) BCW_TRACE(s, m, 10);
       cbar();
+      if (tid == 0) BCW_TRACE(s, m, 11);
       if (tid < 2 * B) {
         double acc = 0.0;
 #pragma unroll
@@ -763,6 +765,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         pyv[tid] = (tid >= L) ? acc : tau * acc;
       }
       cbar();
+      if (tid == 0) BCW_TRACE(s, m, 12);
       double pv = 0.0;
       for (int i = lane; i < L; i += 32) pv += pyv[i] * v[i];
       pv = warp_sum(pv);
@@ -788,6 +791,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
     }
     cbar();
+    if (tid == 0) BCW_TRACE(s, m, 13);
     double tau_next = 0.0;
     House h2;
     h2.beta = 0.0;
@@ -840,9 +844,11 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       }
     }
     cbar();   // all reads of the raw O(:, 0) done; zv ready
+    if (tid == 0) BCW_TRACE(s, m, 14);
     if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
     fence_proxy_async_smem();
     cbar();
+    if (tid == 0) BCW_TRACE(s, m, 15);
     if (tid == 0) {
       BCW_TRACE(s, m, 1);
       mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it

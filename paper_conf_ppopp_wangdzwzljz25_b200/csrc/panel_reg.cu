@@ -41,7 +41,18 @@ struct PanelRegArgs {
   double* gpart;     // 2 x NC x 2w cluster partials
   unsigned* bar;     // grid barrier counter (zero at launch)
   int rows;          // rows per CTA
+  long long* trace;  // debug (TRID_PANEL_TRACE=m): %globaltimer per column phase, CTAs 0 and G-1
 };
+__device__ __forceinline__ long long pr_gtimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define PR_TRACE(k)                                                                        \
+  do {                                                                                     \
+    if (a.trace && tid == 0 && (g == 0 || g == G - 1) && t < 256)                          \
+      a.trace[((g == 0 ? 0 : 1) * 256 + t) * 8 + (k)] = pr_gtimer();                       \
+  } while (0)
 
 template <int CPW>
 __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_constant__ PanelRegArgs a) {
@@ -79,6 +90,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
   for (int t = 0; t < a.kk; ++t) {
     const int par = t & 1;
     const int wt = t / CPW, ct = t % CPW;
+    PR_TRACE(0);
     // ---- 1. Gram slots of this warp's columns over rows > t, and row-t values
     double acc[CPW];
 #pragma unroll
@@ -130,7 +142,9 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       }
     }
     // ---- 2. cluster reduction through DSMEM (fixed order over the 8 CTAs)
+    PR_TRACE(1);
     cl.sync();
+    PR_TRACE(2);
     {
       // thread -> (slot s = crank + 8*k, member c): 8 lanes per slot
       const int k = tid / PR_CL, c = tid % PR_CL;
@@ -146,6 +160,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     }
     // ---- 3. one grid barrier
     __syncthreads();
+    PR_TRACE(3);
     epoch += 1;
     if (tid == 0) {
       asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar) : "memory");
@@ -155,6 +170,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       (void)ld_acquire_u32(a.bar);
     }
     __syncthreads();
+    PR_TRACE(4);
     // ---- 4. totals over the NC cluster partials, fixed order
     for (int s = tid; s < RS; s += PR_NT) {
       double vals[PR_MAXNC];
@@ -167,6 +183,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       tot[s] = v;
     }
     __syncthreads();
+    PR_TRACE(5);
     // ---- 5. reflector, update, T column
     const House h = make_house(tot[W + t], tot[t]);
 #pragma unroll
@@ -201,6 +218,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       if (tid == 0) a.tau[t] = h.tau;
     }
     __syncthreads();   // everyone is done with xs / tot of column t
+    PR_TRACE(6);
     // next column -> xs
     if (t + 1 < a.kk && warp == (t + 1) / CPW) {
       const int cn = (t + 1) % CPW;
@@ -249,6 +267,12 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   PanelRegArgs a;
   a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);
   a.P = P; a.ldp = ldp; a.tau = tau; a.T = T; a.ldt = ldt; a.Y = Y; a.ldy = ldy; a.gpart = gpart; a.bar = bar;
+  {
+    // trace area: past the cluster partials inside the panel workspace (panel_red_bytes reserves it)
+    static const char* tr = getenv("TRID_PANEL_TRACE");
+    a.trace = (tr && atoll(tr) == m) ? (long long*)(gpart + 2 * (size_t)kNumSMsB200 * 2 * w + 2 * 2 * (size_t)w)
+                                     : nullptr;
+  }
   const size_t smem = sizeof(double) * (size_t)(32 * PR_RL + 2 * 2 * w + 2 * w + w * w);
   // co-resident clusters of 8 (a cluster must fit in one GPC): query once per kernel instantiation
   static int max_clusters[3] = {0, 0, 0};

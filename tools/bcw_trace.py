@@ -46,6 +46,12 @@ out = {
     "body_dep_wait_us (7 -> 8)": np.mean(c[m, 8] - c[m, 7]) / 1e3,
     "step_period_us (cons 0 -> next 0)": np.mean(np.diff(c[2:steps - 3, 0])) / 1e3,
     "link_us (prod 5(m+1) -> cons 5(m))": np.mean(c[m, 5] - p[m + 1, 5]) / 1e3,
+    "c: matvec partial (0 -> 10)": np.mean(c[m, 10] - c[m, 0]) / 1e3,
+    "c: cbar1 (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
+    "c: reduce+cbar2 (11 -> 12)": np.mean(c[m, 12] - c[m, 11]) / 1e3,
+    "c: pv+update+writeback+cbar3 (12 -> 13)": np.mean(c[m, 13] - c[m, 12]) / 1e3,
+    "c: house+z+cbar4 (13 -> 14)": np.mean(c[m, 14] - c[m, 13]) / 1e3,
+    "c: finalize+fence+cbar5 (14 -> 15)": np.mean(c[m, 15] - c[m, 14]) / 1e3,
     "data_ready_gap (cons 0 - max(9 of cons, 2 of cons prev))": np.mean(c[m, 0] - np.maximum(c[m, 9], c[m - 1, 2])) / 1e3,
 }
 print(json.dumps({k: round(float(v), 3) for k, v in out.items()}, indent=1))

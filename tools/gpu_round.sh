@@ -28,7 +28,7 @@ if has full; then
   P8="python tools/prof_run.py --n 8192 --b 64 --k 1024 --nb 16"
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:bc_ -c 1 -o $O/prof_bc8192 $P8 > $O/prof_bc8192.log 2>&1
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:ws_kernel -s 1 -c 1 -o $O/prof_symm $P > $O/prof_symm.log 2>&1
-  timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:ws_kernel<\\(int\\)128, \\(int\\)128' -c 1 -o $O/prof_syr2k $P > $O/prof_syr2k.log 2>&1
+  timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:ws_kernel<\(int\)128, \(int\)128' -c 1 -o $O/prof_syr2k $P > $O/prof_syr2k.log 2>&1
   TRID_PANEL_NOCOOP=1 timeout 900 ncu --set full --clock-control none --import-source on -k regex:panel_reg -s 5 -c 1 -o $O/prof_panel $P > $O/prof_panel.log 2>&1
   timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bc_fast -c 1 -o $O/prof_bc $P > $O/prof_bc.log 2>&1
 fi
