@@ -916,6 +916,287 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
   }
 }
 
+// ---- row-per-thread chase (default for b <= 64) ---------------------------------------------------------
+// One compute thread per window row (2B threads: row r of [D; O], all L <= B columns in registers), plus the
+// LOAD and STORE warps of bc_ws_kernel.  A row's matvec needs no cross-thread reduction, so the path from
+// "last column arrived" to "column 0 published" is: one FMA (the body matvec is done while the last column
+// is in flight), one warp-sum + named barrier (p^T v), the column-0 update, one warp-sum + barrier (|x|^2),
+// the reflector, the stores of column 0 and one barrier before the st.release.  The remaining work (full
+// two-sided update, z = vn^T O by transposed warp butterflies, left application, write-back, V2) follows.
+template <int B>
+__global__ void __launch_bounds__(2 * B + 64, 1) bc_row_kernel(BcArgs a) {
+  constexpr int NT = 2 * B;           // compute threads = window rows
+  constexpr int NWc = NT / 32;        // compute warps
+  extern __shared__ __align__(16) double sm[];
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int lda1 = ldab - 1;
+  const int64_t n = a.n;
+  const int wsz = B * ldab;
+  double* colb = sm + 2 * wsz;        // 2 x ldab: column s of a sweep's step 0, per buffer
+  double* vb = colb + 2 * ldab;       // 2 x B   (v / vn)
+  double* pyv = vb + 2 * B;           // 2B      p (D rows) | y (O rows)
+  double* zs = pyv + 2 * B;           // NWc x B z partials
+  double* wred = zs + NWc * B;        // 2 x NWc warp partials (p^T v, |x|^2) + 2 (alpha)
+  __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], colsb[2];
+  __shared__ int64_t info_s[2];
+  __shared__ int info_m[2];
+  if (tid == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&lastb[i], 1);
+      mbar_init(&empty[i], 1);
+      mbar_init(&colsb[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp == NWc) {
+    // ============================== LOAD warp (as bc_ws_kernel) ==============================
+    if (lane != 0) return;
+    uint32_t it = 0;
+    for (;;) {
+      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
+      const bool done = s > n - 3;
+      const int64_t nst = done ? 1 : bc_steps(n, b, s);
+      const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+      for (int64_t m = 0; m < nst; ++m, ++it) {
+        const int bi = it & 1;
+        if (it >= 2) mbar_wait(&empty[bi], ((it >> 1) - 1) & 1u);
+        if (done) {
+          info_s[bi] = -1;
+          mbar_arrive(&full[bi]);
+          return;
+        }
+        info_s[bi] = s;
+        info_m[bi] = (int)m;
+        BCW_TRACE(s, m, 7);
+        const int64_t r0 = s + 1 + m * b;
+        const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+        const int L = (int)(r1 - r0 + 1);
+        double* win = sm + bi * wsz;
+        mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
+        mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
+        if (s > 0) {
+          if (m == 0) wait_geq(a.prog + (s - 1), 1);
+          wait_geq(a.prog_full + (s - 1), (int)(m + 1));
+        }
+        BCW_TRACE(s, m, 8);
+        fence_proxy_async_global();
+        if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
+        if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
+        if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        BCW_TRACE(s, m, 9);
+        fence_proxy_async_global();
+        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
+      }
+    }
+  }
+  if (warp == NWc + 1) {
+    // ============================== STORE warp: columns 1..L-1 ==============================
+    if (lane != 0) return;
+    for (uint32_t it = 0;; ++it) {
+      const int bi = it & 1;
+      const unsigned ph = (it >> 1) & 1u;
+      mbar_wait(&colsb[bi], ph);
+      const int64_t s = info_s[bi];
+      if (s < 0) return;
+      const int m = info_m[bi];
+      const int64_t r0 = s + 1 + (int64_t)m * b;
+      const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
+      const int L = (int)(r1 - r0 + 1);
+      double* win = sm + bi * wsz;
+      BCW_TRACE(s, m, 3);
+      if (L > 1) {
+        bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
+        bulk_commit();
+        bulk_wait_all();
+        fence_proxy_async_global();
+      }
+      st_release_s32(a.prog_full + s, m + 1);
+      BCW_TRACE(s, m, 6);
+      mbar_arrive(&empty[bi]);
+    }
+  }
+  // ============================== compute threads: one window row each ==============================
+  auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NT) : "memory"); };
+  const int r = tid;
+  double tau = 0.0;
+  int64_t off = 0;
+  for (uint32_t it = 0;; ++it) {
+    const int bi = it & 1;
+    const unsigned ph = (it >> 1) & 1u;
+    mbar_wait(&full[bi], ph);
+    const int64_t s = info_s[bi];
+    if (s < 0) {
+      if (tid == 0) mbar_arrive(&colsb[bi]);
+      return;
+    }
+    const int m = info_m[bi];
+    if (tid == 0) BCW_TRACE(s, m, 0);
+    const int64_t r0 = s + 1 + (int64_t)m * b;
+    const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
+    const int L = (int)(r1 - r0 + 1);
+    const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
+    const int L2 = (int)(r2 - r1);
+    double* win = sm + bi * wsz;
+    double* v = vb + (m & 1) * B;
+    double* vn = vb + ((m & 1) ^ 1) * B;
+    if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
+      off = bc_offset(n, b, s);
+      const double* col = colb + bi * ldab + 1;
+      double sig = 0.0;
+      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
+      sig = warp_sum(sig);
+      const House hh = make_house(col[0], sig);
+      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
+      if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
+      tau = hh.tau;
+      cbar();
+    }
+    const bool active = r < L + L2;
+    const bool isD = r < L;
+    // ---- row r of [D; O] into registers; element (r, j) lives at win[j*lda1 + r] for j <= r (lower D and
+    // all of O) and at win[r*lda1 + j] for j > r (upper D = column r).  Only (r >= L-1, j = L-1) is in the
+    // separately loaded last column.
+    double e[B];
+    double acc0 = 0.0, acc1 = 0.0;
+#pragma unroll
+    for (int j = 0; j < B; ++j) {
+      double x = 0.0;
+      if (active && j < L && !(j == L - 1 && r >= L - 1)) x = win[j <= r ? j * lda1 + r : r * lda1 + j];
+      e[j] = x;
+      if (j & 1) acc1 = fma(x, v[j], acc1);
+      else acc0 = fma(x, v[j], acc0);
+    }
+    mbar_wait(&lastb[bi], ph);
+    if (tid == 0) BCW_TRACE(s, m, 10);
+    if (active && r >= L - 1) {
+#pragma unroll
+      for (int j = 0; j < B; ++j)
+        if (j == L - 1) {
+          e[j] = win[j * lda1 + r];
+          acc0 = fma(e[j], v[j], acc0);
+        }
+    }
+    const double vr = isD ? v[r] : 0.0;
+    const double raw0 = r < ldab ? win[r] : 0.0;   // column 0 (for rows past the window: untouched band)
+    double pr = 0.0, hp = 0.0, wr = 0.0;
+    if (tau != 0.0) {
+      pr = isD ? tau * (acc0 + acc1) : (acc0 + acc1);   // p_r = tau (D v)_r  |  y_r = (O v)_r
+      if (active) pyv[r] = pr;
+      double t = isD ? pr * vr : 0.0;
+      t = warp_sum(t);
+      if (lane == 0) wred[warp] = t;
+      cbar();
+      double pv = 0.0;
+#pragma unroll
+      for (int w = 0; w < NWc; ++w) pv += wred[w];
+      hp = 0.5 * tau * pv;
+      wr = fma(-hp, vr, pr);   // w_r = p_r - 1/2 tau (p^T v) v_r
+    }
+    if (tid == 0) BCW_TRACE(s, m, 11);
+    // ---- column 0 of the updated window, the next reflector from x = O(:, 0), publish column 0
+    double x0 = e[0];
+    if (tau != 0.0) {
+      if (isD) {
+        const double w0 = fma(-hp, v[0], pyv[0]);
+        x0 = fma(-wr, v[0], fma(-vr, w0, x0));
+      } else if (active) {
+        x0 = fma(-tau * pr, v[0], x0);
+      }
+    }
+    {
+      double t = (active && r > L) ? x0 * x0 : 0.0;
+      t = warp_sum(t);
+      if (lane == 0) wred[NWc + warp] = t;
+      if (r == L) wred[2 * NWc] = x0;
+    }
+    cbar();
+    House h2;
+    h2.beta = 0.0;
+    h2.tau = 0.0;
+    h2.scale = 0.0;
+    if (L2 > 0) {
+      double sg = 0.0;
+#pragma unroll
+      for (int w = 0; w < NWc; ++w) sg += wred[NWc + w];
+      h2 = make_house(wred[2 * NWc], sg);
+    }
+    if (r < ldab) {
+      const double outv = isD ? x0 : (active ? (r == L ? h2.beta : 0.0) : raw0);
+      __stcg(a.band + r0 * ldab + r, outv);
+    }
+    if (tid == 0) BCW_TRACE(s, m, 12);
+    cbar();
+    if (tid == 0) {
+      st_release_s32(a.prog + s, m + 1);   // cumulative over the compute threads' stores (bar.sync above)
+      BCW_TRACE(s, m, 1);
+      BCW_TRACE(s, m, 5);
+    }
+    // ---- the rest of the two-sided update (D) and the right update of the bulge (O)
+    if (tau != 0.0) {
+      if (isD) {
+#pragma unroll
+        for (int j = 0; j < B; ++j) {
+          const double vj = v[j];
+          const double wj = fma(-hp, vj, pyv[j]);
+          e[j] = fma(-wr, vj, fma(-vr, wj, e[j]));
+        }
+      } else if (active) {
+        const double ty = tau * pr;
+#pragma unroll
+        for (int j = 0; j < B; ++j) e[j] = fma(-ty, v[j], e[j]);
+      }
+    }
+    // e[0] now equals x0 (same arithmetic); next reflector vn (rows L..L+L2-1)
+    const bool isO = active && !isD;
+    const double vnr = isO ? (r == L ? 1.0 : h2.scale * e[0]) : 0.0;
+    if (r >= L && r - L < B) vn[r - L] = vnr;
+    // ---- write back columns 1..L-1 (lower D, all of O)
+    if (active) {
+#pragma unroll
+      for (int j = 1; j < B; ++j)
+        if (j < L && j <= r) win[j * lda1 + r] = e[j];
+    }
+    cbar();
+    if (tid == 0) BCW_TRACE(s, m, 13);
+    // ---- z_j = vn^T O(:, j), j >= 1 (thread j walks column j of O), then left-apply to O(:, 1:)
+    if (L2 > 0 && h2.tau != 0.0) {
+      if (r >= 1 && r < L) {
+        const double* oc = win + r * lda1 + L;   // O(i, r) = oc[i]
+        double z0 = 0.0, z1 = 0.0;
+        int i = 0;
+        for (; i + 1 < L2; i += 2) {
+          z0 = fma(vn[i], oc[i], z0);
+          z1 = fma(vn[i + 1], oc[i + 1], z1);
+        }
+        if (i < L2) z0 = fma(vn[i], oc[i], z0);
+        zs[r] = z0 + z1;
+      }
+      cbar();
+      if (isO) {
+        const double tv = h2.tau * vnr;
+#pragma unroll
+        for (int j = 1; j < B; ++j)
+          if (j < L) win[j * lda1 + r] = fma(-tv, zs[j], e[j]);
+      }
+    }
+    fence_proxy_async_smem();
+    if (a.V2) {
+      double* vd = a.V2 + (off + m) * a.vs;
+      for (int i = tid; i < a.vs; i += NT) vd[i] = i < L ? v[i] : 0.0;
+      if (tid == 0) a.tau2[off + m] = tau;
+    }
+    cbar();
+    if (tid == 0) {
+      BCW_TRACE(s, m, 2);
+      mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
+    }
+    tau = h2.tau;
+  }
+}
+
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
   const size_t flags = sizeof(int) * (size_t)(2 * n + 128);
@@ -967,8 +1248,17 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       // single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel.
       const int B = beff <= 32 ? 32 : 64;
       const char* force = getenv("TRID_BC_FORCE");
-      const int variant = force ? force[0] - '0' : 3;
-      if (variant == 3) {
+      const int variant = force ? force[0] - '0' : 4;
+      if (variant == 4) {
+        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B +
+                                              (size_t)(2 * B / 32) * B + 2 * (2 * B / 32) + 8);
+        const void* fn = B == 32 ? (const void*)bc_row_kernel<32> : (const void*)bc_row_kernel<64>;
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int64_t grid = kNumSMsB200;
+        if (grid > n - 2) grid = n - 2;
+        if (B == 32) bc_row_kernel<32><<<(unsigned)grid, 64 + 64, smem, st>>>(a);
+        else bc_row_kernel<64><<<(unsigned)grid, 128 + 64, smem, st>>>(a);
+      } else if (variant == 3) {
         const int nth = B == 32 ? 256 : 512;
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B + B +
                                               (size_t)(nth / (2 * B)) * 2 * B + 2 * B + 8);

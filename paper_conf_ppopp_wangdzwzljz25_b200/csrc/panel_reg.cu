@@ -54,6 +54,22 @@ __device__ __forceinline__ long long pr_gtimer() {
       a.trace[((g == 0 ? 0 : 1) * 256 + t) * 8 + (k)] = pr_gtimer();                       \
   } while (0)
 
+// T(0:c, c) = -tau_c T(0:c, 0:c) (V(:, 0:c)^T v_c), T(c, c) = tau_c (dlarft forward columnwise);
+// Dm[c*W + p] = v_c^T v_p.  Reads T columns < c (complete: a __syncthreads separates the calls).
+__device__ __forceinline__ void t_column(double* Ts, const double* Dm, const double* taus, int c, int W, int tid) {
+  for (int q2 = tid; q2 < W; q2 += PR_NT) {
+    double v = 0.0;
+    if (q2 < c) {
+      double sacc = 0.0;
+      for (int p = q2; p < c; ++p) sacc += Ts[q2 + p * W] * Dm[c * W + p];
+      v = -taus[c] * sacc;
+    } else if (q2 == c) {
+      v = taus[c];
+    }
+    Ts[q2 + c * W] = v;
+  }
+}
+
 template <int CPW>
 __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_constant__ PanelRegArgs a) {
   constexpr int W = 8 * CPW;
@@ -63,6 +79,9 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
   double* mypart = xs + 32 * PR_RL;   // 2 x RS   (double-buffered per column parity)
   double* tot = mypart + 2 * RS;      // RS
   double* Ts = tot + RS;              // W x W    (CTA 0)
+  double* Dm = Ts + W * W;            // W x W    (CTA 0): v_t^T v_p, p < t, for the T factor
+  double* taus = Dm + W * W;          // W        (CTA 0)
+  double* tot2 = taus + W;            // RS       second half of the partial sums
   cg::cluster_group cl = cg::this_cluster();
   const int g = blockIdx.x, G = gridDim.x, NC = G / PR_CL;
   const int crank = (int)cl.block_rank(), cid = g / PR_CL;
@@ -162,8 +181,10 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     __syncthreads();
     PR_TRACE(3);
     epoch += 1;
+    if (tid == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar) : "memory");
+    // CTA 0 builds the T column of the previous reflector while the other CTAs arrive (off the critical path)
+    if (g == 0 && t > 0) t_column(Ts, Dm, taus, t - 1, W, tid);
     if (tid == 0) {
-      asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar) : "memory");
       const unsigned target = epoch * (unsigned)G;
       while (ld_relaxed_u32(a.bar) < target) {
       }
@@ -172,16 +193,24 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     __syncthreads();
     PR_TRACE(4);
     // ---- 4. totals over the NC cluster partials, fixed order
-    for (int s = tid; s < RS; s += PR_NT) {
-      double vals[PR_MAXNC];
+    {
+      // 2 threads per slot: cluster partials [0, NC/2) and [NC/2, NC), each summed in order, then added
+      const int s = tid % RS, hh = tid / RS, q0 = hh ? NC / 2 : 0, q1 = hh ? NC : NC / 2;
+      constexpr int HALF = (PR_MAXNC + 1) / 2;
+      if (tid < 2 * RS) {
+        double vals[HALF];
 #pragma unroll
-      for (int q = 0; q < PR_MAXNC; ++q) vals[q] = q < NC ? __ldcg(a.gpart + ((size_t)par * NC + q) * RS + s) : 0.0;
-      double v = vals[0];
+        for (int q = 0; q < HALF; ++q)
+          vals[q] = q0 + q < q1 ? __ldcg(a.gpart + ((size_t)par * NC + q0 + q) * RS + s) : 0.0;
+        double v = vals[0];
 #pragma unroll
-      for (int q = 1; q < PR_MAXNC; ++q)
-        if (q < NC) v += vals[q];
-      tot[s] = v;
+        for (int q = 1; q < HALF; ++q)
+          if (q0 + q < q1) v += vals[q];
+        (hh ? tot2 : tot)[s] = v;
+      }
     }
+    __syncthreads();
+    for (int s = tid; s < RS; s += PR_NT) tot[s] += tot2[s];
     __syncthreads();
     PR_TRACE(5);
     // ---- 5. reflector, update, T column
@@ -204,18 +233,12 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       }
     }
     if (g == 0) {
-      for (int q2 = tid; q2 < W; q2 += PR_NT) {
-        double v = 0.0;
-        if (q2 < t) {
-          double sacc = 0.0;
-          for (int p = q2; p < t; ++p) sacc += Ts[q2 + p * W] * (tot[W + p] + h.scale * tot[p]);
-          v = -h.tau * sacc;
-        } else if (q2 == t) {
-          v = h.tau;
-        }
-        Ts[q2 + t * W] = v;
+      // v_t^T v_p = P(t, p) + scale * sum_{r>t} x_r P(r, p) for p < t (the Gram row), saved for the T column
+      for (int p = tid; p < t; p += PR_NT) Dm[t * W + p] = tot[W + p] + h.scale * tot[p];
+      if (tid == 0) {
+        taus[t] = h.tau;
+        a.tau[t] = h.tau;
       }
-      if (tid == 0) a.tau[t] = h.tau;
     }
     __syncthreads();   // everyone is done with xs / tot of column t
     PR_TRACE(6);
@@ -231,6 +254,10 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
         xs[lane + 32 * q] = v;
       }
     }
+    __syncthreads();
+  }
+  if (g == 0 && a.kk > 0) {
+    t_column(Ts, Dm, taus, a.kk - 1, W, tid);
     __syncthreads();
   }
   // ---- write back R/V, explicit Y, T
@@ -273,7 +300,7 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
     a.trace = (tr && atoll(tr) == m) ? (long long*)(gpart + 2 * (size_t)kNumSMsB200 * 2 * w + 2 * 2 * (size_t)w)
                                      : nullptr;
   }
-  const size_t smem = sizeof(double) * (size_t)(32 * PR_RL + 2 * 2 * w + 2 * w + w * w);
+  const size_t smem = sizeof(double) * (size_t)(32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
   // co-resident clusters of 8 (a cluster must fit in one GPC): query once per kernel instantiation
   static int max_clusters[3] = {0, 0, 0};
   const int wi = w == 16 ? 0 : (w == 32 ? 1 : 2);

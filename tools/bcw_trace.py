@@ -43,12 +43,11 @@ out = {
     "link_us (prod 5(m+1) -> cons 5(m))": np.mean(c[m, 5] - p[m + 1, 5]) / 1e3,
     "c: body matvec + last-col wait (0 -> 10)": np.mean(c[m, 10] - c[m, 0]) / 1e3,
     "c: last col (cons 9 -> 10)": np.mean(c[m, 10] - c[m, 9]) / 1e3,
-    "c: part+cbar1 (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
-    "c: reduce+cbar2 (11 -> 12)": np.mean(c[m, 12] - c[m, 11]) / 1e3,
-    "c: update+col0 house+store (12 -> 13)": np.mean(c[m, 13] - c[m, 12]) / 1e3,
-    "c: gbar+release (13 -> 1)": np.mean(c[m, 1] - c[m, 13]) / 1e3,
-    "c: writeback+cbar3 (1 -> 14)": np.mean(c[m, 14] - c[m, 1]) / 1e3,
-    "c: z+cbar4 (14 -> 15)": np.mean(c[m, 15] - c[m, 14]) / 1e3,
+    "c: matvec end + pv bar (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
+    "c: col0 + sigma bar + house + stores (11 -> 12)": np.mean(c[m, 12] - c[m, 11]) / 1e3,
+    "c: bar + release (12 -> 1)": np.mean(c[m, 1] - c[m, 12]) / 1e3,
+    "c: update + writeback + bar (1 -> 13)": np.mean(c[m, 13] - c[m, 1]) / 1e3,
+    "c: z + left-apply + V2 + bar (13 -> 2)": np.mean(c[m, 2] - c[m, 13]) / 1e3,
     "data_ready_gap (cons 0 - max(9 of cons, 2 of cons prev))": np.mean(c[m, 0] - np.maximum(c[m, 9], c[m - 1, 2])) / 1e3,
 }
 print(json.dumps({k: round(float(v), 3) for k, v in out.items()}, indent=1))
