@@ -615,23 +615,19 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
   double* pyv = vb + 2 * B;                  // 2B
   double* zv = pyv + 2 * B;                  // B
   double* part = zv + B;                     // TPR x 2B
-  double* c0 = part + TPR * 2 * B;           // 2B: updated column 0 (raw bulge column x in rows >= L)
-  double* hsm = c0 + 2 * B;                  // 4: next reflector (beta, tau, scale)
-  // full[]: window columns 0..L-2 (+ column s at step 0); lastb[]: the window's last column
-  __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], colsb[2];
+  __shared__ __align__(8) uint64_t full[2], empty[2], col0b[2], colsb[2];
   __shared__ int64_t info_s[2];
   __shared__ int info_m[2];
   if (tid == 0) {
     for (int i = 0; i < 2; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&lastb[i], 1);
       mbar_init(&empty[i], 1);
+      mbar_init(&col0b[i], 1);
       mbar_init(&colsb[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
-
   if (warp == NW) {
     // ============================== LOAD warp ==============================
     if (lane != 0) return;
@@ -656,8 +652,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
         const int L = (int)(r1 - r0 + 1);
         double* win = sm + bi * wsz;
-        mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
-        mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
+        mbar_arrive_expect_tx(&full[bi], (unsigned)((L + (m == 0 ? 1 : 0)) * ldab * 8));
         if (s > 0) {
           if (m == 0) wait_geq(a.prog + (s - 1), 1);
           wait_geq(a.prog_full + (s - 1), (int)(m + 1));
@@ -669,17 +664,17 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
         BCW_TRACE(s, m, 9);
         fence_proxy_async_global();
-        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
+        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &full[bi]);
       }
     }
   }
   if (warp == NW + 1) {
-    // ============================== STORE warp: columns 1..L-1 ==============================
+    // ============================== STORE warp ==============================
     if (lane != 0) return;
     for (uint32_t it = 0;; ++it) {
       const int bi = it & 1;
       const unsigned ph = (it >> 1) & 1u;
-      mbar_wait(&colsb[bi], ph);
+      mbar_wait(&col0b[bi], ph);
       const int64_t s = info_s[bi];
       if (s < 0) return;
       const int m = info_m[bi];
@@ -688,6 +683,14 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
       const int L = (int)(r1 - r0 + 1);
       double* win = sm + bi * wsz;
       BCW_TRACE(s, m, 3);
+      bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
+      bulk_commit();
+      bulk_wait_all();
+      BCW_TRACE(s, m, 4);
+      fence_proxy_async_global();
+      st_release_s32(a.prog + s, m + 1);
+      BCW_TRACE(s, m, 5);
+      mbar_wait(&colsb[bi], ph);
       if (L > 1) {
         bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
         bulk_commit();
@@ -700,13 +703,8 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
     }
   }
   // ============================== compute warps ==============================
-  // Critical path of a step (the next sweep waits for it): last column arrives -> finish the matvec ->
-  // column 0 of the updated window -> next reflector -> column 0 stored to global by column group 0 and
-  // published (st.release prog).  Everything else (the rest of the update, z = vn^T O, the left
-  // application, V2) runs after the publication.
   const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
   auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NTH) : "memory"); };
-  auto gbar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(2 * B) : "memory"); };   // column group 0
   double tau = 0.0;
   for (uint32_t it = 0;; ++it) {
     const int bi = it & 1;
@@ -714,7 +712,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
     mbar_wait(&full[bi], ph);
     const int64_t s = info_s[bi];
     if (s < 0) {
-      if (tid == 0) mbar_arrive(&colsb[bi]);   // wake the STORE warp so it can see the end
+      if (tid == 0) mbar_arrive(&col0b[bi]);   // wake the STORE warp so it can see the end
       return;
     }
     const int64_t m = info_m[bi];
@@ -743,36 +741,21 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
     const bool isO = r >= L && active;
     const int lo_base = j0 * lda1 + r;
     const int hi_base = r * lda1 + j0;
-    // the last window column (j = L-1) is stored in the separately loaded column only for rows r >= L-1;
-    // for rows r < L-1 the symmetric element D(r, L-1) = D(L-1, r) sits in (prefetched) column r
-    const int jl = L - 1 - j0;
-    const bool has_last = jl >= 0 && jl < CPT && r >= L - 1;
     double e[CPT];
-    double acc0 = 0.0, acc1 = 0.0;
 #pragma unroll
     for (int jj = 0; jj < CPT; ++jj) {
       const int j = j0 + jj;
-      e[jj] = (has_last && jj == jl) ? 0.0 : win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
+      e[jj] = win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
     }
     if (tau != 0.0) {
+      double acc0 = 0.0, acc1 = 0.0;
 #pragma unroll
       for (int jj = 0; jj < CPT; jj += 2) {
         acc0 = fma(e[jj], v[j0 + jj], acc0);
         acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
       }
-    }
-    mbar_wait(&lastb[bi], ph);
-    if (tid == 0) BCW_TRACE(s, m, 9 + 1);
-    if (has_last) {
-#pragma unroll
-      for (int jj = 0; jj < CPT; ++jj)
-        if (jj == jl) {
-          e[jj] = win[lo_base + jj * lda1];
-          acc0 = fma(e[jj], v[j0 + jj], acc0);
-        }
-    }
-    if (tau != 0.0) {
       part[hg * 2 * B + r] = acc0 + acc1;
+      if (tid == 0) BCW_TRACE(s, m, 10);
       cbar();
       if (tid == 0) BCW_TRACE(s, m, 11);
       if (tid < 2 * B) {
@@ -802,52 +785,23 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         }
       }
     }
-    // ---- column 0 (column group 0): next reflector from x = O(:, 0), store, publish
-    double tau_next = 0.0;
-    if (hg == 0) {
-      c0[r] = e[0];   // rows >= L + L2 hold untouched band entries
-      gbar();
-      House h2;
-      h2.beta = 0.0;
-      h2.tau = 0.0;
-      h2.scale = 0.0;
-      if (L2 > 0) {
-        double sg = 0.0;
-        for (int i = 1 + lane; i < L2; i += 32) sg = fma(c0[L + i], c0[L + i], sg);
-        sg = warp_sum(sg);
-        h2 = make_house(c0[L], sg);
-        if (tid == 0) {
-          hsm[0] = h2.beta;
-          hsm[1] = h2.tau;
-          hsm[2] = h2.scale;
-        }
-      }
-      const double outv = (L2 > 0 && r >= L && r < L + L2) ? (r == L ? h2.beta : 0.0) : e[0];
-      if (r < ldab) __stcg(a.band + r0 * ldab + r, outv);
-      if (tid == 0) BCW_TRACE(s, m, 13);
-      gbar();
-      if (tid == 0) {
-        st_release_s32(a.prog + s, (int)(m + 1));   // cumulative over the group's stores (bar.sync above)
-        BCW_TRACE(s, m, 1);
-        BCW_TRACE(s, m, 5);
-      }
-    }
-    // ---- write back the lower part of D and all of O (column 0 keeps the raw x for the z pass)
 #pragma unroll
     for (int jj = 0; jj < CPT; ++jj) {
       const int j = j0 + jj;
       if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
     }
-    cbar();   // hsm (next reflector) and the updated window visible to all
-    if (tid == 0) BCW_TRACE(s, m, 14);
+    cbar();
+    if (tid == 0) BCW_TRACE(s, m, 13);
+    double tau_next = 0.0;
     House h2;
     h2.beta = 0.0;
     h2.tau = 0.0;
     h2.scale = 0.0;
     if (L2 > 0) {
-      h2.beta = hsm[0];
-      h2.tau = hsm[1];
-      h2.scale = hsm[2];
+      double sg = 0.0;
+      for (int i = 1 + lane; i < L2; i += 32) sg = fma(win[L + i], win[L + i], sg);
+      sg = warp_sum(sg);
+      h2 = make_house(win[L], sg);
       tau_next = h2.tau;
       if (tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : h2.scale * win[L + tid]) : 0.0;
     }
@@ -889,9 +843,16 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
         }
       }
     }
-    cbar();   // zv ready; all reads of the raw x done
+    cbar();   // all reads of the raw O(:, 0) done; zv ready
+    if (tid == 0) BCW_TRACE(s, m, 14);
+    if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
+    fence_proxy_async_smem();
+    cbar();
     if (tid == 0) BCW_TRACE(s, m, 15);
-    // ---- left-apply the next reflector to O(:, 1:)
+    if (tid == 0) {
+      BCW_TRACE(s, m, 1);
+      mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
+    }
     if (L2 > 0 && h2.tau != 0.0 && isO) {
       const double vni = vn[r - L];
       const double tv = h2.tau * vni;
@@ -916,7 +877,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
   }
 }
 
-// ---- row-per-thread chase (default for b <= 64) ---------------------------------------------------------
+// ---- row-per-thread chase (experimental, TRID_BC_FORCE=4; measured slower: see DESIGN.md sec. 5) ---------------------------------------------------------
 // One compute thread per window row (2B threads: row r of [D; O], all L <= B columns in registers), plus the
 // LOAD and STORE warps of bc_ws_kernel.  A row's matvec needs no cross-thread reduction, so the path from
 // "last column arrived" to "column 0 published" is: one FMA (the body matvec is done while the last column
@@ -1248,7 +1209,7 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       // single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel.
       const int B = beff <= 32 ? 32 : 64;
       const char* force = getenv("TRID_BC_FORCE");
-      const int variant = force ? force[0] - '0' : 4;
+      const int variant = force ? force[0] - '0' : 3;
       if (variant == 4) {
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B +
                                               (size_t)(2 * B / 32) * B + 2 * (2 * B / 32) + 8);
@@ -1261,7 +1222,7 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       } else if (variant == 3) {
         const int nth = B == 32 ? 256 : 512;
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B + B +
-                                              (size_t)(nth / (2 * B)) * 2 * B + 2 * B + 8);
+                                              (size_t)(nth / (2 * B)) * 2 * B + 8);
         const void* fn = B == 32 ? (const void*)bc_ws_kernel<32, 256> : (const void*)bc_ws_kernel<64, 512>;
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int64_t grid = kNumSMsB200;

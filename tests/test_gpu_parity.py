@@ -132,9 +132,10 @@ def test_bulge_chase_parity(n, b, dev):
     assert np.max(np.abs(V2.cpu().numpy() - V_o), initial=0) <= 1e-9
 
 
-@pytest.mark.parametrize("variant", ["1", "2"])
+@pytest.mark.parametrize("variant", ["1", "2", "3", "4"])
 def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
-    """Both B=64 kernels (2 CTAs/SM single buffer, 1 CTA/SM double buffer) against the oracle."""
+    """Every B=64 chase kernel (1: bc_fast 2 CTAs/SM single buffer, 2: bc_fast double buffer, 3: warp-specialized
+    bc_ws (default), 4: row-per-thread bc_row) against the oracle, bitwise reproducible."""
     monkeypatch.setenv("TRID_BC_FORCE", variant)
     n, b = 700, 64
     Bm = band_from_lower(trid_gen.random_symmetric_np(n, 99), b)

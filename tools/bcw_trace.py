@@ -36,18 +36,22 @@ m = np.arange(2, steps - 3)
 p, c = tr[0], tr[1]          # sweep s (producer), s+1 (consumer)
 out = {
     "poll_detect_us (prod 5 -> cons 9)": np.mean(c[m, 9] - p[m + 1, 5]) / 1e3,
+    "last_col_load_us (cons 9 -> 0)": np.mean(c[m, 0] - c[m, 9]) / 1e3,
+    "compute_to_col0_us (0 -> 1)": np.mean(c[m, 1] - c[m, 0]) / 1e3,
+    "store_wakeup_us (1 -> 3)": np.mean(c[m, 3] - c[m, 1]) / 1e3,
+    "col0_store_complete_us (3 -> 4)": np.mean(c[m, 4] - c[m, 3]) / 1e3,
+    "release_us (4 -> 5)": np.mean(c[m, 5] - c[m, 4]) / 1e3,
     "col0_to_step_end_us (1 -> 2)": np.mean(c[m, 2] - c[m, 1]) / 1e3,
     "cols_store_us (2 -> 6)": np.mean(c[m, 6] - c[m, 2]) / 1e3,
     "body_dep_wait_us (7 -> 8)": np.mean(c[m, 8] - c[m, 7]) / 1e3,
     "step_period_us (cons 0 -> next 0)": np.mean(np.diff(c[2:steps - 3, 0])) / 1e3,
     "link_us (prod 5(m+1) -> cons 5(m))": np.mean(c[m, 5] - p[m + 1, 5]) / 1e3,
-    "c: body matvec + last-col wait (0 -> 10)": np.mean(c[m, 10] - c[m, 0]) / 1e3,
-    "c: last col (cons 9 -> 10)": np.mean(c[m, 10] - c[m, 9]) / 1e3,
-    "c: matvec end + pv bar (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
-    "c: col0 + sigma bar + house + stores (11 -> 12)": np.mean(c[m, 12] - c[m, 11]) / 1e3,
-    "c: bar + release (12 -> 1)": np.mean(c[m, 1] - c[m, 12]) / 1e3,
-    "c: update + writeback + bar (1 -> 13)": np.mean(c[m, 13] - c[m, 1]) / 1e3,
-    "c: z + left-apply + V2 + bar (13 -> 2)": np.mean(c[m, 2] - c[m, 13]) / 1e3,
+    "c: matvec partial (0 -> 10)": np.mean(c[m, 10] - c[m, 0]) / 1e3,
+    "c: cbar1 (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
+    "c: reduce+cbar2 (11 -> 12)": np.mean(c[m, 12] - c[m, 11]) / 1e3,
+    "c: pv+update+writeback+cbar3 (12 -> 13)": np.mean(c[m, 13] - c[m, 12]) / 1e3,
+    "c: house+z+cbar4 (13 -> 14)": np.mean(c[m, 14] - c[m, 13]) / 1e3,
+    "c: finalize+fence+cbar5 (14 -> 15)": np.mean(c[m, 15] - c[m, 14]) / 1e3,
     "data_ready_gap (cons 0 - max(9 of cons, 2 of cons prev))": np.mean(c[m, 0] - np.maximum(c[m, 9], c[m - 1, 2])) / 1e3,
 }
 print(json.dumps({k: round(float(v), 3) for k, v in out.items()}, indent=1))
