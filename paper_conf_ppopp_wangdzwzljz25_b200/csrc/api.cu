@@ -120,7 +120,7 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
   w.part_elems = pe;
   w.part = c.take<double>((size_t)pe);
   w.red = (double*)c.take<char>(panel_red_bytes(b));
-  w.bar = c.take<unsigned>(64);
+  w.bar = c.take<unsigned>(256);   // panel grid-barrier counters (8 x 128 B)
   w.sem = c.take<unsigned>(1024);
   w.bytes = c.off;
   return w;
@@ -436,7 +436,7 @@ int trid_panel_qr_bufsize(int64_t m, int w, size_t* dwork_bytes) {
   if (w < 1) return -2;
   if (!dwork_bytes) return -3;
   if (w > TRID_MAX_B) return TRID_ERR_UNSUPPORTED;
-  *dwork_bytes = align256(panel_red_bytes(w)) + 256;
+  *dwork_bytes = align256(panel_red_bytes(w)) + 1024;
   return TRID_SUCCESS;
 }
 
@@ -455,7 +455,7 @@ int trid_panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double*
   if (!dwork || dwork_bytes < need) return TRID_ERR_WORKSPACE;
   Carver c(dwork);
   double* red = (double*)c.take<char>(panel_red_bytes(w));
-  unsigned* bar = c.take<unsigned>(64);
+  unsigned* bar = c.take<unsigned>(256);
   TRID_CUDA_TRY(panel_qr(m, w, P, ldp, tau, T, ldt, Y, ldy, red, bar, stream));
   return TRID_SUCCESS;
 }

@@ -322,7 +322,7 @@ MgWork carve_mg(void* base, int64_t n, int b, int k, int g, int q) {
   w.part_elems = pe;
   w.part = c.take<double>((size_t)pe);
   w.red = (double*)c.take<char>(panel_red_bytes(b));
-  w.bar = c.take<unsigned>(64);
+  w.bar = c.take<unsigned>(256);   // panel grid-barrier counters (8 x 128 B)
   w.sem = c.take<unsigned>(1024);
   w.bytes = c.off;
   return w;

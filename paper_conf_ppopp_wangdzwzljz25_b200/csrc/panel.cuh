@@ -6,7 +6,7 @@
 
 namespace trid {
 
-// Panel QR + T + explicit Y (see panel_qr.cu).  red: panel_red_bytes(w) bytes; bar: one zeroed word.
+// Panel QR + T + explicit Y (see panel_qr.cu).  red: panel_red_bytes(w) bytes; bar: 256 words (zeroed by the launcher).
 size_t panel_red_bytes(int w);
 cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
                      int64_t ldy, double* red, unsigned* bar, cudaStream_t st);

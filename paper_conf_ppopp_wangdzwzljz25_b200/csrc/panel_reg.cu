@@ -27,6 +27,7 @@ constexpr int PR_NT = 256;   // 8 warps
 constexpr int PR_CL = 4;     // cluster size (33 co-resident 4-CTA clusters at 1 CTA/SM on B200)
 constexpr int PR_MAXNC = 40; // max clusters
 constexpr int PR_RL = 8;     // rows per lane (rows per CTA <= 256)
+constexpr int PR_NBAR = 8;   // grid-barrier counters (128 B apart)
 
 struct PanelRegArgs {
   int64_t m;
@@ -75,8 +76,8 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
   constexpr int W = 8 * CPW;
   constexpr int RS = 2 * W;
   extern __shared__ __align__(16) double sm[];
-  double* xs = sm;                    // rows of this CTA: column t (broadcast)
-  double* mypart = xs + 32 * PR_RL;   // 2 x RS   (double-buffered per column parity)
+  double* xsb = sm;                   // 2 x rows of this CTA: column t (broadcast), by column parity
+  double* mypart = xsb + 2 * 32 * PR_RL;   // 2 x RS   (double-buffered per column parity)
   double* tot = mypart + 2 * RS;      // RS
   double* Ts = tot + RS;              // W x W    (CTA 0)
   double* Dm = Ts + W * W;            // W x W    (CTA 0): v_t^T v_p, p < t, for the T factor
@@ -98,17 +99,17 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     for (int c = 0; c < CPW; ++c)
       P[q][c] = (i < nr && j0 + c < a.w) ? a.P[(rlo + i) + (int64_t)(j0 + c) * a.ldp] : 0.0;
   }
-  // column 0 -> xs
+  // column 0 -> xs (buffer 0)
   if (warp == 0) {
 #pragma unroll
-    for (int q = 0; q < PR_RL; ++q) xs[lane + 32 * q] = P[q][0];
+    for (int q = 0; q < PR_RL; ++q) xsb[lane + 32 * q] = P[q][0];
   }
   unsigned epoch = 0;
   __syncthreads();
 
   for (int t = 0; t < a.kk; ++t) {
     const int par = t & 1;
-    const int wt = t / CPW, ct = t % CPW;
+    const double* xs = xsb + par * 32 * PR_RL;
     PR_TRACE(0);
     // ---- 1. Gram slots of this warp's columns over rows > t, and row-t values
     double acc[CPW];
@@ -181,14 +182,16 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     __syncthreads();
     PR_TRACE(3);
     epoch += 1;
-    if (tid == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar) : "memory");
+    // grid barrier on PR_NBAR counters (128 B apart) so the G arrivals do not serialise on one L2 line
+    if (tid == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar + 32 * (g % PR_NBAR)) : "memory");
     // CTA 0 builds the T column of the previous reflector while the other CTAs arrive (off the critical path)
     if (g == 0 && t > 0) t_column(Ts, Dm, taus, t - 1, W, tid);
-    if (tid == 0) {
-      const unsigned target = epoch * (unsigned)G;
-      while (ld_relaxed_u32(a.bar) < target) {
+    if (tid < PR_NBAR) {
+      const unsigned target = epoch * (unsigned)((G - tid + PR_NBAR - 1) / PR_NBAR);
+      const unsigned* cnt = a.bar + 32 * tid;
+      while (ld_relaxed_u32(cnt) < target) {
       }
-      (void)ld_acquire_u32(a.bar);
+      (void)ld_acquire_u32(cnt);
     }
     __syncthreads();
     PR_TRACE(4);
@@ -215,6 +218,9 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     PR_TRACE(5);
     // ---- 5. reflector, update, T column
     const House h = make_house(tot[W + t], tot[t]);
+    double tw[CPW];   // -tau * w_j for this warp's columns (w_j = v^T P(:, j))
+#pragma unroll
+    for (int c = 0; c < CPW; ++c) tw[c] = -h.tau * fma(h.scale, tot[j0 + c], tot[W + j0 + c]);
 #pragma unroll
     for (int q = 0; q < PR_RL; ++q) {
       const int i = lane + 32 * q;
@@ -225,8 +231,7 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
       for (int c = 0; c < CPW; ++c) {
         const int j = j0 + c;
         if (j > t) {
-          const double wj = tot[W + j] + h.scale * tot[j];
-          P[q][c] = fma(-h.tau * wj, vr, P[q][c]);
+          P[q][c] = fma(tw[c], vr, P[q][c]);
         } else if (j == t) {
           P[q][c] = r > t ? vr : h.beta;
         }
@@ -240,10 +245,10 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
         a.tau[t] = h.tau;
       }
     }
-    __syncthreads();   // everyone is done with xs / tot of column t
     PR_TRACE(6);
-    // next column -> xs
+    // next column -> the other xs buffer (its previous readers finished before this column's grid barrier)
     if (t + 1 < a.kk && warp == (t + 1) / CPW) {
+      double* xn = xsb + (par ^ 1) * 32 * PR_RL;
       const int cn = (t + 1) % CPW;
 #pragma unroll
       for (int q = 0; q < PR_RL; ++q) {
@@ -251,10 +256,10 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
 #pragma unroll
         for (int c = 0; c < CPW; ++c)
           if (c == cn) v = P[q][c];
-        xs[lane + 32 * q] = v;
+        xn[lane + 32 * q] = v;
       }
     }
-    __syncthreads();
+    __syncthreads();   // xs of column t+1 visible; all reads of tot / xs of column t done
   }
   if (g == 0 && a.kk > 0) {
     t_column(Ts, Dm, taus, a.kk - 1, W, tid);
@@ -300,7 +305,7 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
     a.trace = (tr && atoll(tr) == m) ? (long long*)(gpart + 2 * (size_t)kNumSMsB200 * 2 * w + 2 * 2 * (size_t)w)
                                      : nullptr;
   }
-  const size_t smem = sizeof(double) * (size_t)(32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
+  const size_t smem = sizeof(double) * (size_t)(2 * 32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
   // co-resident clusters of 8 (a cluster must fit in one GPC): query once per kernel instantiation
   static int max_clusters[3] = {0, 0, 0};
   const int wi = w == 16 ? 0 : (w == 32 ? 1 : 2);
@@ -330,7 +335,7 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   if (G < PR_CL) G = PR_CL;
   a.rows = (int)((m + G - 1) / G);
   if (a.rows > 32 * PR_RL) return cudaErrorInvalidConfiguration;   // caller checks panel_reg_supported
-  cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), st);
+  cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned) * 32 * PR_NBAR, st);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)G);
