@@ -95,7 +95,7 @@ int64_t max_skinny_part(int64_t n, int b, int k) {
 }
 
 struct DbbrWork {
-  double *Y, *Z, *W, *X, *T, *U1, *U2, *S, *part, *red;
+  double *Y, *Z, *W, *X, *T, *U, *S, *part, *red;
   unsigned *bar, *sem;
   int64_t part_elems;
   size_t bytes;
@@ -109,11 +109,10 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
   w.W = c.take<double>((size_t)n * b);
   w.X = c.take<double>((size_t)n * b);
   w.T = c.take<double>((size_t)b * b);
-  w.U1 = c.take<double>((size_t)k * b);
-  w.U2 = c.take<double>((size_t)k * b);
+  w.U = c.take<double>((size_t)2 * k * b);   // [Z_<^T W; Y_<^T W], ld 2k
   w.S = c.take<double>((size_t)b * b);
   int64_t pe = max_symm_part(n, b);
-  const int64_t tn = (int64_t)32 * k * b;  // split-K partials of the tall reductions
+  const int64_t tn = (int64_t)64 * k * b;  // split-K partials of the tall reductions (2k x b stacked)
   if (pe < tn) pe = tn;
   const int64_t sk = max_skinny_part(n, b, k);   // next-panel update / corrections split-K
   if (pe < sk) pe = sk;
@@ -132,20 +131,21 @@ namespace trid {
 // ---- the Z builder after the SYMM (a3): corrections for the block's earlier panels (R4e), S = W^T X,
 // Z_p = X - 1/2 Y_p S (Eq. (1)).  X (m x kk, ld ldx) holds A_blk W_p on entry and is updated.
 cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
-                    const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U1,
-                    double* U2, int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems,
-                    unsigned* sem, cudaStream_t st) {
+                    const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U,
+                    int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems, unsigned* sem,
+                    cudaStream_t st) {
   cudaError_t e;
   ProfScope ps(PROF_ZY, st);
   if (nprev > 0) {
-    // U1 = Z_<^T W, U2 = Y_<^T W   (TN, K = m, deterministic split-K)
+    // [U1; U2] = [Z_<^T W; Y_<^T W]   (TN, K = m, deterministic split-K; one launch, stacked rows)
+    double* U1 = U;
+    double* U2 = U + nprev;
     GemmArgs g;
-    g.M = nprev; g.N = kk; g.K[0] = m; g.A[0] = Zprev; g.lda[0] = ldyz; g.B[0] = Wp; g.ldb[0] = ldw;
-    g.C = U1; g.ldc = ldu; g.alpha = 1.0; g.beta = 0.0;
-    g.splits = pick_splits(nprev, kk, m, TILE_64x64, part_elems);
-    g.part = part; g.part_ld = nprev; g.part_stride = nprev * kk;
-    if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
-    g.A[0] = Yprev; g.C = U2;
+    g.M = 2 * nprev; g.N = kk; g.K[0] = m; g.A[0] = Zprev; g.lda[0] = ldyz; g.B[0] = Wp; g.ldb[0] = ldw;
+    g.A2m = Yprev; g.msplit = nprev;
+    g.C = U; g.ldc = ldu; g.alpha = 1.0; g.beta = 0.0;
+    g.splits = pick_splits(2 * nprev, kk, m, TILE_64x64, part_elems);
+    g.part = part; g.part_ld = 2 * nprev; g.part_stride = 2 * nprev * kk;
     if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
     // X -= Y_< U1 + Z_< U2
     GemmArgs h;
@@ -175,7 +175,7 @@ namespace {
 // ---- the Z builder for one panel (a3): X = A W (SYMM); then zy_tail
 cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const double* Wp, int64_t ldw,
                      const double* Yp, const double* Yprev, const double* Zprev, int64_t ldyz, int64_t nprev,
-                     double* Zp, double* X, int64_t ldx, double* U1, double* U2, int64_t ldu, double* S, int64_t lds,
+                     double* Zp, double* X, int64_t ldx, double* U, int64_t ldu, double* S, int64_t lds,
                      double* part, int64_t part_elems, unsigned* sem, cudaStream_t st) {
   cudaError_t e;
   {
@@ -183,8 +183,7 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
     e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
   }
   if (e != cudaSuccess) return e;
-  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U1, U2, ldu, S, lds, part, part_elems, sem,
-                 st);
+  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U, ldu, S, lds, part, part_elems, sem, st);
 }
 
 int check_common(int64_t n, const void* A, int64_t lda, int b) {
@@ -362,7 +361,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
       }
       // Z builder against the implicitly updated trailing matrix (R4e)
       TRID_CUDA_TRY(zy_panel(m, kk, A + o + o * lda, lda, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ld,
-                             w.U1, w.U2, k, w.S, b, w.part, w.part_elems, w.sem, stream));
+                             w.U, 2 * k, w.S, b, w.part, w.part_elems, w.sem, stream));
       ncols += kk;                                                  // l.6
       jlast = j;
       const int64_t jn = j + b;

@@ -877,6 +877,372 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
   }
 }
 
+// ---- v6: warp-specialized chase with a short column-0 path (default for b <= 64) ------------------------
+// Same roles, window mapping and step arithmetic as bc_ws_kernel, reorganised around the chain that bounds
+// the chase (Delta per sweep = step period + link, link = predecessor's column 0 -> our column 0):
+//   * the last window column (sweep s-1's freshly published column 0) lands on its own mbarrier (lastb);
+//     it contributes to one row of D v (the diagonal D(L-1,L-1)) and to every row of O v, so the body
+//     matvec (columns 0..L-2) and its cross-group reduction run while it is in flight;
+//   * column 0 of the step is then produced by 2B threads (one per window row) with ONE named barrier:
+//     p = tau D v / y = O v are completed with one FMA, p^T v and |x(1:)|^2 (x = the right-updated O(:,0))
+//     are warp-summed together, the reflector of x is formed once (its beta/tau/scale go to shared memory
+//     for the rest of the step), and the new D(:,0), beta e1 are written to a column-0 staging buffer the
+//     STORE warp publishes (prog) while the full two-sided update, the z pass and the left application of
+//     the step continue on all compute threads;
+//   * the predecessor counters are polled without back-off (one lane per CTA).
+// The arithmetic of every element is the same expression as in bc_ws_kernel (fixed-order sums): bitwise
+// reproducible, independent of scheduling.
+__device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
+  while (ld_relaxed_s32(p) < need) {
+  }
+  (void)ld_acquire_s32(p);
+}
+
+template <int B, int NTH>
+__global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
+  constexpr int TPR = NTH / (2 * B);
+  constexpr int CPT = B / TPR;
+  constexpr int RW = (2 * B) / 32;   // warps of the column-0 path (column group 0)
+  constexpr int NW = NTH / 32;
+  constexpr int CPW = B / NW;
+  static_assert(CPW == 4 || CPW == 8, "z-pass butterfly assumes 4 or 8 columns per warp");
+  extern __shared__ __align__(16) double sm[];
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int lda1 = ldab - 1;
+  const int64_t n = a.n;
+  const int wsz = B * ldab;
+  double* colb = sm + 2 * wsz;               // 2 x ldab: column s of a sweep's step 0, per buffer
+  double* c0s = colb + 2 * ldab;             // 2 x ldab: column-0 staging, per buffer
+  double* vb = c0s + 2 * ldab;               // 2 x B   (v / vn)
+  double* pyv = vb + 2 * B;                  // 2B
+  double* zv = pyv + 2 * B;                  // B
+  double* red = zv + B;                      // 2*RW warp partials, x0, beta/tau/scale (16)
+  double* part = red + 16;                   // TPR x 2B
+  __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], col0b[2], colsb[2], c0done[2];
+  __shared__ int64_t info_s[2];
+  __shared__ int info_m[2];
+  if (tid == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&lastb[i], 1);
+      mbar_init(&empty[i], 1);
+      mbar_init(&col0b[i], 2 * B);
+      mbar_init(&colsb[i], 1);
+      mbar_init(&c0done[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == NW) {
+    // ============================== LOAD warp ==============================
+    if (lane != 0) return;
+    uint32_t it = 0;
+    for (;;) {
+      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
+      const bool done = s > n - 3;
+      const int64_t nst = done ? 1 : bc_steps(n, b, s);
+      const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+      for (int64_t m = 0; m < nst; ++m, ++it) {
+        const int bi = it & 1;
+        if (it >= 2) mbar_wait(&empty[bi], ((it >> 1) - 1) & 1u);
+        if (done) {
+          info_s[bi] = -1;
+          mbar_arrive(&full[bi]);
+          return;
+        }
+        info_s[bi] = s;
+        info_m[bi] = (int)m;
+        BCW_TRACE(s, m, 7);
+        const int64_t r0 = s + 1 + m * b;
+        const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+        const int L = (int)(r1 - r0 + 1);
+        double* win = sm + bi * wsz;
+        mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
+        mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
+        if (s > 0) {
+          if (m == 0) wait_geq_spin(a.prog + (s - 1), 1);
+          wait_geq_spin(a.prog_full + (s - 1), (int)(m + 1));
+        }
+        BCW_TRACE(s, m, 8);
+        fence_proxy_async_global();
+        if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
+        if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
+        if (s > 0) wait_geq_spin(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        BCW_TRACE(s, m, 9);
+        fence_proxy_async_global();
+        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
+      }
+    }
+  }
+  if (warp == NW + 1) {
+    // ============================== STORE0 warp: column 0 (the chain) ==============================
+    if (lane != 0) return;
+    for (uint32_t it = 0;; ++it) {
+      const int bi = it & 1;
+      const unsigned ph = (it >> 1) & 1u;
+      mbar_wait(&col0b[bi], ph);
+      const int64_t s = info_s[bi];
+      if (s < 0) return;
+      const int m = info_m[bi];
+      const int64_t r0 = s + 1 + (int64_t)m * b;
+      BCW_TRACE(s, m, 3);
+      bulk_s2g(a.band + r0 * ldab, c0s + bi * ldab, (unsigned)(ldab * 8));
+      bulk_commit();
+      bulk_wait_all();
+      BCW_TRACE(s, m, 4);
+      fence_proxy_async_global();
+      st_release_s32(a.prog + s, m + 1);
+      BCW_TRACE(s, m, 5);
+      mbar_arrive(&c0done[bi]);
+    }
+  }
+  if (warp == NW + 2) {
+    // ============================== STORE1 warp: columns 1..L-1 ==============================
+    // frees the window buffer as soon as the bulk store has READ it; prog_full after the writes landed
+    if (lane != 0) return;
+    for (uint32_t it = 0;; ++it) {
+      const int bi = it & 1;
+      const unsigned ph = (it >> 1) & 1u;
+      mbar_wait(&colsb[bi], ph);
+      const int64_t s = info_s[bi];
+      if (s < 0) return;
+      const int m = info_m[bi];
+      const int64_t r0 = s + 1 + (int64_t)m * b;
+      const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
+      const int L = (int)(r1 - r0 + 1);
+      double* win = sm + bi * wsz;
+      if (L > 1) {
+        bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
+        bulk_commit();
+        bulk_wait_read();
+      }
+      mbar_wait(&c0done[bi], ph);   // column 0's staging buffer was read too
+      mbar_arrive(&empty[bi]);
+      if (L > 1) {
+        bulk_wait_all();
+        fence_proxy_async_global();
+      }
+      st_release_s32(a.prog_full + s, m + 1);
+      BCW_TRACE(s, m, 6);
+    }
+  }
+  // ============================== compute warps ==============================
+  const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
+  const bool c0path = tid < 2 * B;   // column group 0 = one thread per window row
+  auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NTH) : "memory"); };
+  auto c0bar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(2 * B) : "memory"); };
+  double tau = 0.0;
+  for (uint32_t it = 0;; ++it) {
+    const int bi = it & 1;
+    const unsigned ph = (it >> 1) & 1u;
+    mbar_wait(&full[bi], ph);
+    const int64_t s = info_s[bi];
+    if (s < 0) {
+      if (c0path) mbar_arrive(&col0b[bi]);   // wake the STORE warps so they can see the end
+      if (tid == 0) mbar_arrive(&colsb[bi]);
+      return;
+    }
+    const int64_t m = info_m[bi];
+    if (tid == 0) BCW_TRACE(s, m, 0);
+    const int64_t r0 = s + 1 + m * b;
+    const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+    const int L = (int)(r1 - r0 + 1);
+    const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
+    const int L2 = (int)(r2 - r1);
+    double* win = sm + bi * wsz;
+    double* v = vb + (m & 1) * B;
+    double* vn = vb + ((m & 1) ^ 1) * B;
+    if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
+      const double* col = colb + bi * ldab + 1;
+      double sig = 0.0;
+      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
+      sig = warp_sum(sig);
+      const House hh = make_house(col[0], sig);
+      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
+      if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
+      tau = hh.tau;
+      cbar();
+    }
+    const bool active = r < L + L2;
+    const bool isO = r >= L && active;
+    const int lo_base = j0 * lda1 + r;
+    const int hi_base = r * lda1 + j0;
+    // the element (r, L-1) of rows r >= L-1 lives in the last column (in flight on lastb)
+    const int jd = L - 1 - j0;
+    const bool defer = r >= L - 1 && jd >= 0 && jd < CPT;
+    double e[CPT];
+    double acc0 = 0.0, acc1 = 0.0;
+#pragma unroll
+    for (int jj = 0; jj < CPT; ++jj) {
+      const int j = j0 + jj;
+      const bool ok = j < L && !(defer && jj == jd);
+      e[jj] = ok ? win[j <= r ? lo_base + jj * lda1 : hi_base + jj] : 0.0;
+    }
+    const double2* v2 = reinterpret_cast<const double2*>(v + j0);
+#pragma unroll
+    for (int jj = 0; jj < CPT; jj += 2) {
+      const double2 vv = v2[jj / 2];
+      acc0 = fma(e[jj], vv.x, acc0);
+      acc1 = fma(e[jj + 1], vv.y, acc1);
+    }
+    part[hg * 2 * B + r] = acc0 + acc1;
+    cbar();   // (1) body partials of D v / O v
+    if (tid == 0) BCW_TRACE(s, m, 10);
+    if (c0path) {
+      // ---------------- column-0 path: thread r = window row r ----------------
+      double acc = 0.0;
+#pragma unroll
+      for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + r];
+      mbar_wait(&lastb[bi], ph);
+      if (tid == 0) BCW_TRACE(s, m, 11);
+      if (active && r >= L - 1) acc = fma(win[(L - 1) * lda1 + r], v[L - 1], acc);
+      const double py = (r >= L) ? acc : tau * acc;   // p_r = tau (D v)_r  |  y_r = (O v)_r
+      pyv[r] = py;
+      const double vr = r < L ? v[r] : 0.0;
+      const double raw = r < ldab ? win[r] : 0.0;        // column 0, row r0 + r
+      double x = 0.0;
+      if (isO) x = fma(-(tau * py), v[0], raw);         // right-updated O(r-L, 0)
+      double tD = r < L ? py * vr : 0.0;
+      double tO = (isO && r > L) ? x * x : 0.0;
+      tD = warp_sum(tD);
+      tO = warp_sum(tO);
+      if (lane == 0) {
+        red[warp] = tD;
+        red[RW + warp] = tO;
+      }
+      if (r == L) red[2 * RW] = x;
+      c0bar();
+      double pv = 0.0, sg = 0.0;
+#pragma unroll
+      for (int w = 0; w < RW; ++w) {
+        pv += red[w];
+        sg += red[RW + w];
+      }
+      const double hp = 0.5 * tau * pv;
+      double val = raw;
+      if (r < L) {
+        const double w0 = fma(-hp, v[0], pyv[0]);
+        const double wr = fma(-hp, vr, py);
+        val = fma(-wr, v[0], fma(-vr, w0, raw));
+      } else if (isO) {
+        val = 0.0;
+        if (r == L) {
+          const House h2 = make_house(red[2 * RW], sg);
+          val = h2.beta;
+          red[2 * RW + 1] = h2.beta;
+          red[2 * RW + 2] = h2.tau;
+          red[2 * RW + 3] = h2.scale;
+        }
+      }
+      if (r < ldab) c0s[bi * ldab + r] = val;
+      fence_proxy_async_smem();
+      mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
+      if (tid == 0) BCW_TRACE(s, m, 1);
+    }
+    if (defer) {
+      mbar_wait(&lastb[bi], ph);
+      const double el = win[(L - 1) * lda1 + r];
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj)
+        if (jj == jd) e[jj] = el;
+    }
+    cbar();   // (2) pyv, p^T v partials, the next reflector's scalars
+    if (tid == 0) BCW_TRACE(s, m, 12);
+    double tau_next = 0.0, hscale = 0.0;
+    if (L2 > 0) {
+      tau_next = red[2 * RW + 2];
+      hscale = red[2 * RW + 3];
+    }
+    if (tau != 0.0) {
+      double pv = 0.0;
+#pragma unroll
+      for (int w = 0; w < RW; ++w) pv += red[w];
+      const double hp = 0.5 * tau * pv;
+      if (isO) {
+        const double ty = tau * pyv[r];
+#pragma unroll
+        for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
+      } else {
+        const double vr = r < L ? v[r] : 0.0;
+        const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
+#pragma unroll
+        for (int jj = 0; jj < CPT; ++jj) {
+          const double vj = v[j0 + jj];
+          const double wj = fma(-hp, vj, pyv[j0 + jj]);
+          e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
+        }
+      }
+    }
+#pragma unroll
+    for (int jj = 0; jj < CPT; ++jj) {
+      const int j = j0 + jj;
+      if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
+    }
+    cbar();   // (3) right-updated window in shared memory
+    if (tid == 0) BCW_TRACE(s, m, 13);
+    if (L2 > 0 && tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : hscale * win[L + tid]) : 0.0;
+    if (L2 > 0 && tau_next != 0.0 && L > 1) {
+      const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
+      const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
+      double c[CPW];
+#pragma unroll
+      for (int q = 0; q < CPW; ++q) {
+        const int j = warp + q * NW;
+        double acc = 0.0;
+        if (j >= 1 && j < L) {
+          const int ob = j * lda1 + L;
+          if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
+          if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
+        }
+        c[q] = acc;
+      }
+      int qbase = 0;
+#pragma unroll
+      for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
+        const bool up = (lane & o) != 0;
+#pragma unroll
+        for (int i = 0; i < K / 2; ++i) {
+          const double send = up ? c[i] : c[i + K / 2];
+          const double keep = up ? c[i + K / 2] : c[i];
+          c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+        }
+        if (up) qbase += K / 2;
+      }
+      constexpr int LV = CPW == 4 ? 2 : 3;
+      double f = c[0];
+#pragma unroll
+      for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+      if ((lane & ((32 >> LV) - 1)) == 0) {
+        const int j = warp + qbase * NW;
+        if (j >= 1 && j < L) zv[j] = fma(hscale, f, win[j * lda1 + L]);
+      }
+    }
+    cbar();   // (4) z = vn^T O(:, 1:), vn
+    if (tid == 0) BCW_TRACE(s, m, 14);
+    if (L2 > 0 && tau_next != 0.0 && isO) {
+      const double tv = tau_next * vn[r - L];
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
+      }
+    }
+    fence_proxy_async_smem();
+    if (a.V2) {
+      const int64_t off = bc_offset(n, b, s);
+      double* vd = a.V2 + (off + m) * a.vs;
+      for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
+      if (tid == 0) a.tau2[off + m] = tau;
+    }
+    cbar();   // (5) columns 1..L-1 final
+    if (tid == 0) {
+      BCW_TRACE(s, m, 2);
+      mbar_arrive(&colsb[bi]);   // -> STORE
+    }
+    tau = tau_next;
+  }
+}
+
 // ---- row-per-thread chase (experimental, TRID_BC_FORCE=4; measured slower: see DESIGN.md sec. 5) ---------------------------------------------------------
 // One compute thread per window row (2B threads: row r of [D; O], all L <= B columns in registers), plus the
 // LOAD and STORE warps of bc_ws_kernel.  A row's matvec needs no cross-thread reduction, so the path from
@@ -1205,12 +1571,23 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
     a.trace_sweep = tr ? atoll(tr) : -1;
     int occ = 1;
     if (beff <= 64) {
-      // default: warp-specialized chase (bc_ws_kernel, 1 CTA/SM).  TRID_BC_FORCE (debug/tests): "1" the
-      // single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel.
+      // default: bc_v6_kernel (warp-specialized, short column-0 path, 1 CTA/SM).  TRID_BC_FORCE (debug/tests):
+      // "1" the single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel, "3" bc_ws_kernel,
+      // "4" bc_row_kernel.
       const int B = beff <= 32 ? 32 : 64;
       const char* force = getenv("TRID_BC_FORCE");
-      const int variant = force ? force[0] - '0' : 3;
-      if (variant == 4) {
+      const int variant = force ? force[0] - '0' : 6;
+      if (variant == 6) {
+        const int nth = B == 32 ? 256 : 512;
+        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 4 * (size_t)ldab + 2 * B + 2 * B + B + 16 +
+                                              (size_t)(nth / (2 * B)) * 2 * B + 8);
+        const void* fn = B == 32 ? (const void*)bc_v6_kernel<32, 256> : (const void*)bc_v6_kernel<64, 512>;
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int64_t grid = kNumSMsB200;
+        if (grid > n - 2) grid = n - 2;
+        if (B == 32) bc_v6_kernel<32, 256><<<(unsigned)grid, 256 + 96, smem, st>>>(a);
+        else bc_v6_kernel<64, 512><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
+      } else if (variant == 4) {
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B +
                                               (size_t)(2 * B / 32) * B + 2 * (2 * B / 32) + 8);
         const void* fn = B == 32 ? (const void*)bc_row_kernel<32> : (const void*)bc_row_kernel<64>;

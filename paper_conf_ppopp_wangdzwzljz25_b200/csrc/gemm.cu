@@ -43,7 +43,7 @@ constexpr int stage_elems_max() {
 template <int BM, int BN, int NT, int OPA, int OPB, int MASK>
 __device__ __forceinline__ void load_stage(double* As, double* Bs, const double* A, int64_t lda, const double* B,
                                            int64_t ldb, int64_t m0, int64_t n0, int64_t M, int64_t N, int64_t k0,
-                                           int64_t kend) {
+                                           int64_t kend, const double* A2 = nullptr, int64_t msplit = INT64_MAX) {
   const int tid = threadIdx.x;
 #pragma unroll
   for (int e = tid; e < BM * BK; e += NT) {
@@ -54,7 +54,12 @@ __device__ __forceinline__ void load_stage(double* As, double* Bs, const double*
     if (MASK == 1) p = p && (k <= row);
     if (MASK == 2) p = p && (k > row);
     const double* src = A;
-    if (p) src = OPA == OP_N ? A + row + k * lda : A + k + row * lda;
+    if (p) {
+      // rows >= msplit come from A2 (row - msplit): two stacked operands in one launch
+      const double* Ab = row < msplit ? A : A2;
+      const int64_t rr = row < msplit ? row : row - msplit;
+      src = OPA == OP_N ? Ab + rr + k * lda : Ab + k + rr * lda;
+    }
     cp_async8(As + ATile<BM, OPA>::idx(r, kk), src, p);
   }
 #pragma unroll
@@ -73,7 +78,8 @@ __device__ __forceinline__ void load_stage(double* As, double* Bs, const double*
 template <int BM, int BN, int WGM, int WGN, int OPA, int OPB, int MASK>
 __device__ __forceinline__ void mainloop(double (&acc)[BM / WGM / 16][BN / WGN / 8][4], double* smem, const double* A,
                                          int64_t lda, const double* B, int64_t ldb, int64_t m0, int64_t n0,
-                                         int64_t M, int64_t N, int64_t kbeg, int64_t kend) {
+                                         int64_t M, int64_t N, int64_t kbeg, int64_t kend,
+                                         const double* A2 = nullptr, int64_t msplit = INT64_MAX) {
   constexpr int NT = WGM * WGN * 32;
   constexpr int WTM = BM / WGM, WTN = BN / WGN;
   constexpr int MT = WTM / 16, NTL = WTN / 8;
@@ -90,7 +96,7 @@ __device__ __forceinline__ void mainloop(double (&acc)[BM / WGM / 16][BN / WGN /
   for (int s = 0; s < STAGES - 1; ++s) {
     if (s < ntile)
       load_stage<BM, BN, NT, OPA, OPB, MASK>(As + s * AE, Bs + s * BE, A, lda, B, ldb, m0, n0, M, N, kbeg + s * BK,
-                                             kend);
+                                             kend, A2, msplit);
     cp_async_commit();
   }
   for (int it = 0; it < ntile; ++it) {
@@ -100,7 +106,7 @@ __device__ __forceinline__ void mainloop(double (&acc)[BM / WGM / 16][BN / WGN /
     if (nxt < ntile) {
       const int st = nxt % STAGES;
       load_stage<BM, BN, NT, OPA, OPB, MASK>(As + st * AE, Bs + st * BE, A, lda, B, ldb, m0, n0, M, N,
-                                             kbeg + (int64_t)nxt * BK, kend);
+                                             kbeg + (int64_t)nxt * BK, kend, A2, msplit);
     }
     cp_async_commit();
     const double* Ast = As + (it % STAGES) * AE;
@@ -166,7 +172,8 @@ __global__ void __launch_bounds__(WGM* WGN * 32, (BM * BN <= 4096 ? 3 : 2)) gemm
   if (tb < kt0) {
     const int64_t e = te < kt0 ? te : kt0;
     const int64_t kb = tb * BK, ke = (e * BK < a.K[0]) ? e * BK : a.K[0];
-    mainloop<BM, BN, WGM, WGN, OPA, OPB, 0>(acc, smem, a.A[0], a.lda[0], a.B[0], a.ldb[0], m0, n0, a.M, a.N, kb, ke);
+    mainloop<BM, BN, WGM, WGN, OPA, OPB, 0>(acc, smem, a.A[0], a.lda[0], a.B[0], a.ldb[0], m0, n0, a.M, a.N, kb, ke,
+                                            a.A2m, a.msplit);
   }
   if (te > kt0) {
     const int64_t b0 = (tb > kt0 ? tb : kt0) - kt0, e = te - kt0;

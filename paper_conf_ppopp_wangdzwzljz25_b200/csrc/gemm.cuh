@@ -20,6 +20,10 @@ enum { TILE_128x128 = 0, TILE_128x64 = 1, TILE_64x64 = 2 };
 struct GemmArgs {
   int64_t M = 0, N = 0;
   int nseg = 1;
+  // gemm() only, segment 0: rows >= msplit of op(A) are rows (row - msplit) of A2m (same ld) -- two
+  // stacked operands [op(A); op(A2m)] in one launch
+  const double* A2m = nullptr;
+  int64_t msplit = INT64_MAX;
   const double* A[2] = {nullptr, nullptr};
   int64_t lda[2] = {1, 1};
   const double* B[2] = {nullptr, nullptr};

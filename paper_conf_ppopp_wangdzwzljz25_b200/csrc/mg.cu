@@ -281,7 +281,7 @@ struct Carver {
 };
 
 struct MgWork {
-  double *Y, *Z, *W, *X, *Xl, *Wl, *Yl, *Zl, *T, *U1, *U2, *S, *pk, *part, *red;
+  double *Y, *Z, *W, *X, *Xl, *Wl, *Yl, *Zl, *T, *U, *S, *pk, *part, *red;
   unsigned *bar, *sem;
   int64_t part_elems;
   size_t bytes;
@@ -315,8 +315,7 @@ MgWork carve_mg(void* base, int64_t n, int b, int k, int g, int q) {
   w.Yl = c.take<double>(nqp * k);
   w.Zl = c.take<double>(nqp * k);
   w.T = c.take<double>((size_t)b * b);
-  w.U1 = c.take<double>((size_t)k * b);
-  w.U2 = c.take<double>((size_t)k * b);
+  w.U = c.take<double>((size_t)2 * k * b);   // [Z_<^T W; Y_<^T W], ld 2k
   w.S = c.take<double>((size_t)b * b);
   w.pk = c.take<double>((size_t)n * b + (size_t)b * b + b);
   w.part_elems = pe;
@@ -504,7 +503,7 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
         }
         if ((r = comm_sum(comm, w.X, ldx * kk, true, 0, st))) return r;   // padding rows ride along unread
       }
-      TRID_CUDA_TRY(zy_tail(m, kk, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ldx, w.U1, w.U2, k, w.S, b,
+      TRID_CUDA_TRY(zy_tail(m, kk, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ldx, w.U, 2 * k, w.S, b,
                             w.part, w.part_elems, w.sem, st));
       ncols += kk;                                                  // l.6
       jlast = j;

@@ -132,7 +132,7 @@ def test_bulge_chase_parity(n, b, dev):
     assert np.max(np.abs(V2.cpu().numpy() - V_o), initial=0) <= 1e-9
 
 
-@pytest.mark.parametrize("variant", ["1", "2", "3", "4"])
+@pytest.mark.parametrize("variant", ["1", "2", "3", "4", "6"])
 def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
     """Every B=64 chase kernel (1: bc_fast 2 CTAs/SM single buffer, 2: bc_fast double buffer, 3: warp-specialized
     bc_ws (default), 4: row-per-thread bc_row) against the oracle, bitwise reproducible."""
