@@ -20,6 +20,7 @@
 #include "driver.cuh"
 
 #include <stdlib.h>
+#include <type_traits>
 
 namespace trid {
 
@@ -909,6 +910,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   extern __shared__ __align__(16) double sm[];
   const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int lda1 = ldab - 1;
+  const int ldab_rt = ldab, lda1_rt = lda1;
   const int64_t n = a.n;
   const int wsz = B * ldab;
   double* colb = sm + 2 * wsz;               // 2 x ldab: column s of a sweep's step 0, per buffer
@@ -918,6 +920,8 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   double* zv = pyv + 2 * B;                  // B
   double* red = zv + B;                      // 2*RW warp partials, x0, beta/tau/scale (16)
   double* part = red + 16;                   // TPR x 2B
+  double* xs = part + TPR * 2 * B;           // 2B: x = right-updated O(:, 0) by window row
+  double* zp = xs + 2 * B;                   // RW x B: per-row-warp partials of z = vn^T O
   __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], col0b[2], colsb[2], c0done[2];
   __shared__ int64_t info_s[2];
   __shared__ int info_m[2];
@@ -1032,6 +1036,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NTH) : "memory"); };
   auto c0bar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(2 * B) : "memory"); };
   double tau = 0.0;
+  int64_t off = 0;   // V2/tau2 offset of the current sweep (once per sweep: bc_offset divides)
   for (uint32_t it = 0;; ++it) {
     const int bi = it & 1;
     const unsigned ph = (it >> 1) & 1u;
@@ -1046,23 +1051,34 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
     if (tid == 0) BCW_TRACE(s, m, 0);
     const int64_t r0 = s + 1 + m * b;
     const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-    const int L = (int)(r1 - r0 + 1);
+    const int Lx = (int)(r1 - r0 + 1);
     const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
-    const int L2 = (int)(r2 - r1);
+    const int L2x = (int)(r2 - r1);
     double* win = sm + bi * wsz;
     double* v = vb + (m & 1) * B;
     double* vn = vb + ((m & 1) ^ 1) * B;
     if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
+      if (a.V2) off = bc_offset(n, b, s);
       const double* col = colb + bi * ldab + 1;
       double sig = 0.0;
-      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
+      for (int i = 1 + lane; i < Lx; i += 32) sig = fma(col[i], col[i], sig);
       sig = warp_sum(sig);
       const House hh = make_house(col[0], sig);
-      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
+      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < Lx ? hh.scale * col[tid] : 0.0);
       if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
       tau = hh.tau;
       cbar();
     }
+    // Full windows (L = L2 = B: every step but the last of a sweep) are compiled separately, so the
+    // row/column predicates and the O/D split (warp-uniform for B % 32 == 0) fold at compile time.
+    double tau_next = 0.0;
+    auto step = [&](auto fullc) {
+      constexpr bool FULL = decltype(fullc)::value;
+      const int L = FULL ? B : Lx;
+      const int L2 = FULL ? B : L2x;
+      // a full window implies b == B, so the column stride ldab = 2B is a compile-time constant there
+      const int lda1 = FULL ? 2 * B - 1 : lda1_rt;
+      const int ldab = FULL ? 2 * B : ldab_rt;
     const bool active = r < L + L2;
     const bool isO = r >= L && active;
     const int lo_base = j0 * lda1 + r;
@@ -1111,6 +1127,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
         red[RW + warp] = tO;
       }
       if (r == L) red[2 * RW] = x;
+      xs[r] = x;
       c0bar();
       double pv = 0.0, sg = 0.0;
 #pragma unroll
@@ -1146,9 +1163,9 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       for (int jj = 0; jj < CPT; ++jj)
         if (jj == jd) e[jj] = el;
     }
-    cbar();   // (2) pyv, p^T v partials, the next reflector's scalars
+    cbar();   // (2) pyv, p^T v partials, x, the next reflector's scalars
     if (tid == 0) BCW_TRACE(s, m, 12);
-    double tau_next = 0.0, hscale = 0.0;
+    double hscale = 0.0;
     if (L2 > 0) {
       tau_next = red[2 * RW + 2];
       hscale = red[2 * RW + 3];
@@ -1160,45 +1177,46 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       const double hp = 0.5 * tau * pv;
       if (isO) {
         const double ty = tau * pyv[r];
+        const double2* v2u = reinterpret_cast<const double2*>(v + j0);
 #pragma unroll
-        for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
+        for (int jj = 0; jj < CPT; jj += 2) {
+          const double2 vj = v2u[jj / 2];
+          e[jj] = fma(-ty, vj.x, e[jj]);
+          e[jj + 1] = fma(-ty, vj.y, e[jj + 1]);
+        }
       } else {
         const double vr = r < L ? v[r] : 0.0;
         const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
+        const double2* v2u = reinterpret_cast<const double2*>(v + j0);
+        const double2* p2u = reinterpret_cast<const double2*>(pyv + j0);
 #pragma unroll
-        for (int jj = 0; jj < CPT; ++jj) {
-          const double vj = v[j0 + jj];
-          const double wj = fma(-hp, vj, pyv[j0 + jj]);
-          e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
+        for (int jj = 0; jj < CPT; jj += 2) {
+          const double2 vj = v2u[jj / 2], pj = p2u[jj / 2];
+          const double wj0 = fma(-hp, vj.x, pj.x), wj1 = fma(-hp, vj.y, pj.y);
+          e[jj] = fma(-wr, vj.x, fma(-vr, wj0, e[jj]));
+          e[jj + 1] = fma(-wr, vj.y, fma(-vr, wj1, e[jj + 1]));
         }
       }
     }
+    // D rows are final: write the lower triangle back (column 0 goes out through the staging buffer)
+    if (active && !isO) {
 #pragma unroll
-    for (int jj = 0; jj < CPT; ++jj) {
-      const int j = j0 + jj;
-      if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
-    }
-    cbar();   // (3) right-updated window in shared memory
-    if (tid == 0) BCW_TRACE(s, m, 13);
-    if (L2 > 0 && tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : hscale * win[L + tid]) : 0.0;
-    if (L2 > 0 && tau_next != 0.0 && L > 1) {
-      const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
-      const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
-      double c[CPW];
-#pragma unroll
-      for (int q = 0; q < CPW; ++q) {
-        const int j = warp + q * NW;
-        double acc = 0.0;
-        if (j >= 1 && j < L) {
-          const int ob = j * lda1 + L;
-          if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
-          if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
-        }
-        c[q] = acc;
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        if (j >= 1 && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
       }
-      int qbase = 0;
+    }
+    // next reflector vn (rows L..L+L2-1 of the window): vn_0 = 1, vn_i = scale * x_i
+    const double vnr = isO ? (r == L ? 1.0 : hscale * xs[r]) : 0.0;
+    if (L2 > 0 && tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : hscale * xs[L + tid]) : 0.0;
+    const bool zwarp = L2 > 0 && tau_next != 0.0 && L > 1 && (warp % RW) * 32 + 31 >= L;   // warp holds O rows
+    if (zwarp) {
+      // z_j = sum_i vn_i O(i, j) over this warp's 32 rows for the group's CPT columns: transposed butterfly
+      double c[CPT];
 #pragma unroll
-      for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
+      for (int jj = 0; jj < CPT; ++jj) c[jj] = vnr * e[jj];
+#pragma unroll
+      for (int o = 16, K = CPT; K > 1; o >>= 1, K >>= 1) {
         const bool up = (lane & o) != 0;
 #pragma unroll
         for (int i = 0; i < K / 2; ++i) {
@@ -1206,39 +1224,58 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
           const double keep = up ? c[i + K / 2] : c[i];
           c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
         }
-        if (up) qbase += K / 2;
       }
-      constexpr int LV = CPW == 4 ? 2 : 3;
+      constexpr int SH = CPT == 16 ? 1 : (CPT == 8 ? 2 : 3);   // lanes per column after the butterfly
       double f = c[0];
 #pragma unroll
-      for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
-      if ((lane & ((32 >> LV) - 1)) == 0) {
-        const int j = warp + qbase * NW;
-        if (j >= 1 && j < L) zv[j] = fma(hscale, f, win[j * lda1 + L]);
-      }
+      for (int o = (1 << SH) >> 1; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+      if ((lane & ((1 << SH) - 1)) == 0) zp[(warp % RW) * B + j0 + (lane >> SH)] = f;
+    } else if (lane < CPT) {
+      zp[(warp % RW) * B + j0 + lane] = 0.0;
     }
-    cbar();   // (4) z = vn^T O(:, 1:), vn
-    if (tid == 0) BCW_TRACE(s, m, 14);
-    if (L2 > 0 && tau_next != 0.0 && isO) {
-      const double tv = tau_next * vn[r - L];
+    cbar();   // (3) z partials, vn
+    if (tid == 0) BCW_TRACE(s, m, 13);
+    if (FULL && isO) {
+      // full window: the O rows are the last two row-warps of the group (the others' partials are zero, and
+      // 0 + x == x, so this is the generic sum below bit for bit)
+      const double tv = tau_next * vnr;
+      const double2* za = reinterpret_cast<const double2*>(zp + (RW - 2) * B + j0);
+      const double2* zb = reinterpret_cast<const double2*>(zp + (RW - 1) * B + j0);
+#pragma unroll
+      for (int jj = 0; jj < CPT; jj += 2) {
+        const double2 x = za[jj / 2], y = zb[jj / 2];
+        const double z0 = x.x + y.x, z1 = x.y + y.y;
+        if (j0 + jj >= 1) win[lo_base + jj * lda1] = tau_next != 0.0 ? fma(-tv, z0, e[jj]) : e[jj];
+        win[lo_base + (jj + 1) * lda1] = tau_next != 0.0 ? fma(-tv, z1, e[jj + 1]) : e[jj + 1];
+      }
+    } else if (isO) {
+      const double tv = tau_next * vnr;
 #pragma unroll
       for (int jj = 0; jj < CPT; ++jj) {
         const int j = j0 + jj;
-        if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
+        if (j >= 1 && j < L) {
+          double z = 0.0;
+#pragma unroll
+          for (int w = 0; w < RW; ++w) z += zp[w * B + j];
+          win[lo_base + jj * lda1] = (L2 > 0 && tau_next != 0.0) ? fma(-tv, z, e[jj]) : e[jj];
+        }
       }
     }
     fence_proxy_async_smem();
+    if (tid == 0) BCW_TRACE(s, m, 14);
     if (a.V2) {
-      const int64_t off = bc_offset(n, b, s);
       double* vd = a.V2 + (off + m) * a.vs;
       for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
       if (tid == 0) a.tau2[off + m] = tau;
     }
-    cbar();   // (5) columns 1..L-1 final
+    cbar();   // (4) columns 1..L-1 final
     if (tid == 0) {
       BCW_TRACE(s, m, 2);
-      mbar_arrive(&colsb[bi]);   // -> STORE
+      mbar_arrive(&colsb[bi]);   // -> STORE1
     }
+    };
+    if (Lx == B && L2x == B) step(std::true_type{});
+    else step(std::false_type{});
     tau = tau_next;
   }
 }
@@ -1580,7 +1617,7 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       if (variant == 6) {
         const int nth = B == 32 ? 256 : 512;
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 4 * (size_t)ldab + 2 * B + 2 * B + B + 16 +
-                                              (size_t)(nth / (2 * B)) * 2 * B + 8);
+                                              (size_t)(nth / (2 * B)) * 2 * B + 2 * B + (2 * B / 32) * B + 8);
         const void* fn = B == 32 ? (const void*)bc_v6_kernel<32, 256> : (const void*)bc_v6_kernel<64, 512>;
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int64_t grid = kNumSMsB200;

@@ -62,8 +62,8 @@ if os.environ.get("TRID_BC_FORCE", "6") == "6":   # bc_v6_kernel slot meanings
         "v6: last-col wait (10 -> 11)": np.mean(c[m, 11] - c[m, 10]) / 1e3,
         "v6: col0 path (11 -> 1)": np.mean(c[m, 1] - c[m, 11]) / 1e3,
         "v6: cbar2 (1 -> 12)": np.mean(c[m, 12] - c[m, 1]) / 1e3,
-        "v6: update+writeback+cbar3 (12 -> 13)": np.mean(c[m, 13] - c[m, 12]) / 1e3,
-        "v6: z pass+cbar4 (13 -> 14)": np.mean(c[m, 14] - c[m, 13]) / 1e3,
-        "v6: left apply+V2+cbar5 (14 -> 2)": np.mean(c[m, 2] - c[m, 14]) / 1e3,
+        "v6: update+D writeback+z partials+cbar3 (12 -> 13)": np.mean(c[m, 13] - c[m, 12]) / 1e3,
+        "v6: z sum+left apply+O writeback (13 -> 14)": np.mean(c[m, 14] - c[m, 13]) / 1e3,
+        "v6: V2+cbar4 (14 -> 2)": np.mean(c[m, 2] - c[m, 14]) / 1e3,
     })
 print(json.dumps({k: round(float(v), 3) for k, v in out.items()}, indent=1))
