@@ -19,7 +19,7 @@ import os
 import torch
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libtrid.so")
+LIB_PATH = os.environ.get("TRID_LIB_PATH") or os.path.join(HERE, "libtrid.so")   # override: A/B timing tools
 
 _lib = None
 _I64 = ctypes.c_int64

@@ -899,8 +899,57 @@ __device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
   (void)ld_acquire_s32(p);
 }
 
-template <int B, int NTH>
-__global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
+__device__ __forceinline__ bool bc_step_full(int64_t n, int b, int B, int64_t s, int64_t m) {
+  if (b != B || s < 0 || s > n - 3 || m < 0) return false;
+  const int64_t r0 = s + 1 + m * b;
+  return r0 + 2 * (int64_t)B - 1 <= n - 1;   // L == B and L2 == B
+}
+__device__ __forceinline__ unsigned cl_rank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;\n" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned cl_size() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_nctarank;\n" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned cl_mapa(const void* p, unsigned rank) {
+  unsigned r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;\n" : "=r"(r) : "r"(smem_u32(p)), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void cl_st_release(unsigned raddr, int v) {
+  asm volatile("st.release.cluster.shared::cluster.s32 [%0], %1;\n" ::"r"(raddr), "r"(v) : "memory");
+}
+__device__ __forceinline__ void cl_wait_geq(const int* p, int need) {
+  int v;
+  do {
+    asm volatile("ld.acquire.cluster.shared::cta.s32 %0, [%1];\n" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  } while (v < need);
+}
+// shared (this CTA) -> shared (peer CTA) bulk copy completing on the peer's mbarrier
+__device__ __forceinline__ void bulk_s2s_cl(unsigned rdst, const void* src, unsigned bytes, unsigned rbar) {
+  asm volatile("cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                   rdst),
+               "r"(smem_u32(src)), "r"(bytes), "r"(rbar)
+               : "memory");
+}
+__device__ __forceinline__ void cl_sync_all() {
+  asm volatile("barrier.cluster.arrive.release;\nbarrier.cluster.wait.acquire;\n" ::: "memory");
+}
+
+// CL (clusters of C CTAs, DSMEM forwarding): CTA rank q of cluster c runs sweeps (c + i*NC)*C + q, i = 0, 1, ...
+// (static order; the persistent grid is sized to co-resident clusters).  Inside a cluster, sweep s+1 (rank q+1)
+// receives sweep s's data for every full-window step straight from rank q's shared memory: the step's columns
+// 1..L-1 (its window body) and column 0 of the next step (its last column) are bulk-copied CTA-to-CTA onto the
+// consumer's own mbarriers, after the consumer announced (armed, a monotone step count in the producer's shared
+// memory) that the target buffer is free and expecting them; the consumer acknowledges arrival (recv) so the
+// producer can recycle its buffer.  The global band and the prog/prog_full counters are still written for every
+// step (final result, cross-cluster consumers, ragged steps), but the in-cluster link no longer pays the release /
+// poll / L2 round trips.
+template <int B, int NTH, bool CL>
+__device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
   constexpr int TPR = NTH / (2 * B);
   constexpr int CPT = B / TPR;
   constexpr int RW = (2 * B) / 32;   // warps of the column-0 path (column group 0)
@@ -925,7 +974,11 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], col0b[2], colsb[2], c0done[2];
   __shared__ int64_t info_s[2];
   __shared__ int info_m[2];
+  __shared__ int info_f[2];            // CL: the step's body/last column arrive from the producer CTA
+  __shared__ int armed_ctr, recv_ctr;  // CL: written by the consumer CTA (monotone step counts)
   if (tid == 0) {
+    armed_ctr = 0;
+    recv_ctr = 0;
     for (int i = 0; i < 2; ++i) {
       mbar_init(&full[i], 1);
       mbar_init(&lastb[i], 1);
@@ -936,13 +989,24 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
-  __syncthreads();
+  unsigned crank = 0, csize = 1;
+  if constexpr (CL) {
+    crank = cl_rank();
+    csize = cl_size();
+    cl_sync_all();   // peers' barriers and counters are initialised before any remote access
+  } else {
+    __syncthreads();
+  }
+  const bool has_prod = CL && crank > 0;            // sweep s-1 runs on rank crank-1 of this cluster
+  const bool has_cons = CL && crank + 1 < csize;    // sweep s+1 runs on rank crank+1
   if (warp == NW) {
     // ============================== LOAD warp ==============================
     if (lane != 0) return;
     uint32_t it = 0;
-    for (;;) {
-      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
+    for (int64_t sweep_i = 0;; ++sweep_i) {
+      int64_t s;
+      if constexpr (CL) s = ((int64_t)(blockIdx.x / csize) + sweep_i * (int64_t)(gridDim.x / csize)) * csize + crank;
+      else s = (int64_t)atomicAdd(a.ticket, 1u);
       const bool done = s > n - 3;
       const int64_t nst = done ? 1 : bc_steps(n, b, s);
       const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
@@ -961,8 +1025,16 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
         const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
         const int L = (int)(r1 - r0 + 1);
         double* win = sm + bi * wsz;
+        const bool fwd = has_prod && bc_step_full(n, b, B, s, m);
+        info_f[bi] = fwd;
         mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
         mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
+        if (fwd) {   // the producer CTA copies body (+ column s at m = 0) and the last column into this buffer
+          cl_st_release(cl_mapa(&armed_ctr, crank - 1), (int)(it + 1));
+          BCW_TRACE(s, m, 8);
+          BCW_TRACE(s, m, 9);
+          continue;
+        }
         if (s > 0) {
           if (m == 0) wait_geq_spin(a.prog + (s - 1), 1);
           wait_geq_spin(a.prog_full + (s - 1), (int)(m + 1));
@@ -981,6 +1053,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   if (warp == NW + 1) {
     // ============================== STORE0 warp: column 0 (the chain) ==============================
     if (lane != 0) return;
+    uint32_t cbase = 0, cnext = 0;   // CL: the consumer CTA's step count at the start of its current sweep
     for (uint32_t it = 0;; ++it) {
       const int bi = it & 1;
       const unsigned ph = (it >> 1) & 1u;
@@ -990,6 +1063,26 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       const int m = info_m[bi];
       const int64_t r0 = s + 1 + (int64_t)m * b;
       BCW_TRACE(s, m, 3);
+      if (has_cons) {
+        if (m == 0) {
+          cbase = cnext;
+          cnext += (uint32_t)bc_steps(n, b, s + 1);
+        }
+        // column 0 of step m is column s+1 of the consumer's step 0 (m = 0) or the last column of its step m-1
+        const int mt = m == 0 ? 0 : m - 1;
+        if (bc_step_full(n, b, B, s + 1, mt)) {
+          const uint32_t itc = cbase + (uint32_t)mt;
+          const int bc = itc & 1;
+          cl_wait_geq(&armed_ctr, (int)(itc + 1));
+          const unsigned dst = m == 0 ? cl_mapa(colb + bc * ldab, crank + 1)
+                                      : cl_mapa(sm + bc * wsz + (B - 1) * ldab, crank + 1);
+          const unsigned bar = m == 0 ? cl_mapa(&full[bc], crank + 1) : cl_mapa(&lastb[bc], crank + 1);
+          bulk_s2s_cl(dst, c0s + bi * ldab, (unsigned)(ldab * 8), bar);
+        }
+      }
+      // CL: this step may have been fed by DSMEM before the producer's own global stores of the same columns
+      // landed; never let an older global store overwrite ours (write-after-write on the band)
+      if (has_prod) wait_geq_spin(a.prog_full + (s - 1), m + 1);
       bulk_s2g(a.band + r0 * ldab, c0s + bi * ldab, (unsigned)(ldab * 8));
       bulk_commit();
       bulk_wait_all();
@@ -1004,6 +1097,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
     // ============================== STORE1 warp: columns 1..L-1 ==============================
     // frees the window buffer as soon as the bulk store has READ it; prog_full after the writes landed
     if (lane != 0) return;
+    uint32_t cbase = 0, cnext = 0;
     for (uint32_t it = 0;; ++it) {
       const int bi = it & 1;
       const unsigned ph = (it >> 1) & 1u;
@@ -1015,11 +1109,35 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
       const int L = (int)(r1 - r0 + 1);
       double* win = sm + bi * wsz;
+      int recv_need = 0;
+      if (has_cons) {
+        if (m == 0) {
+          cbase = cnext;
+          cnext += (uint32_t)bc_steps(n, b, s + 1);
+        }
+        // columns 1..L-1 of step m are the body of the consumer's step m
+        if (bc_step_full(n, b, B, s + 1, m)) {
+          const uint32_t itc = cbase + (uint32_t)m;
+          const int bc = itc & 1;
+          cl_wait_geq(&armed_ctr, (int)(itc + 1));
+          bulk_s2s_cl(cl_mapa(sm + bc * wsz, crank + 1), win + ldab, (unsigned)((B - 1) * ldab * 8),
+                      cl_mapa(&full[bc], crank + 1));
+          recv_need = (int)(itc + 1);
+        }
+        const int mt = m == 0 ? 0 : m - 1;   // where STORE0 sent this step's column 0
+        if (bc_step_full(n, b, B, s + 1, mt) && (int)(cbase + mt + 1) > recv_need) recv_need = (int)(cbase + mt + 1);
+      }
+      if (has_prod) {   // as in STORE0: the producer's global stores of these columns landed first
+        const int np = (int)bc_steps(n, b, s - 1);
+        wait_geq_spin(a.prog_full + (s - 1), m + 1);
+        wait_geq_spin(a.prog + (s - 1), m + 2 < np ? m + 2 : np);
+      }
       if (L > 1) {
         bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
         bulk_commit();
         bulk_wait_read();
       }
+      if (recv_need) cl_wait_geq(&recv_ctr, recv_need);   // the consumer holds both copies (they read this buffer)
       mbar_wait(&c0done[bi], ph);   // column 0's staging buffer was read too
       mbar_arrive(&empty[bi]);
       if (L > 1) {
@@ -1079,6 +1197,9 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       // a full window implies b == B, so the column stride ldab = 2B is a compile-time constant there
       const int lda1 = FULL ? 2 * B - 1 : lda1_rt;
       const int ldab = FULL ? 2 * B : ldab_rt;
+      // the window through the extern __shared__ base (keeps the shared address space visible to the compiler
+      // inside the lambda; in full windows the buffer stride is a constant too)
+      double* const win = sm + bi * (FULL ? B * 2 * B : wsz);
     const bool active = r < L + L2;
     const bool isO = r >= L && active;
     const int lo_base = j0 * lda1 + r;
@@ -1111,6 +1232,7 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
       for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + r];
       mbar_wait(&lastb[bi], ph);
       if (tid == 0) BCW_TRACE(s, m, 11);
+      if (CL && tid == 0 && info_f[bi]) cl_st_release(cl_mapa(&recv_ctr, crank - 1), (int)(it + 1));
       if (active && r >= L - 1) acc = fma(win[(L - 1) * lda1 + r], v[L - 1], acc);
       const double py = (r >= L) ? acc : tau * acc;   // p_r = tau (D v)_r  |  y_r = (O v)_r
       pyv[r] = py;
@@ -1203,7 +1325,8 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
 #pragma unroll
       for (int jj = 0; jj < CPT; ++jj) {
         const int j = j0 + jj;
-        if (j >= 1 && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
+        // (column 0 is published from the staging buffer and never read back: a full window may write it)
+        if ((FULL || (j >= 1 && j < L)) && j <= r) win[lo_base + jj * lda1] = e[jj];
       }
     }
     // next reflector vn (rows L..L+L2-1 of the window): vn_0 = 1, vn_i = scale * x_i
@@ -1278,6 +1401,12 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
     else step(std::false_type{});
     tau = tau_next;
   }
+}
+
+template <int B, int NTH, bool CL>
+__global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
+  bc_v6_body<B, NTH, CL>(a);
+  if constexpr (CL) cl_sync_all();   // no CTA leaves while a peer may still copy into / signal its shared memory
 }
 
 // ---- row-per-thread chase (experimental, TRID_BC_FORCE=4; measured slower: see DESIGN.md sec. 5) ---------------------------------------------------------
@@ -1614,16 +1743,52 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       const int B = beff <= 32 ? 32 : 64;
       const char* force = getenv("TRID_BC_FORCE");
       const int variant = force ? force[0] - '0' : 6;
-      if (variant == 6) {
+      if (variant == 6 || variant == 7) {
         const int nth = B == 32 ? 256 : 512;
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 4 * (size_t)ldab + 2 * B + 2 * B + B + 16 +
                                               (size_t)(nth / (2 * B)) * 2 * B + 2 * B + (2 * B / 32) * B + 8);
-        const void* fn = B == 32 ? (const void*)bc_v6_kernel<32, 256> : (const void*)bc_v6_kernel<64, 512>;
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        int64_t grid = kNumSMsB200;
-        if (grid > n - 2) grid = n - 2;
-        if (B == 32) bc_v6_kernel<32, 256><<<(unsigned)grid, 256 + 96, smem, st>>>(a);
-        else bc_v6_kernel<64, 512><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
+        const void* fn6 = B == 32 ? (const void*)bc_v6_kernel<32, 256, false> : (const void*)bc_v6_kernel<64, 512, false>;
+        const void* fn7 = B == 32 ? (const void*)bc_v6_kernel<32, 256, true> : (const void*)bc_v6_kernel<64, 512, true>;
+        bool launched = false;
+        if (variant == 7) {
+          // clusters of C (env TRID_BC_CLUSTER, default 2) sized to the co-resident cluster count
+          const char* ce = getenv("TRID_BC_CLUSTER");
+          const int C = ce ? atoi(ce) : 2;
+          cudaFuncSetAttribute(fn7, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+          if (C > 8) cudaFuncSetAttribute(fn7, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+          cudaLaunchConfig_t cfg = {};
+          cfg.blockDim = dim3((unsigned)(nth + 96));
+          cfg.dynamicSmemBytes = smem;
+          cfg.stream = st;
+          cudaLaunchAttribute at[1];
+          at[0].id = cudaLaunchAttributeClusterDimension;
+          at[0].val.clusterDim.x = (unsigned)C;
+          at[0].val.clusterDim.y = 1;
+          at[0].val.clusterDim.z = 1;
+          cfg.attrs = at;
+          cfg.numAttrs = 1;
+          cfg.gridDim = dim3((unsigned)(C * 40));
+          int nc = 0;
+          if (C >= 2 && cudaOccupancyMaxActiveClusters(&nc, fn7, &cfg) == cudaSuccess && nc >= 1) {
+            int64_t ncl = nc;
+            const int64_t need = (n - 2 + C - 1) / C;   // clusters with at least one sweep
+            if (ncl > need) ncl = need;
+            cfg.gridDim = dim3((unsigned)(ncl * C));
+            cudaError_t le = B == 32 ? cudaLaunchKernelEx(&cfg, bc_v6_kernel<32, 256, true>, a)
+                                     : cudaLaunchKernelEx(&cfg, bc_v6_kernel<64, 512, true>, a);
+            if (le != cudaSuccess) return le;
+            launched = true;
+          } else {
+            (void)cudaGetLastError();
+          }
+        }
+        if (!launched) {
+          cudaFuncSetAttribute(fn6, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+          int64_t grid = kNumSMsB200;
+          if (grid > n - 2) grid = n - 2;
+          if (B == 32) bc_v6_kernel<32, 256, false><<<(unsigned)grid, 256 + 96, smem, st>>>(a);
+          else bc_v6_kernel<64, 512, false><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
+        }
       } else if (variant == 4) {
         const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B +
                                               (size_t)(2 * B / 32) * B + 2 * (2 * B / 32) + 8);

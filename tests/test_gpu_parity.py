@@ -132,10 +132,11 @@ def test_bulge_chase_parity(n, b, dev):
     assert np.max(np.abs(V2.cpu().numpy() - V_o), initial=0) <= 1e-9
 
 
-@pytest.mark.parametrize("variant", ["1", "2", "3", "4", "6"])
+@pytest.mark.parametrize("variant", ["1", "2", "3", "4", "6", "7"])
 def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
     """Every B=64 chase kernel (1: bc_fast 2 CTAs/SM single buffer, 2: bc_fast double buffer, 3: warp-specialized
-    bc_ws (default), 4: row-per-thread bc_row) against the oracle, bitwise reproducible."""
+    bc_ws, 4: row-per-thread bc_row, 6: bc_v6 (default), 7: bc_v6 in CTA clusters with DSMEM forwarding) against
+    the oracle, bitwise reproducible."""
     monkeypatch.setenv("TRID_BC_FORCE", variant)
     n, b = 700, 64
     Bm = band_from_lower(trid_gen.random_symmetric_np(n, 99), b)
@@ -147,6 +148,20 @@ def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
     assert np.max(np.abs(V2.cpu().numpy() - V_o)) <= 1e-9
     r1 = [x.clone() for x in trid.bulge_chase(to_dev(Bm), b)]
     for x, y in zip(r1, (d, e, V2, tau2)):
+        assert torch.equal(x, y)
+
+
+@pytest.mark.parametrize("n,b,cl", [(3000, 64, "2"), (3000, 64, "4"), (2500, 32, "2"), (1001, 48, "2"), (300, 64, "8"), (12000, 64, "2")])
+def test_bulge_chase_cluster_forwarding_bitwise(n, b, cl, dev, monkeypatch):
+    """The cluster variant (sweep s+1 fed from sweep s's shared memory) moves data differently but computes the
+    same expressions in the same order: its output equals the single-CTA chase's bit for bit (R9)."""
+    Bm = band_from_lower(trid_gen.random_symmetric_np(n, 5 + n), b)
+    monkeypatch.setenv("TRID_BC_FORCE", "6")
+    ref = [x.clone() for x in trid.bulge_chase(to_dev(Bm), b)]
+    monkeypatch.setenv("TRID_BC_FORCE", "7")
+    monkeypatch.setenv("TRID_BC_CLUSTER", cl)
+    got = trid.bulge_chase(to_dev(Bm), b)
+    for x, y in zip(ref, got):
         assert torch.equal(x, y)
 
 

@@ -8,5 +8,6 @@ timeout 300 python tools/bcw_trace.py 32768 64 2000 > $O/bcw6_trace_n32768_s2000
 timeout 900 python bench.py --no-cpu-baseline > $O/bench_n32768.json 2> $O/bench_n32768.err
 timeout 600 python bench.py --config n8192 --steps 3 --no-cpu-baseline --no-e2e > $O/bench_n8192.json 2> $O/bench_n8192.err
 if [ -n "$2" ]; then
-  timeout 600 ncu --set full --clock-control none --import-source on -k regex:bc_v6 -c 1 -o $O/prof_bcv6_8192 python tools/prof_run.py --n 8192 --b 64 --k 1024 --nb 16 > $O/prof.log 2>&1
+  TRID_BC_FORCE=7 timeout 600 python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > $O/bench7_n32768.json 2> $O/bench7_n32768.err
+  TRID_BC_FORCE=7 timeout 600 python bench.py --config n8192 --steps 3 --no-cpu-baseline --no-e2e > $O/bench7_n8192.json 2> $O/bench7_n8192.err
 fi
