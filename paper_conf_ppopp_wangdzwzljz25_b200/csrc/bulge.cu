@@ -899,6 +899,15 @@ __device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
   (void)ld_acquire_s32(p);
 }
 
+// 32-bit shared-window accesses for the full-window path (immediate offsets, no generic address arithmetic)
+__device__ __forceinline__ double lds_f64(uint32_t addr) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];\n" : "=d"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_f64(uint32_t addr, double v) {
+  asm volatile("st.shared.f64 [%0], %1;\n" ::"r"(addr), "d"(v) : "memory");
+}
 __device__ __forceinline__ bool bc_step_full(int64_t n, int b, int B, int64_t s, int64_t m) {
   if (b != B || s < 0 || s > n - 3 || m < 0) return false;
   const int64_t r0 = s + 1 + m * b;
@@ -1209,11 +1218,24 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
     const bool defer = r >= L - 1 && jd >= 0 && jd < CPT;
     double e[CPT];
     double acc0 = 0.0, acc1 = 0.0;
+    // shared byte addresses of (r, j0) in the lower (column j0) and the mirrored (column r) layout
+    const uint32_t a_lo = smem_u32(win) + 8u * (uint32_t)lo_base;
+    const uint32_t a_hi = smem_u32(win) + 8u * (uint32_t)hi_base;
+    const int rj = r - j0;   // element jj is in the stored lower triangle iff jj <= rj
+    if constexpr (FULL) {
 #pragma unroll
-    for (int jj = 0; jj < CPT; ++jj) {
-      const int j = j0 + jj;
-      const bool ok = j < L && !(defer && jj == jd);
-      e[jj] = ok ? win[j <= r ? lo_base + jj * lda1 : hi_base + jj] : 0.0;
+      for (int jj = 0; jj < CPT; ++jj) {
+        const bool skip = defer && jj == CPT - 1;   // full window: only the last column can be deferred
+        const uint32_t ad = jj <= rj ? a_lo + 8u * (uint32_t)(jj * lda1) : a_hi + 8u * (uint32_t)jj;
+        e[jj] = skip ? 0.0 : lds_f64(ad);
+      }
+    } else {
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj) {
+        const int j = j0 + jj;
+        const bool ok = j < L && !(defer && jj == jd);
+        e[jj] = ok ? win[j <= r ? lo_base + jj * lda1 : hi_base + jj] : 0.0;
+      }
     }
     const double2* v2 = reinterpret_cast<const double2*>(v + j0);
 #pragma unroll
@@ -1321,12 +1343,16 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       }
     }
     // D rows are final: write the lower triangle back (column 0 goes out through the staging buffer)
-    if (active && !isO) {
+    if (FULL && !isO) {
+      // (column 0 is published from the staging buffer and never read back: a full window may write it)
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj)
+        if (jj <= rj) sts_f64(a_lo + 8u * (uint32_t)(jj * lda1), e[jj]);
+    } else if (active && !isO) {
 #pragma unroll
       for (int jj = 0; jj < CPT; ++jj) {
         const int j = j0 + jj;
-        // (column 0 is published from the staging buffer and never read back: a full window may write it)
-        if ((FULL || (j >= 1 && j < L)) && j <= r) win[lo_base + jj * lda1] = e[jj];
+        if (j >= 1 && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
       }
     }
     // next reflector vn (rows L..L+L2-1 of the window): vn_0 = 1, vn_i = scale * x_i
@@ -1368,8 +1394,8 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       for (int jj = 0; jj < CPT; jj += 2) {
         const double2 x = za[jj / 2], y = zb[jj / 2];
         const double z0 = x.x + y.x, z1 = x.y + y.y;
-        if (j0 + jj >= 1) win[lo_base + jj * lda1] = tau_next != 0.0 ? fma(-tv, z0, e[jj]) : e[jj];
-        win[lo_base + (jj + 1) * lda1] = tau_next != 0.0 ? fma(-tv, z1, e[jj + 1]) : e[jj + 1];
+        if (j0 + jj >= 1) sts_f64(a_lo + 8u * (uint32_t)(jj * lda1), tau_next != 0.0 ? fma(-tv, z0, e[jj]) : e[jj]);
+        sts_f64(a_lo + 8u * (uint32_t)((jj + 1) * lda1), tau_next != 0.0 ? fma(-tv, z1, e[jj + 1]) : e[jj + 1]);
       }
     } else if (isO) {
       const double tv = tau_next * vnr;

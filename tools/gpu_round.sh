@@ -30,7 +30,7 @@ if has full; then
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:ws_kernel -s 1 -c 1 -o $O/prof_symm $P > $O/prof_symm.log 2>&1
   timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:ws_kernel<\(int\)128, \(int\)128' -c 1 -o $O/prof_syr2k $P > $O/prof_syr2k.log 2>&1
   TRID_PANEL_NOCOOP=1 timeout 900 ncu --set full --clock-control none --import-source on -k regex:panel_reg -s 5 -c 1 -o $O/prof_panel $P > $O/prof_panel.log 2>&1
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bc_fast -c 1 -o $O/prof_bc $P > $O/prof_bc.log 2>&1
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:bc_v6 -c 1 -o $O/prof_bc $P > $O/prof_bc.log 2>&1
 fi
 if has bctrace; then
   timeout 300 python tools/bcw_trace.py 8192 64 1000 > $O/bcw_trace_n8192.json 2>&1
