@@ -312,6 +312,12 @@ def main():
             traffic = json.load(open(tpath)).get(f"{args.config}:{dom}")
         except Exception:
             traffic = None
+    bc_traffic = None
+    if os.path.exists(tpath):
+        try:
+            bc_traffic = json.load(open(tpath)).get(f"{args.config}:bulge_chase")
+        except Exception:
+            bc_traffic = None
     hbm, hbm_kind = peaks()
     bcb = bc_bytes(n, b)
     bc_gbs = bcb / (t_bc * 1e-3) / 1e9 if t_bc > 0 else 0.0
@@ -336,7 +342,7 @@ def main():
                      "peak_source": "measured FP64 DMMA microbenchmark (profiles/r01_fp64_microbench.jsonl); "
                                     "MEASURED_PEAKS.json has no FP64 figure"},
         "roofline_bc": {"bound": "hbm", "kernel": "bulge_chase", "achieved": round(bc_gbs, 1), "peak": hbm,
-                        "unit": "GB/s", "frac": round(bc_gbs / hbm, 4), "traffic": None,
+                        "unit": "GB/s", "frac": round(bc_gbs / hbm, 4), "traffic": bc_traffic,
                         "algorithmic_bytes": bcb, "peak_source": hbm_kind},
         "sbr_tflops": round(flop / (t_sbr * 1e-3) / 1e12, 3) if t_sbr > 0 else None,
         "gpu_launches": int(launches),

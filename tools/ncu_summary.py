@@ -163,11 +163,9 @@ def main():
     if os.path.exists(tp) and read_ncu_csv(tp):
         t = summarize_traffic(tp)
         json.dump(t, open(out + "_traffic.json", "w"), indent=1)
-        merged_p = os.path.join(os.path.dirname(out), "ncu_traffic.json")
-        merged = json.load(open(merged_p)) if os.path.exists(merged_p) else {}
-        for c, v in t.items():
-            merged[f"n32768:{c}"] = v["dram_bytes_per_launch"]
-        json.dump(merged, open(merged_p, "w"), indent=1)
+        # per-class averages over every launch of the class (incl. its split-K reductions) stay in <out>_traffic.json;
+        # profiles/ncu_traffic.json (bench.py's roofline.traffic) holds per-kernel figures from --set full captures,
+        # curated by hand with their provenance
         print(json.dumps(t, indent=1))
     full = {}
     for f in sorted(os.listdir(src)):
