@@ -11,6 +11,7 @@
 // and per block:
 //   a5     syr2k  A(e:, e:) -= Y Z^T + Z Y^T  lower triangle, e = end of the block's last panel (l.15)
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <atomic>
@@ -128,6 +129,17 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
 }  // namespace
 
 namespace trid {
+// C = alpha A B + beta Cin with a short inner dimension (K <= b: W = Y T, Z = X - 1/2 Y S).  Measured at
+// n = 32768 (gpurun_out/r01x/env): the persistent warp-specialized engine beats the plain multi-CTA engine
+// here (wy 11.4 vs 14.6 ms, zy 142 vs 147 ms per step), so it is the default; TRID_SKINNY_WS=0 selects the
+// plain engine (A/B).
+cudaError_t gemm_skinny_k(GemmArgs g, cudaStream_t st) {
+  static const bool plain = getenv("TRID_SKINNY_WS") != nullptr && getenv("TRID_SKINNY_WS")[0] == '0';
+  if (!plain) return gemm_ws(g, OP_N, st);
+  g.splits = 1;
+  return gemm(g, OP_N, OP_N, TILE_128x64, st);
+}
+
 // ---- the Z builder after the SYMM (a3): corrections for the block's earlier panels (R4e), S = W^T X,
 // Z_p = X - 1/2 Y_p S (Eq. (1)).  X (m x kk, ld ldx) holds A_blk W_p on entry and is updated.
 cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
@@ -153,6 +165,14 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
     h.A[0] = Yprev; h.lda[0] = ldyz; h.B[0] = U1; h.ldb[0] = ldu; h.K[0] = nprev;
     h.A[1] = Zprev; h.lda[1] = ldyz; h.B[1] = U2; h.ldb[1] = ldu; h.K[1] = nprev;
     h.alpha = -1.0; h.beta = 1.0; h.Cin = X; h.ldcin = ldx; h.C = X; h.ldc = ldx;
+    // split-K as for the next-panel update (same m x b, K = 2 * nprev shape): the 128 x 64 tile grid alone is
+    // about one wave (measured: zy 161 -> 147 ms per step at n = 32768); TRID_XUPD_SPLIT=0 turns it off (A/B)
+    static const bool xsplit = !(getenv("TRID_XUPD_SPLIT") && getenv("TRID_XUPD_SPLIT")[0] == '0');
+    if (xsplit) {
+      h.splits = ws_skinny_splits(m, kk, 2 * nprev);
+      if ((int64_t)h.splits * m * kk > part_elems) h.splits = 1;
+      h.part = part; h.part_ld = m; h.part_stride = m * kk;
+    }
     if ((e = gemm_ws(h, OP_N, st)) != cudaSuccess) return e;
   }
   // S = W^T X
@@ -167,7 +187,7 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
   GemmArgs z;
   z.M = m; z.N = kk; z.K[0] = kk; z.A[0] = Yp; z.lda[0] = ldyz; z.B[0] = S; z.ldb[0] = lds;
   z.alpha = -0.5; z.beta = 1.0; z.Cin = X; z.ldcin = ldx; z.C = Zp; z.ldc = ldyz;
-  return gemm_ws(z, OP_N, st);
+  return gemm_skinny_k(z, st);
 }
 }  // namespace trid
 
@@ -357,7 +377,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
         g.M = m; g.N = kk; g.K[0] = kk; g.A[0] = Yp; g.lda[0] = ld; g.B[0] = w.T; g.ldb[0] = b;
         g.C = w.W; g.ldc = ld;
         ProfScope ps(PROF_WY, stream);
-        TRID_CUDA_TRY(gemm_ws(g, OP_N, stream));
+        TRID_CUDA_TRY(gemm_skinny_k(g, stream));
       }
       // Z builder against the implicitly updated trailing matrix (R4e)
       TRID_CUDA_TRY(zy_panel(m, kk, A + o + o * lda, lda, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ld,

@@ -25,6 +25,7 @@
 namespace trid {
 
 constexpr int BC_NT = 256;
+constexpr int BC_FLAG_STRIDE = 8;
 
 struct BcArgs {
   int64_t n;
@@ -36,6 +37,7 @@ struct BcArgs {
   int* prog;        // prog[s] = m+1: column 0 of step (s, m) published
   int* prog_full;   // prog_full[s] = m+1: all columns of step (s, m) stored
   unsigned* ticket;
+  int fs;           // flag stride in ints (bc_v6: one 32-byte sector per sweep counter; other kernels: 1)
   long long* trace;     // debug (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1
   int64_t trace_sweep;
 };
@@ -1045,14 +1047,14 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
           continue;
         }
         if (s > 0) {
-          if (m == 0) wait_geq_spin(a.prog + (s - 1), 1);
-          wait_geq_spin(a.prog_full + (s - 1), (int)(m + 1));
+          if (m == 0) wait_geq_spin(a.prog + (s - 1) * a.fs, 1);
+          wait_geq_spin(a.prog_full + (s - 1) * a.fs, (int)(m + 1));
         }
         BCW_TRACE(s, m, 8);
         fence_proxy_async_global();
         if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
         if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
-        if (s > 0) wait_geq_spin(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
+        if (s > 0) wait_geq_spin(a.prog + (s - 1) * a.fs, (int)((m + 2 < nprev) ? m + 2 : nprev));
         BCW_TRACE(s, m, 9);
         fence_proxy_async_global();
         bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
@@ -1091,13 +1093,13 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       }
       // CL: this step may have been fed by DSMEM before the producer's own global stores of the same columns
       // landed; never let an older global store overwrite ours (write-after-write on the band)
-      if (has_prod) wait_geq_spin(a.prog_full + (s - 1), m + 1);
+      if (has_prod) wait_geq_spin(a.prog_full + (s - 1) * a.fs, m + 1);
       bulk_s2g(a.band + r0 * ldab, c0s + bi * ldab, (unsigned)(ldab * 8));
       bulk_commit();
       bulk_wait_all();
       BCW_TRACE(s, m, 4);
       fence_proxy_async_global();
-      st_release_s32(a.prog + s, m + 1);
+      st_release_s32(a.prog + s * a.fs, m + 1);
       BCW_TRACE(s, m, 5);
       mbar_arrive(&c0done[bi]);
     }
@@ -1138,8 +1140,8 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       }
       if (has_prod) {   // as in STORE0: the producer's global stores of these columns landed first
         const int np = (int)bc_steps(n, b, s - 1);
-        wait_geq_spin(a.prog_full + (s - 1), m + 1);
-        wait_geq_spin(a.prog + (s - 1), m + 2 < np ? m + 2 : np);
+        wait_geq_spin(a.prog_full + (s - 1) * a.fs, m + 1);
+        wait_geq_spin(a.prog + (s - 1) * a.fs, m + 2 < np ? m + 2 : np);
       }
       if (L > 1) {
         bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
@@ -1153,7 +1155,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
         bulk_wait_all();
         fence_proxy_async_global();
       }
-      st_release_s32(a.prog_full + s, m + 1);
+      st_release_s32(a.prog_full + s * a.fs, m + 1);
       BCW_TRACE(s, m, 6);
     }
   }
@@ -1718,7 +1720,7 @@ __global__ void __launch_bounds__(2 * B + 64, 1) bc_row_kernel(BcArgs a) {
 
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
-  const size_t flags = sizeof(int) * (size_t)(2 * n + 128);
+  const size_t flags = sizeof(int) * (size_t)(2 * n + 128) * BC_FLAG_STRIDE;
   const size_t trace = sizeof(long long) * 2 * 1024 * 16;
   return ((band + 255) / 256) * 256 + ((flags + 255) / 256) * 256 + trace;
 }
@@ -1735,10 +1737,14 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   const int ldab = bc_ldab(n, beff);
   double* band = (double*)work;
   const size_t band_bytes = ((sizeof(double) * (size_t)n * ldab + 255) / 256) * 256;
+  // per-sweep counters: BC_FLAG_STRIDE ints apart for bc_v6 (no two sweeps' counters in one 32-byte sector),
+  // packed (stride 1) for the older kernels; the region is sized for the strided layout
+  const char* forcev = getenv("TRID_BC_FORCE");
+  const int fs = (beff <= 64 && (!forcev || forcev[0] == '6' || forcev[0] == '7')) ? BC_FLAG_STRIDE : 1;
   int* prog = (int*)((char*)work + band_bytes);
-  int* prog_full = prog + n + 32;
-  unsigned* ticket = (unsigned*)(prog_full + n + 32);
-  const size_t flags_bytes = ((sizeof(int) * (size_t)(2 * n + 128) + 255) / 256) * 256;
+  int* prog_full = prog + (n + 32) * fs;
+  unsigned* ticket = (unsigned*)(prog_full + (n + 32) * fs);
+  const size_t flags_bytes = ((sizeof(int) * (size_t)(2 * n + 128) * BC_FLAG_STRIDE + 255) / 256) * 256;
   long long* trace = (long long*)((char*)work + band_bytes + flags_bytes);
   const char* tr = getenv("TRID_BC_TRACE");
   {
@@ -1751,13 +1757,14 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
     if (err != cudaSuccess) return err;
   }
   if (beff >= 2 && n >= 3) {
-    cudaError_t err = cudaMemsetAsync(prog, 0, sizeof(int) * (size_t)(2 * n + 128), st);
+    cudaError_t err = cudaMemsetAsync(prog, 0, sizeof(int) * (size_t)(2 * n + 128) * fs, st);
     if (err != cudaSuccess) return err;
     BcArgs a;
     // beff = min(b, n-1) gives the same step geometry as b (for b >= n-1 every sweep is one step on
     // rows s+1..n-1); V2 keeps the caller's stride b (header contract).
     a.n = n; a.b = beff; a.ldab = ldab; a.vs = b; a.band = band; a.V2 = V2; a.tau2 = tau2; a.prog = prog;
     a.prog_full = prog_full;
+    a.fs = fs;
     a.ticket = ticket;
     a.trace = tr ? trace : nullptr;
     a.trace_sweep = tr ? atoll(tr) : -1;
