@@ -25,7 +25,7 @@
 namespace trid {
 
 constexpr int BC_NT = 256;
-constexpr int BC_FLAG_STRIDE = 8;
+constexpr int BC_FLAG_STRIDE = 32;   // workspace room per counter (ints); bc_v6 uses 8 (one sector) unless TRID_BC_FS
 
 struct BcArgs {
   int64_t n;
@@ -1740,7 +1740,10 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   // per-sweep counters: BC_FLAG_STRIDE ints apart for bc_v6 (no two sweeps' counters in one 32-byte sector),
   // packed (stride 1) for the older kernels; the region is sized for the strided layout
   const char* forcev = getenv("TRID_BC_FORCE");
-  const int fs = (beff <= 64 && (!forcev || forcev[0] == '6' || forcev[0] == '7')) ? BC_FLAG_STRIDE : 1;
+  const char* fse = getenv("TRID_BC_FS");
+  int fsv = fse ? atoi(fse) : 8;
+  if (fsv < 1 || fsv > BC_FLAG_STRIDE) fsv = 8;
+  const int fs = (beff <= 64 && (!forcev || forcev[0] == '6' || forcev[0] == '7')) ? fsv : 1;
   int* prog = (int*)((char*)work + band_bytes);
   int* prog_full = prog + (n + 32) * fs;
   unsigned* ticket = (unsigned*)(prog_full + (n + 32) * fs);

@@ -28,7 +28,7 @@ for _ in range(2):
 torch.cuda.synchronize()
 ldab = 2 * b
 band = (8 * n * ldab + 255) // 256 * 256
-flags = (4 * (2 * n + 128) * 8 + 255) // 256 * 256   # BC_FLAG_STRIDE = 8
+flags = (4 * (2 * n + 128) * 32 + 255) // 256 * 256   # BC_FLAG_STRIDE = 32
 tr = work[band + flags: band + flags + 8 * 2 * 1024 * 16].view(torch.int64).cpu().numpy().reshape(2, 1024, 16)
 tr = tr.astype(np.float64)
 steps = (n - 3 - (sw + 1)) // b + 1
