@@ -1143,7 +1143,10 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
         wait_geq_spin(a.prog_full + (s - 1) * a.fs, m + 1);
         wait_geq_spin(a.prog + (s - 1) * a.fs, m + 2 < np ? m + 2 : np);
       }
-      if (L > 1) {
+      // full windows (not CL): the compute threads stored columns 1..L-1 to the band themselves; their stores are
+      // ordered before prog_full by the CTA barrier + colsb arrival this warp synchronised with (release below)
+      const bool direct = !CL && bc_step_full(n, b, B, s, m);
+      if (L > 1 && !direct) {
         bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
         bulk_commit();
         bulk_wait_read();
@@ -1151,7 +1154,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       if (recv_need) cl_wait_geq(&recv_ctr, recv_need);   // the consumer holds both copies (they read this buffer)
       mbar_wait(&c0done[bi], ph);   // column 0's staging buffer was read too
       mbar_arrive(&empty[bi]);
-      if (L > 1) {
+      if (L > 1 && !direct) {
         bulk_wait_all();
         fence_proxy_async_global();
       }
@@ -1345,7 +1348,16 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       }
     }
     // D rows are final: write the lower triangle back (column 0 goes out through the staging buffer)
-    if (FULL && !isO) {
+    // full windows (not CL): final values go straight from registers to the global band (coalesced along the
+    // rows of a column); column 0 goes out through the staging buffer.  STORE1 then only releases prog_full
+    // (after the CTA barrier, like a split-K semaphore), so no shared write-back and no bulk store sit between
+    // this step's end and the next sweep's load of these columns.
+    double* const gwin = a.band + r0 * ldab + lo_base;   // element (r, j0 + jj) at gwin[jj * lda1]
+    if (FULL && !CL && !isO) {
+#pragma unroll
+      for (int jj = 0; jj < CPT; ++jj)
+        if (jj <= rj && j0 + jj >= 1) gwin[jj * lda1] = e[jj];
+    } else if (FULL && !isO) {
       // (column 0 is published from the staging buffer and never read back: a full window may write it)
 #pragma unroll
       for (int jj = 0; jj < CPT; ++jj)
@@ -1396,8 +1408,15 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       for (int jj = 0; jj < CPT; jj += 2) {
         const double2 x = za[jj / 2], y = zb[jj / 2];
         const double z0 = x.x + y.x, z1 = x.y + y.y;
-        if (j0 + jj >= 1) sts_f64(a_lo + 8u * (uint32_t)(jj * lda1), tau_next != 0.0 ? fma(-tv, z0, e[jj]) : e[jj]);
-        sts_f64(a_lo + 8u * (uint32_t)((jj + 1) * lda1), tau_next != 0.0 ? fma(-tv, z1, e[jj + 1]) : e[jj + 1]);
+        const double o0 = tau_next != 0.0 ? fma(-tv, z0, e[jj]) : e[jj];
+        const double o1 = tau_next != 0.0 ? fma(-tv, z1, e[jj + 1]) : e[jj + 1];
+        if constexpr (!CL) {
+          if (j0 + jj >= 1) gwin[jj * lda1] = o0;
+          gwin[(jj + 1) * lda1] = o1;
+        } else {
+          if (j0 + jj >= 1) sts_f64(a_lo + 8u * (uint32_t)(jj * lda1), o0);
+          sts_f64(a_lo + 8u * (uint32_t)((jj + 1) * lda1), o1);
+        }
       }
     } else if (isO) {
       const double tv = tau_next * vnr;
