@@ -1431,7 +1431,9 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
         }
       }
     }
-    fence_proxy_async_smem();
+    // the window goes out through a bulk store only for CL or ragged windows; full windows were stored from
+    // registers (a proxy fence here would also wait for those global stores)
+    if (CL || !FULL) fence_proxy_async_smem();
     if (tid == 0) BCW_TRACE(s, m, 14);
     if (a.V2) {
       double* vd = a.V2 + (off + m) * a.vs;
