@@ -149,6 +149,9 @@ def dist_env():
     return ws, rank, local
 
 
+METRIC = "FP64 TFLOPs (4n^3/3) full tridiag at n=32768, SBR/BC time split, 1/2/4/8 GPU"   # BASELINE.json
+
+
 def run_reference(args):
     ws, rank, _ = dist_env()
     if rank != 0:
@@ -162,7 +165,7 @@ def run_reference(args):
             times.append(r["seconds"])
     t = sum(times)
     value = 4.0 * n_s ** 3 / 3.0 * args.steps / t / 1e12
-    line = {"impl": "reference", "metric": "FP64 TFLOPs (4n^3/3) full tridiag", "value": round(value, 6),
+    line = {"impl": "reference", "metric": METRIC, "value": round(value, 6),
             "unit": "TFLOP/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(1e3 * t / args.steps, 3), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
@@ -323,7 +326,7 @@ def main():
     bc_gbs = bcb / (t_bc * 1e-3) / 1e9 if t_bc > 0 else 0.0
 
     line = {
-        "metric": "FP64 TFLOPs (4n^3/3) full tridiag at n=32768, SBR/BC time split, 1/2/4/8 GPU",
+        "metric": METRIC,
         "value": round(value, 4), "unit": "TFLOP/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "strong" if ws > 1 else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
