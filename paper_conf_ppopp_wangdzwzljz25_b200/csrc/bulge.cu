@@ -38,6 +38,8 @@ struct BcArgs {
   int* prog_full;   // prog_full[s] = m+1: all columns of step (s, m) stored
   unsigned* ticket;
   int fs;           // flag stride in ints (bc_v6: one 32-byte sector per sweep counter; other kernels: 1)
+  int opt;          // bc_v6 hand-off options (TRID_BC_OPT bitmask, A/B): 1 STORE0 spins on test_wait, 2 column 0
+                    // stored by its 2B threads (STORE0 only releases), 4 LOAD polls with acquire loads
   long long* trace;     // debug (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1
   int64_t trace_sweep;
 };
@@ -901,6 +903,26 @@ __device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
   (void)ld_acquire_s32(p);
 }
 
+__device__ __forceinline__ void mbar_spin(uint64_t* bar, unsigned parity) {
+  unsigned done = 0;
+  do {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void wait_geq_opt(const int* p, int need, bool acq_loop) {
+  if (acq_loop) {
+    while (ld_acquire_s32(p) < need) {
+    }
+  } else {
+    while (ld_relaxed_s32(p) < need) {
+    }
+    (void)ld_acquire_s32(p);
+  }
+}
 // 32-bit shared-window accesses for the full-window path (immediate offsets, no generic address arithmetic)
 __device__ __forceinline__ double lds_f64(uint32_t addr) {
   double v;
@@ -1047,14 +1069,14 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
           continue;
         }
         if (s > 0) {
-          if (m == 0) wait_geq_spin(a.prog + (s - 1) * a.fs, 1);
-          wait_geq_spin(a.prog_full + (s - 1) * a.fs, (int)(m + 1));
+          if (m == 0) wait_geq_opt(a.prog + (s - 1) * a.fs, 1, a.opt & 4);
+          wait_geq_opt(a.prog_full + (s - 1) * a.fs, (int)(m + 1), a.opt & 4);
         }
         BCW_TRACE(s, m, 8);
         fence_proxy_async_global();
         if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
         if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
-        if (s > 0) wait_geq_spin(a.prog + (s - 1) * a.fs, (int)((m + 2 < nprev) ? m + 2 : nprev));
+        if (s > 0) wait_geq_opt(a.prog + (s - 1) * a.fs, (int)((m + 2 < nprev) ? m + 2 : nprev), a.opt & 4);
         BCW_TRACE(s, m, 9);
         fence_proxy_async_global();
         bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
@@ -1068,7 +1090,8 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
     for (uint32_t it = 0;; ++it) {
       const int bi = it & 1;
       const unsigned ph = (it >> 1) & 1u;
-      mbar_wait(&col0b[bi], ph);
+      if (a.opt & 1) mbar_spin(&col0b[bi], ph);
+      else mbar_wait(&col0b[bi], ph);
       const int64_t s = info_s[bi];
       if (s < 0) return;
       const int m = info_m[bi];
@@ -1094,11 +1117,13 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       // CL: this step may have been fed by DSMEM before the producer's own global stores of the same columns
       // landed; never let an older global store overwrite ours (write-after-write on the band)
       if (has_prod) wait_geq_spin(a.prog_full + (s - 1) * a.fs, m + 1);
-      bulk_s2g(a.band + r0 * ldab, c0s + bi * ldab, (unsigned)(ldab * 8));
-      bulk_commit();
-      bulk_wait_all();
+      if (CL || !(a.opt & 2)) {
+        bulk_s2g(a.band + r0 * ldab, c0s + bi * ldab, (unsigned)(ldab * 8));
+        bulk_commit();
+        bulk_wait_all();
+        fence_proxy_async_global();
+      }
       BCW_TRACE(s, m, 4);
-      fence_proxy_async_global();
       st_release_s32(a.prog + s * a.fs, m + 1);
       BCW_TRACE(s, m, 5);
       mbar_arrive(&c0done[bi]);
@@ -1300,7 +1325,10 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
           red[2 * RW + 3] = h2.scale;
         }
       }
-      if (r < ldab) c0s[bi * ldab + r] = val;
+      if (r < ldab) {
+        c0s[bi * ldab + r] = val;
+        if (!CL && (a.opt & 2)) a.band[r0 * ldab + r] = val;
+      }
       fence_proxy_async_smem();
       mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
       if (tid == 0) BCW_TRACE(s, m, 1);
@@ -1789,6 +1817,10 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
     a.n = n; a.b = beff; a.ldab = ldab; a.vs = b; a.band = band; a.V2 = V2; a.tau2 = tau2; a.prog = prog;
     a.prog_full = prog_full;
     a.fs = fs;
+    {
+      const char* oe = getenv("TRID_BC_OPT");
+      a.opt = oe ? atoi(oe) : 0;
+    }
     a.ticket = ticket;
     a.trace = tr ? trace : nullptr;
     a.trace_sweep = tr ? atoll(tr) : -1;
