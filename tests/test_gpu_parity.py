@@ -165,6 +165,20 @@ def test_bulge_chase_cluster_forwarding_bitwise(n, b, cl, dev, monkeypatch):
         assert torch.equal(x, y)
 
 
+@pytest.mark.parametrize("env", [("TRID_BC_FS", "1"), ("TRID_BC_FS", "32"), ("TRID_BC_OPT", "1"), ("TRID_BC_OPT", "2"),
+                                 ("TRID_BC_OPT", "4"), ("TRID_BC_OPT", "7")])
+def test_bulge_chase_handoff_options_bitwise(env, dev, monkeypatch):
+    """Counter layout (TRID_BC_FS) and hand-off options (TRID_BC_OPT) change only how data and progress move
+    between CTAs, never the arithmetic: the chase output is bitwise that of the default (R9)."""
+    n, b = 3000, 64
+    Bm = band_from_lower(trid_gen.random_symmetric_np(n, 123), b)
+    ref = [x.clone() for x in trid.bulge_chase(to_dev(Bm), b)]
+    monkeypatch.setenv(*env)
+    got = trid.bulge_chase(to_dev(Bm), b)
+    for x, y in zip(ref, got):
+        assert torch.equal(x, y)
+
+
 def test_bulge_chase_bitwise_deterministic(dev):
     n, b = 2000, 32
     Bm = band_from_lower(trid_gen.random_symmetric_np(n, 11), b)
