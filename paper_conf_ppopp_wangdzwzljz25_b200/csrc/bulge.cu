@@ -894,9 +894,15 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
 //     for the rest of the step), and the new D(:,0), beta e1 are written to a column-0 staging buffer the
 //     STORE warp publishes (prog) while the full two-sided update, the z pass and the left application of
 //     the step continue on all compute threads;
-//   * the predecessor counters are polled without back-off (one lane per CTA).
-// The arithmetic of every element is the same expression as in bc_ws_kernel (fixed-order sums): bitwise
-// reproducible, independent of scheduling.
+//   * the rest of the step takes two barriers: the rank-2 update of D and the right update of O in registers,
+//     z = vn^T O by transposed warp butterflies from registers, then the left update of O;
+//   * full windows (L = L2 = b = B) are compiled separately (constant strides, warp-uniform D/O split) and
+//     store columns 1..L-1 straight from registers to the band; STORE1 then only releases prog_full after the
+//     CTA barrier (ragged windows and the CL variant bulk-store the shared window);
+//   * the per-sweep counters sit one 32-byte sector apart (a.fs) and are polled without back-off (one lane
+//     per CTA).
+// All sums run in a fixed order (the last-column term is added after the body, z is summed by fixed
+// butterflies): bitwise reproducible and independent of scheduling, though not bitwise equal to bc_ws_kernel.
 __device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
   while (ld_relaxed_s32(p) < need) {
   }
