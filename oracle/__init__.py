@@ -20,20 +20,69 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "trid_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
+# Compiler-flag builds of the same source (bench.py's cpu_baseline times the oracle "as it stands" under the
+# flags SURVEY 8(d) names; the code is never changed for speed).  The tests use the default -O2 build.
+FLAG_BUILDS = {"O2": ["-O2"], "O3native": ["-O3", "-march=native"]}
+_variant_libs = {}
 
 _D = ctypes.c_double
 _I = ctypes.c_int64
 _P = ctypes.c_void_p
 
 
-def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc (plain -O2, no fast-math)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(
+def _build_one(path, flags, force):
+    if force or not os.path.exists(path) or os.path.getmtime(path) < max(
             os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "trid_oracle.h"))):
-        tmp = _LIB + ".tmp%d" % os.getpid()
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-o", tmp, _SRC, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+        tmp = path + ".tmp%d" % os.getpid()
+        subprocess.check_call(["gcc", *flags, "-std=c11", "-fPIC", "-shared", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, path)
+    return path
+
+
+def build(force: bool = False, variant: str | None = None) -> str:
+    """Compile liboracle.so with gcc (plain -O2, no fast-math); variant (FLAG_BUILDS key) builds the same source
+    with other flags into liboracle_<variant>.so."""
+    if variant and variant != "O2":
+        return _build_one(os.path.join(_HERE, f"liboracle_{variant}.so"), FLAG_BUILDS[variant], force)
+    return _build_one(_LIB, FLAG_BUILDS["O2"], force)
+
+
+def timing_lib(variant: str):
+    """The oracle built with FLAG_BUILDS[variant] (for bench.py's cpu_baseline only)."""
+    if variant == "O2":
+        return lib()
+    if variant not in _variant_libs:
+        L = ctypes.CDLL(build(variant=variant))
+        L.oracle_sytd2.argtypes = [_I, _P, _I, _P, _P, _P]
+        L.oracle_sbr_naive.argtypes = [_I, _I, _P, _I, _P]
+        L.oracle_bc_naive.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, ctypes.c_int]
+        L.oracle_bc_total_steps.restype = _I
+        L.oracle_bc_total_steps.argtypes = [_I, _I]
+        _variant_libs[variant] = L
+    return _variant_libs[variant]
+
+
+def timed_run(kind: str, A, b: int, variant: str = "O2") -> float:
+    """Seconds for one run of O1 (kind "O1": sytd2) or O2 (kind "O2": naive SBR + naive bulge chase, vectors
+    stored) on A with the given flag build.  Timing only (bench.py cpu_baseline)."""
+    import time
+    L = timing_lib(variant)
+    A = _f(A)
+    n = A.shape[0]
+    d = np.zeros(n)
+    e = np.zeros(max(n - 1, 1))
+    t0 = time.perf_counter()
+    if kind == "O1":
+        tau = np.zeros(max(n - 1, 1))
+        L.oracle_sytd2(n, _p(A), max(n, 1), _p(d), _p(e), _p(tau))
+    else:
+        tau1 = np.zeros(n)
+        L.oracle_sbr_naive(n, b, _p(A), max(n, 1), _p(tau1))
+        tot = L.oracle_bc_total_steps(n, b)
+        V2 = np.zeros(max(tot * b, 1))
+        tau2 = np.zeros(max(tot, 1))
+        L.oracle_bc_naive(n, b, _p(A), max(n, 1), _p(d), _p(e), _p(V2), _p(tau2), 0)
+    return time.perf_counter() - t0
 
 
 def lib():
@@ -55,6 +104,8 @@ def lib():
         L.oracle_bc_total_steps.restype = _I
         L.oracle_bc_total_steps.argtypes = [_I, _I]
         L.oracle_bc_naive.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, ctypes.c_int]
+        L.oracle_bc_wavefront.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
+        L.oracle_bc_r7.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
         L.oracle_form_q.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
         L.oracle_sturm_eig.argtypes = [_I, _P, _P, _P]
         L.oracle_sturm_count.restype = _I
@@ -169,6 +220,32 @@ def bc_naive(A, b, full=False, want_v=True):
     if want_v:
         V2, tau2 = V2[: tot * b], tau2[:tot]
     return d, e, V2, tau2
+
+
+def bc_wavefront(A, b, lag):
+    """O2b in the pipelined wavefront order with the given lag (R9): returns (d, e, V2, tau2)."""
+    A = _f(A)
+    n = A.shape[0]
+    d = np.zeros(n)
+    e = np.zeros(max(n - 1, 0))
+    tot = bc_total_steps(n, b)
+    V2 = np.zeros(max(tot * b, 1))
+    tau2 = np.zeros(max(tot, 1))
+    lib().oracle_bc_wavefront(n, b, _p(A), max(n, 1), _p(d), _p(e), _p(V2), _p(tau2), lag)
+    return d, e, V2[: tot * b], tau2[:tot]
+
+
+def bc_r7(A, b, lag=0):
+    """O2c: the chase with R7's step grouping (lower triangle only); lag 0 sweep-major, lag >= 1 wavefront."""
+    A = _f(A)
+    n = A.shape[0]
+    d = np.zeros(n)
+    e = np.zeros(max(n - 1, 0))
+    tot = bc_total_steps(n, b)
+    V2 = np.zeros(max(tot * b, 1))
+    tau2 = np.zeros(max(tot, 1))
+    lib().oracle_bc_r7(n, b, _p(A), max(n, 1), _p(d), _p(e), _p(V2), _p(tau2), lag)
+    return d, e, V2[: tot * b], tau2[:tot]
 
 
 def form_q(n, b, A_sbr=None, tau1=None, V2=None, tau2=None):

@@ -269,61 +269,214 @@ int64_t oracle_bc_total_steps(int64_t n, int64_t b) {
   return t;
 }
 
-/* O2b: bulge chasing (sec. 2.4, Fig. 3, Alg. 2), sweep-major, on a dense full-storage copy.
- * Step (s, m): H from column col (= s for m = 0, else the first column of the previous block, which
- * holds the bulge's first column) over rows R_m = [r0, r1]; then A <- H A H, i.e. left-apply to the
+/* One bulge-chasing step (s, m) on the dense full-storage copy M (n x n, ld n) (sec. 2.4, Fig. 3, Alg. 2;
+ * step indexing R7).  H from column col (= s for m = 0, else the first column of the previous block, which
+ * holds the bulge's first column) over rows R_m = [r0, r1]; then M <- H M H, i.e. left-apply to the
  * off-band block (B_ol), two-sided to the diagonal block (B_d), right-apply to the block below (B_od,
- * which creates the bulge).  The eliminated entries are set to beta / exact zero. */
-void oracle_bc_naive(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e,
-                     double* V2, double* tau2, int full) {
-  if (n <= 0) return;
+ * which creates the bulge).  The eliminated entries are set to beta / exact zero.  full != 0 applies H to
+ * the whole matrix instead of the window rows/columns r0-2b .. r1+2b.  v (b doubles) and tmp (n) are
+ * scratch; the reflector goes to V2[off*b ..] / tau2[off] when those are non-NULL. */
+static void bc_step(int64_t n, int64_t b, double* M, int64_t s, int64_t m, int64_t off, double* V2, double* tau2,
+                    int full, double* v, double* tmp) {
+  int64_t r0 = s + 1 + m * b;
+  int64_t r1 = s + (m + 1) * b; if (r1 > n - 1) r1 = n - 1;
+  int64_t L = r1 - r0 + 1;
+  int64_t col = (m == 0) ? s : r0 - b;
+  for (int64_t r = 0; r < L; ++r) v[r] = M[col * n + r0 + r];
+  double beta;
+  double tau = oracle_house(L, v, 1, &beta);
+  v[0] = 1.0;
+  if (V2) { for (int64_t r = 0; r < b; ++r) V2[off * b + r] = r < L ? v[r] : 0.0; }
+  if (tau2) tau2[off] = tau;
+  if (tau != 0.0) {
+    int64_t lo = full ? 0 : (r0 - 2 * b > 0 ? r0 - 2 * b : 0);
+    int64_t hi = full ? n - 1 : (r1 + 2 * b < n - 1 ? r1 + 2 * b : n - 1);
+    /* left: rows R_m of columns lo..hi */
+    for (int64_t c = lo; c <= hi; ++c) {
+      double sum = 0.0;
+      for (int64_t r = 0; r < L; ++r) sum += v[r] * M[c * n + r0 + r];
+      sum *= tau;
+      for (int64_t r = 0; r < L; ++r) M[c * n + r0 + r] -= sum * v[r];
+    }
+    /* right: columns R_m of rows lo..hi */
+    for (int64_t i = lo; i <= hi; ++i) {
+      double sum = 0.0;
+      for (int64_t r = 0; r < L; ++r) sum += M[(r0 + r) * n + i] * v[r];
+      tmp[i] = tau * sum;
+    }
+    for (int64_t r = 0; r < L; ++r)
+      for (int64_t i = lo; i <= hi; ++i) M[(r0 + r) * n + i] -= tmp[i] * v[r];
+  }
+  M[col * n + r0] = beta; M[r0 * n + col] = beta;
+  for (int64_t r = 1; r < L; ++r) { M[col * n + r0 + r] = 0.0; M[(r0 + r) * n + col] = 0.0; }
+}
+
+/* Dense full-storage copy of the band (diagonal + b subdiagonals of A's lower triangle). */
+static double* bc_dense_band(int64_t n, int64_t b, const double* A, int64_t lda) {
   double* M = zalloc((size_t)(n * n));
   for (int64_t j = 0; j < n; ++j)
     for (int64_t i = j; i < n && i <= j + b; ++i) { M[j * n + i] = AT(A, i, j, lda); M[i * n + j] = AT(A, i, j, lda); }
+  return M;
+}
+
+static void bc_extract(int64_t n, const double* M, double* d, double* e) {
+  for (int64_t i = 0; i < n; ++i) d[i] = M[i * n + i];
+  for (int64_t i = 0; i + 1 < n; ++i) e[i] = M[i * n + i + 1];
+}
+
+/* O2b: naive sweep-major bulge chasing (sec. 2.4, Fig. 3, Alg. 2). */
+void oracle_bc_naive(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e,
+                     double* V2, double* tau2, int full) {
+  if (n <= 0) return;
+  double* M = bc_dense_band(n, b, A, lda);
   double* v = zalloc((size_t)(b > 1 ? b : 1));
   double* tmp = zalloc((size_t)n);
   int64_t off = 0;
   if (b >= 2) {
     for (int64_t s = 0; s + 3 <= n; ++s) {
       int64_t nst = oracle_bc_steps(n, b, s);
-      for (int64_t m = 0; m < nst; ++m, ++off) {
-        int64_t r0 = s + 1 + m * b;
-        int64_t r1 = s + (m + 1) * b; if (r1 > n - 1) r1 = n - 1;
-        int64_t L = r1 - r0 + 1;
-        int64_t col = (m == 0) ? s : r0 - b;
-        for (int64_t r = 0; r < L; ++r) v[r] = M[col * n + r0 + r];
-        double beta;
-        double tau = oracle_house(L, v, 1, &beta);
-        v[0] = 1.0;
-        if (V2) { for (int64_t r = 0; r < b; ++r) V2[off * b + r] = r < L ? v[r] : 0.0; }
-        if (tau2) tau2[off] = tau;
-        if (tau != 0.0) {
-          int64_t lo = full ? 0 : (r0 - 2 * b > 0 ? r0 - 2 * b : 0);
-          int64_t hi = full ? n - 1 : (r1 + 2 * b < n - 1 ? r1 + 2 * b : n - 1);
-          /* left: rows R_m of columns lo..hi */
-          for (int64_t c = lo; c <= hi; ++c) {
-            double sum = 0.0;
-            for (int64_t r = 0; r < L; ++r) sum += v[r] * M[c * n + r0 + r];
-            sum *= tau;
-            for (int64_t r = 0; r < L; ++r) M[c * n + r0 + r] -= sum * v[r];
-          }
-          /* right: columns R_m of rows lo..hi */
-          for (int64_t i = lo; i <= hi; ++i) {
-            double sum = 0.0;
-            for (int64_t r = 0; r < L; ++r) sum += M[(r0 + r) * n + i] * v[r];
-            tmp[i] = tau * sum;
-          }
-          for (int64_t r = 0; r < L; ++r)
-            for (int64_t i = lo; i <= hi; ++i) M[(r0 + r) * n + i] -= tmp[i] * v[r];
-        }
-        M[col * n + r0] = beta; M[r0 * n + col] = beta;
-        for (int64_t r = 1; r < L; ++r) { M[col * n + r0 + r] = 0.0; M[(r0 + r) * n + col] = 0.0; }
+      for (int64_t m = 0; m < nst; ++m, ++off) bc_step(n, b, M, s, m, off, V2, tau2, full, v, tmp);
+    }
+  }
+  bc_extract(n, M, d, e);
+  free(M); free(v); free(tmp);
+}
+
+/* The paper's pipelined order (reading R9) executed serially: in time slot t every
+ * sweep s with 0 <= t - lag*s < steps(s) runs its step m = t - lag*s, the sweeps of one slot taken from the
+ * highest s down (the order in which a real pipeline may complete them: a later sweep never waits for an
+ * earlier sweep's step of the same slot).  lag >= 1.  With lag >= 2 no step reads a window another step of
+ * its slot writes, so the result is the sweep-major one bit for bit; lag 1 lets sweep s read sweep s-1's
+ * window before sweep s-1 has updated it. */
+void oracle_bc_wavefront(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e,
+                         double* V2, double* tau2, int64_t lag) {
+  if (n <= 0) return;
+  double* M = bc_dense_band(n, b, A, lda);
+  double* v = zalloc((size_t)(b > 1 ? b : 1));
+  double* tmp = zalloc((size_t)n);
+  if (b >= 2 && n >= 3 && lag >= 1) {
+    const int64_t ns = n - 2;
+    int64_t* S = (int64_t*)calloc((size_t)ns + 1, sizeof(int64_t));
+    if (!S) abort();
+    for (int64_t s = 0; s < ns; ++s) S[s + 1] = S[s] + oracle_bc_steps(n, b, s);
+    const int64_t tmax = lag * (ns - 1) + oracle_bc_steps(n, b, 0);
+    for (int64_t t = 0; t < tmax; ++t) {
+      for (int64_t s = ns - 1; s >= 0; --s) {
+        const int64_t m = t - lag * s;
+        if (m < 0 || m >= oracle_bc_steps(n, b, s)) continue;
+        bc_step(n, b, M, s, m, S[s] + m, V2, tau2, 0, v, tmp);
       }
     }
+    free(S);
+  }
+  bc_extract(n, M, d, e);
+  free(M); free(v); free(tmp);
+}
+
+/* O2c: the same chase with the step grouping of reading R7, on the lower triangle only: step (s, m) owns the
+ * columns R_m.  Given its reflector v (generated from column s at m = 0, else by step m-1 of the sweep) it
+ * applies H = I - tau v v^T two-sided to D = B(R_m, R_m) (p = tau D v, w = p - 1/2 tau (p^T v) v,
+ * D -= v w^T + w v^T), from the right to O = B(R_{m+1}, R_m) (O -= tau (O v) v^T), generates the next
+ * reflector from O(:, 0) and applies it from the left to O(:, 1:) (the paper's "left-apply to B_ol" of the
+ * next step, moved into this one).  Same reflectors and T as O2b up to rounding.
+ * lag = 0: sweep-major order.  lag >= 1: the wavefront order of oracle_bc_wavefront (slot t runs step
+ * t - lag*s of every sweep, highest s first).  With this grouping a step touches only its own columns R_m
+ * (rows R_m u R_{m+1}), so lag 2 is the minimal lag that reproduces the sweep-major result bit for bit
+ * (reading R9); lag 1 reads a window before its predecessor finished it. */
+void oracle_bc_r7(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e, double* V2,
+                  double* tau2, int64_t lag) {
+  if (n <= 0) return;
+  double* M = zalloc((size_t)(n * n));   /* lower triangle only: M(i, j) = M[j*n + i], i >= j */
+  for (int64_t j = 0; j < n; ++j)
+    for (int64_t i = j; i < n && i <= j + b; ++i) M[j * n + i] = AT(A, i, j, lda);
+  if (b >= 2 && n >= 3) {
+    const int64_t ns = n - 2;
+    int64_t* S = (int64_t*)calloc((size_t)ns + 1, sizeof(int64_t));
+    double* vpend = zalloc((size_t)(ns * b));   /* per sweep: the reflector of its next step */
+    double* tpend = zalloc((size_t)ns);
+    double* p = zalloc((size_t)b);
+    double* y = zalloc((size_t)b);
+    double* z = zalloc((size_t)b);
+    if (!S) abort();
+    for (int64_t s = 0; s < ns; ++s) S[s + 1] = S[s] + oracle_bc_steps(n, b, s);
+    const int64_t lg = lag >= 1 ? lag : 0;
+    const int64_t tmax = lg ? lg * (ns - 1) + oracle_bc_steps(n, b, 0) : 1;
+    for (int64_t t = 0; t < tmax; ++t) {
+      for (int64_t q = 0; q < ns; ++q) {
+        const int64_t s = lg ? ns - 1 - q : q;
+        const int64_t m0 = lg ? t - lg * s : 0, m1 = lg ? m0 + 1 : oracle_bc_steps(n, b, s);
+        if (lg && (m0 < 0 || m0 >= oracle_bc_steps(n, b, s))) continue;
+        for (int64_t m = m0; m < m1; ++m) {
+          double* v = &vpend[s * b];
+          const int64_t r0 = s + 1 + m * b;
+          int64_t r1 = s + (m + 1) * b; if (r1 > n - 1) r1 = n - 1;
+          const int64_t L = r1 - r0 + 1;
+          int64_t r2 = r1 + b; if (r2 > n - 1) r2 = n - 1;
+          const int64_t L2 = r2 - r1;
+          double tau;
+          if (m == 0) {   /* the reflector annihilating column s below its first subdiagonal */
+            for (int64_t r = 0; r < L; ++r) v[r] = M[s * n + r0 + r];
+            double beta;
+            tau = oracle_house(L, v, 1, &beta);
+            v[0] = 1.0;
+            M[s * n + r0] = beta;
+            for (int64_t r = 1; r < L; ++r) M[s * n + r0 + r] = 0.0;
+          } else {
+            tau = tpend[s];
+          }
+          if (V2) for (int64_t r = 0; r < b; ++r) V2[(S[s] + m) * b + r] = r < L ? v[r] : 0.0;
+          if (tau2) tau2[S[s] + m] = tau;
+          if (tau != 0.0) {
+            /* two-sided on D (lower), right-apply to O */
+            for (int64_t i = 0; i < L; ++i) {
+              double acc = 0.0;
+              for (int64_t j = 0; j < L; ++j) {
+                const int64_t gi = r0 + i, gj = r0 + j;
+                acc += (gi >= gj ? M[gj * n + gi] : M[gi * n + gj]) * v[j];
+              }
+              p[i] = tau * acc;
+            }
+            for (int64_t i = 0; i < L2; ++i) {
+              double acc = 0.0;
+              for (int64_t j = 0; j < L; ++j) acc += M[(r0 + j) * n + r1 + 1 + i] * v[j];
+              y[i] = acc;
+            }
+            double pv = 0.0;
+            for (int64_t i = 0; i < L; ++i) pv += p[i] * v[i];
+            const double hp = 0.5 * tau * pv;
+            for (int64_t i = 0; i < L; ++i) p[i] -= hp * v[i];   /* p is now w */
+            for (int64_t j = 0; j < L; ++j)
+              for (int64_t i = j; i < L; ++i) M[(r0 + j) * n + r0 + i] -= v[i] * p[j] + p[i] * v[j];
+            for (int64_t j = 0; j < L; ++j)
+              for (int64_t i = 0; i < L2; ++i) M[(r0 + j) * n + r1 + 1 + i] -= tau * y[i] * v[j];
+          }
+          if (L2 > 0) {   /* next reflector from O(:, 0), left-applied to O(:, 1:) */
+            double* vn = z;   /* reuse: vn then copied into vpend */
+            for (int64_t i = 0; i < L2; ++i) vn[i] = M[r0 * n + r1 + 1 + i];
+            double beta;
+            const double tn = oracle_house(L2, vn, 1, &beta);
+            vn[0] = 1.0;
+            M[r0 * n + r1 + 1] = beta;
+            for (int64_t i = 1; i < L2; ++i) M[r0 * n + r1 + 1 + i] = 0.0;
+            if (tn != 0.0) {
+              for (int64_t j = 1; j < L; ++j) {
+                double acc = 0.0;
+                for (int64_t i = 0; i < L2; ++i) acc += vn[i] * M[(r0 + j) * n + r1 + 1 + i];
+                acc *= tn;
+                for (int64_t i = 0; i < L2; ++i) M[(r0 + j) * n + r1 + 1 + i] -= acc * vn[i];
+              }
+            }
+            for (int64_t i = 0; i < b; ++i) v[i] = i < L2 ? vn[i] : 0.0;
+            tpend[s] = tn;
+          }
+        }
+      }
+    }
+    free(S); free(vpend); free(tpend); free(p); free(y); free(z);
   }
   for (int64_t i = 0; i < n; ++i) d[i] = M[i * n + i];
   for (int64_t i = 0; i + 1 < n; ++i) e[i] = M[i * n + i + 1];
-  free(M); free(v); free(tmp);
+  free(M);
 }
 
 /* Q = Q1 Q2 (reading R2).  Right-multiplying by H = I - tau v v^T on index range [o, o+L). */

@@ -64,6 +64,17 @@ int64_t oracle_bc_total_steps(int64_t n, int64_t b);
 void oracle_bc_naive(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e,
                      double* V2, double* tau2, int full);
 
+/* O2b in the paper's pipelined order (reading R9), run serially: time slot t runs
+ * step t - lag*s of every sweep s that has it, highest s first.  Same outputs as oracle_bc_naive. */
+void oracle_bc_wavefront(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e,
+                         double* V2, double* tau2, int64_t lag);
+
+/* O2c: the chase with reading R7's step grouping (a step owns columns R_m; the next reflector is generated
+ * and left-applied inside the step), lower triangle only.  lag = 0 sweep-major, lag >= 1 the wavefront order
+ * above.  Same outputs as oracle_bc_naive up to rounding; lag 2 reproduces lag 0 bit for bit (R9). */
+void oracle_bc_r7(int64_t n, int64_t b, const double* A, int64_t lda, double* d, double* e, double* V2,
+                  double* tau2, int64_t lag);
+
 /* Dense Q = Q1 Q2 (reading R2): Q1 = prod_c H_c from the SBR vectors below the band of A_sbr and
  * tau1 (may be NULL: Q1 = I); Q2 = product of the bulge-chasing reflectors in sweep-major order
  * (V2/tau2 may be NULL: Q2 = I). */

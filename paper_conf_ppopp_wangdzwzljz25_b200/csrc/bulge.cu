@@ -42,6 +42,7 @@ struct BcArgs {
                     // stored by its 2B threads (STORE0 only releases), 4 LOAD polls with acquire loads
   long long* trace;     // debug (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1
   int64_t trace_sweep;
+  int serial;           // debug (TRID_BC_SERIAL=1): sweep s starts after sweep s-1 stored all its steps
 };
 
 __device__ __forceinline__ long long gtimer() {
@@ -168,7 +169,7 @@ __global__ void __launch_bounds__(BC_NT, 3) bc_kernel(BcArgs a) {
       // ---- lag-2 dependency (R9): sweep s-1 must have completed step m+1
       if (s > 0) {
         if (tid == 0) {
-          const int need = (int)((m + 2 < nprev) ? m + 2 : nprev);
+          const int need = (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev);
           wait_geq(a.prog + (s - 1), need);
         }
         __syncthreads();
@@ -306,295 +307,6 @@ __global__ void __launch_bounds__(BC_NT, 3) bc_kernel(BcArgs a) {
   }
 }
 
-// ---- fast path for b <= B (B = 32 or 64) -----------------------------------------------------------
-// Step (s, m) owns the compact columns R_m = [r0, r0+L).  Its window M = [D; O] ((L+L2) x L) is loaded
-// into shared memory by the bulk-copy engine and held in registers, one row slice per thread; a warp
-// covers 32 consecutive rows of one column group, so every compact-window access is bank-conflict free.
-// Dependencies (R9, refined by column ownership):
-//   * column 0 of step (s, m) is final as soon as the next reflector has been generated; it is the
-//     only column sweep s+1 needs to START its step m-1.  It is published first (1 KB bulk store,
-//     then prog[s] = m+1).
-//   * columns 1..L-1 are stored asynchronously afterwards and signalled with prog_full[s] = m+1 at the
-//     start of the next step; sweep s+1 only needs them for its prefetch of step m.
-//   * the window of step m+1 except its last column is prefetched while step m computes; after
-//     prog[s-1] >= m+2 only that last column (sweep s-1's published column 0) is loaded.
-// All sums are in a fixed order: results are bitwise reproducible and identical to sweep-major order.
-template <int B, int NTH, int NBUF>
-__global__ void __launch_bounds__(NTH, 3 - NBUF) bc_fast_kernel(BcArgs a) {
-  constexpr int TPR = NTH / (2 * B);   // column groups
-  constexpr int CPT = B / TPR;         // columns per thread
-  constexpr int RW = (2 * B) / 32;     // warps per column group
-  constexpr int NW = NTH / 32;
-  constexpr int CPW = B / NW;          // columns per warp in the z pass
-  static_assert(CPW == 4 || CPW == 8, "z-pass butterfly assumes 4 or 8 columns per warp");
-  extern __shared__ __align__(16) double sm[];
-  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
-  const int lda1 = ldab - 1;
-  const int64_t n = a.n;
-  const int wsz = B * ldab;
-  double* vb = sm + NBUF * wsz;              // 2 x B   (v / vn)
-  double* pyv = vb + 2 * B;                  // 2B      tau*D v | O v
-  double* zv = pyv + 2 * B;                  // B
-  double* part = zv + B;                     // TPR x 2B matvec partials
-  __shared__ int64_t s_sweep;
-  __shared__ __align__(8) uint64_t mbar[2];   // window buffers: 2 arrivals + tx bytes per use
-  if (tid == 0) {
-    mbar_init(&mbar[0], 2);
-    mbar_init(&mbar[1], 2);
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncthreads();
-  unsigned phase[2] = {0u, 0u};
-  int cur = 0;
-
-  for (;;) {
-    if (tid == 0) s_sweep = (int64_t)atomicAdd(a.ticket, 1u);
-    __syncthreads();
-    const int64_t s = s_sweep;
-    __syncthreads();
-    if (s > n - 3) return;
-    const int64_t nst = bc_steps(n, b, s);
-    const int64_t off = bc_offset(n, b, s);
-    const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
-    double tau = 0.0;
-    for (int64_t m = 0; m < nst; ++m) {
-      const int64_t r0 = s + 1 + m * b;
-      const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-      const int L = (int)(r1 - r0 + 1);
-      const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
-      const int L2 = (int)(r2 - r1);
-      const int bi = NBUF == 2 ? cur : 0;
-      double* win = sm + bi * wsz;
-      double* v = vb + (m & 1) * B;
-      double* vn = vb + ((m & 1) ^ 1) * B;
-      BC_TRACE(0);
-      if (tid == 0) {
-        if (m > 0) {  // step m-1's columns 1..L-1 are in L2 -> signal the prefetch of sweep s+1
-          bulk_wait_all();
-          fence_proxy_async_global();
-          st_release_s32(a.prog_full + s, (int)m);
-        }
-        if (s > 0) {
-          if (m == 0) wait_geq(a.prog_full + (s - 1), 1);
-          wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
-        }
-      }
-      __syncthreads();
-      BC_TRACE(1);
-      const double* gsrc = a.band + r0 * ldab;
-      if (m == 0) {
-        double* col = a.band + s * ldab + 1;
-        double sig = 0.0;
-        for (int i = 1 + lane; i < L; i += 32) {
-          const double x = __ldcg(col + i);
-          sig += x * x;
-        }
-        sig = warp_sum(sig);
-        const House hh = make_house(__ldcg(col), sig);
-        if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * __ldcg(col + tid) : 0.0);
-        __syncthreads();
-        if (tid < L) __stcg(col + tid, tid == 0 ? hh.beta : 0.0);
-        tau = hh.tau;
-        if (tid == 0) {
-          fence_proxy_async_smem();
-          fence_proxy_async_global();
-          mbar_arrive_expect_tx(&mbar[bi], (unsigned)(L * ldab * 8));
-          bulk_g2s(win, gsrc, (unsigned)(L * ldab * 8), &mbar[bi]);
-          mbar_arrive(&mbar[bi]);
-        }
-      } else if (tid == 0) {
-        fence_proxy_async_global();
-        mbar_arrive_expect_tx(&mbar[bi], (unsigned)(ldab * 8));
-        bulk_g2s(win + (L - 1) * ldab, gsrc + (L - 1) * ldab, (unsigned)(ldab * 8), &mbar[bi]);
-      }
-      mbar_wait(&mbar[bi], phase[bi]);
-      phase[bi] ^= 1u;
-      BC_TRACE(2);
-      const bool active = r < L + L2;
-      const bool isO = r >= L && active;
-      const int lo_base = j0 * lda1 + r;   // j <= r: j*(ldab-1) + r
-      const int hi_base = r * lda1 + j0;   // j >  r: r*(ldab-1) + j
-      double e[CPT];
-#pragma unroll
-      for (int jj = 0; jj < CPT; ++jj) {
-        const int j = j0 + jj;
-        e[jj] = win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
-      }
-      if (tau != 0.0) {
-        double acc0 = 0.0, acc1 = 0.0;
-#pragma unroll
-        for (int jj = 0; jj < CPT; jj += 2) {
-          acc0 = fma(e[jj], v[j0 + jj], acc0);
-          acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
-        }
-        part[hg * 2 * B + r] = acc0 + acc1;
-        __syncthreads();
-        if (tid < 2 * B) {
-          double acc = 0.0;
-#pragma unroll
-          for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + tid];
-          pyv[tid] = (tid >= L) ? acc : tau * acc;
-        }
-        __syncthreads();
-        BC_TRACE(3);
-        double pv = 0.0;
-        for (int i = lane; i < L; i += 32) pv += pyv[i] * v[i];
-        pv = warp_sum(pv);
-        const double hp = 0.5 * tau * pv;
-        if (isO) {
-          const double ty = tau * pyv[r];
-#pragma unroll
-          for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
-        } else {
-          const double vr = r < L ? v[r] : 0.0;
-          const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
-#pragma unroll
-          for (int jj = 0; jj < CPT; ++jj) {
-            const double vj = v[j0 + jj];
-            const double wj = fma(-hp, vj, pyv[j0 + jj]);
-            e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
-          }
-        }
-      }
-      // write back the lower part of D and all of O
-#pragma unroll
-      for (int jj = 0; jj < CPT; ++jj) {
-        const int j = j0 + jj;
-        if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
-      }
-      __syncthreads();
-      BC_TRACE(4);
-      // ---- next reflector from x = O(:, 0) (raw, at win[L + i]); every warp derives it identically
-      double tau_next = 0.0;
-      House h2;
-      h2.beta = 0.0;
-      h2.tau = 0.0;
-      h2.scale = 0.0;
-      if (L2 > 0) {
-        double sg = 0.0;
-        for (int i = 1 + lane; i < L2; i += 32) sg = fma(win[L + i], win[L + i], sg);
-        sg = warp_sum(sg);
-        h2 = make_house(win[L], sg);
-        tau_next = h2.tau;
-        if (tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : h2.scale * win[L + tid]) : 0.0;
-      }
-      // ---- z_j = vn^T O(:, j) = O(0, j) + scale * sum_{i>=1} x_i O(i, j), j >= 1 (reads raw column 0)
-      if (L2 > 0 && h2.tau != 0.0 && L > 1) {
-        const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
-        const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
-        double c[CPW];
-#pragma unroll
-        for (int q = 0; q < CPW; ++q) {
-          const int j = warp + q * NW;
-          double acc = 0.0;
-          if (j >= 1 && j < L) {
-            const int ob = j * lda1 + L;
-            if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
-            if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
-          }
-          c[q] = acc;
-        }
-        // transposed butterfly: CPW columns over 32 lanes, halving levels then full levels, fixed partners
-        {
-          int qbase = 0;
-#pragma unroll
-          for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
-            const bool up = (lane & o) != 0;
-#pragma unroll
-            for (int i = 0; i < K / 2; ++i) {
-              const double send = up ? c[i] : c[i + K / 2];
-              const double keep = up ? c[i + K / 2] : c[i];
-              c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
-            }
-            if (up) qbase += K / 2;
-          }
-          constexpr int LV = CPW == 4 ? 2 : 3;   // halving levels used
-          double f = c[0];
-#pragma unroll
-          for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
-          if ((lane & ((32 >> LV) - 1)) == 0) {
-            const int j = warp + qbase * NW;
-            if (j >= 1 && j < L) zv[j] = fma(h2.scale, f, win[j * lda1 + L]);
-          }
-        }
-      }
-      __syncthreads();   // all reads of the raw O(:, 0) done; zv ready
-      BC_TRACE(5);
-      // ---- finalize and publish column 0 (D(:,0) and the annihilated bulge column)
-      if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
-      __syncthreads();
-      if (tid == 0) {
-        fence_proxy_async_smem();
-        bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
-        bulk_commit();
-        bulk_wait_all();
-        fence_proxy_async_global();
-        st_release_s32(a.prog + s, (int)(m + 1));
-      }
-      BC_TRACE(6);
-      // ---- left-apply the next reflector to O(:, 1:)
-      if (L2 > 0 && h2.tau != 0.0 && isO) {
-        const double vni = vn[r - L];
-        const double tv = h2.tau * vni;
-#pragma unroll
-        for (int jj = 0; jj < CPT; ++jj) {
-          const int j = j0 + jj;
-          if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
-        }
-      }
-      __syncthreads();
-      BC_TRACE(7);
-      if (tid == 0) {
-        if (L > 1) {
-          fence_proxy_async_smem();
-          bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
-          bulk_commit();
-        }
-        // prefetch the next step's window (all but its last column) into the other buffer
-        if (m + 1 < nst) {
-          if (s > 0) wait_geq(a.prog_full + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
-          const int64_t q0 = r1 + 1;
-          const int64_t q1 = (r1 + b < n - 1) ? r1 + b : n - 1;
-          const unsigned bytes = (unsigned)((q1 - q0) * ldab * 8);   // (Lnext - 1) columns
-          const int nb2 = NBUF == 2 ? (cur ^ 1) : 0;
-          if (NBUF == 1) bulk_wait_read();   // single buffer: the stores above must have read it
-          fence_proxy_async_smem();
-          fence_proxy_async_global();
-          mbar_arrive_expect_tx(&mbar[nb2], bytes);
-          if (bytes) bulk_g2s(sm + nb2 * wsz, a.band + q0 * ldab, bytes, &mbar[nb2]);
-        }
-      }
-      if (a.V2) {
-        double* vd = a.V2 + (off + m) * a.vs;
-        for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
-        if (tid == 0) a.tau2[off + m] = tau;
-      }
-      BC_TRACE(8);
-      cur ^= 1;
-      tau = tau_next;
-    }
-    if (tid == 0) {
-      bulk_wait_all();
-      fence_proxy_async_global();
-      st_release_s32(a.prog_full + s, (int)nst);
-    }
-  }
-}
-
-// ---- warp-specialized chase (default for b <= 64) -----------------------------------------------------
-// Same step arithmetic and register-resident window as bc_fast_kernel, but no compute warp ever waits on
-// global memory: NTH compute threads (named barrier 1) + a LOAD warp + a STORE warp.
-//   LOAD  (lane 0): claims sweeps (atomic ticket), and for every step fills a window buffer by bulk copies
-//         completing on full[buf] (mbarrier, expect_tx): columns 0..L-2 once the predecessor sweep's
-//         prog_full reached m+1, the last column once its prog reached min(m+2, nprev) (R9, lag 2), plus
-//         column s at a sweep's step 0.  It runs one step ahead (prefetch) and only waits on the
-//         predecessor sweep and on empty[buf] (the STORE warp finished with that buffer).
-//   STORE (lane 0): waits col0[] (compute finalized column 0) -> bulk store, completion, st.release prog;
-//         waits cols[] (left-apply done) -> bulk store of columns 1..L-1, completion, release prog_full,
-//         then frees the buffer (empty[buf]).  It never waits on another CTA, so publication cannot be
-//         held up by this CTA's own prefetch (no cycle through the predecessor chain).
-// Step/sweep ids travel with the buffer (info[buf]); s < 0 terminates all roles.
 // debug trace (TRID_BC_TRACE=s): %globaltimer per step phase for sweeps s and s+1, slot k of 16
 #define BCW_TRACE(S, M, K)                                                                          \
   do {                                                                                              \
@@ -602,289 +314,20 @@ __global__ void __launch_bounds__(NTH, 3 - NBUF) bc_fast_kernel(BcArgs a) {
       a.trace[(((S)-a.trace_sweep) * 1024 + (M)) * 16 + (K)] = gtimer();                            \
   } while (0)
 
-template <int B, int NTH>
-__global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
-  constexpr int TPR = NTH / (2 * B);
-  constexpr int CPT = B / TPR;
-  constexpr int RW = (2 * B) / 32;
-  constexpr int NW = NTH / 32;
-  constexpr int CPW = B / NW;
-  static_assert(CPW == 4 || CPW == 8, "z-pass butterfly assumes 4 or 8 columns per warp");
-  extern __shared__ __align__(16) double sm[];
-  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int lda1 = ldab - 1;
-  const int64_t n = a.n;
-  const int wsz = B * ldab;
-  double* colb = sm + 2 * wsz;               // 2 x ldab: column s of a sweep's step 0, per buffer
-  double* vb = colb + 2 * ldab;              // 2 x B   (v / vn)
-  double* pyv = vb + 2 * B;                  // 2B
-  double* zv = pyv + 2 * B;                  // B
-  double* part = zv + B;                     // TPR x 2B
-  __shared__ __align__(8) uint64_t full[2], empty[2], col0b[2], colsb[2];
-  __shared__ int64_t info_s[2];
-  __shared__ int info_m[2];
-  if (tid == 0) {
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&full[i], 1);
-      mbar_init(&empty[i], 1);
-      mbar_init(&col0b[i], 1);
-      mbar_init(&colsb[i], 1);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncthreads();
-  if (warp == NW) {
-    // ============================== LOAD warp ==============================
-    if (lane != 0) return;
-    uint32_t it = 0;
-    for (;;) {
-      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
-      const bool done = s > n - 3;
-      const int64_t nst = done ? 1 : bc_steps(n, b, s);
-      const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
-      for (int64_t m = 0; m < nst; ++m, ++it) {
-        const int bi = it & 1;
-        if (it >= 2) mbar_wait(&empty[bi], ((it >> 1) - 1) & 1u);
-        if (done) {
-          info_s[bi] = -1;
-          mbar_arrive(&full[bi]);
-          return;
-        }
-        info_s[bi] = s;
-        info_m[bi] = (int)m;
-        BCW_TRACE(s, m, 7);
-        const int64_t r0 = s + 1 + m * b;
-        const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-        const int L = (int)(r1 - r0 + 1);
-        double* win = sm + bi * wsz;
-        mbar_arrive_expect_tx(&full[bi], (unsigned)((L + (m == 0 ? 1 : 0)) * ldab * 8));
-        if (s > 0) {
-          if (m == 0) wait_geq(a.prog + (s - 1), 1);
-          wait_geq(a.prog_full + (s - 1), (int)(m + 1));
-        }
-        BCW_TRACE(s, m, 8);
-        fence_proxy_async_global();
-        if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
-        if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
-        if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
-        BCW_TRACE(s, m, 9);
-        fence_proxy_async_global();
-        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &full[bi]);
-      }
-    }
-  }
-  if (warp == NW + 1) {
-    // ============================== STORE warp ==============================
-    if (lane != 0) return;
-    for (uint32_t it = 0;; ++it) {
-      const int bi = it & 1;
-      const unsigned ph = (it >> 1) & 1u;
-      mbar_wait(&col0b[bi], ph);
-      const int64_t s = info_s[bi];
-      if (s < 0) return;
-      const int m = info_m[bi];
-      const int64_t r0 = s + 1 + (int64_t)m * b;
-      const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
-      const int L = (int)(r1 - r0 + 1);
-      double* win = sm + bi * wsz;
-      BCW_TRACE(s, m, 3);
-      bulk_s2g(a.band + r0 * ldab, win, (unsigned)(ldab * 8));
-      bulk_commit();
-      bulk_wait_all();
-      BCW_TRACE(s, m, 4);
-      fence_proxy_async_global();
-      st_release_s32(a.prog + s, m + 1);
-      BCW_TRACE(s, m, 5);
-      mbar_wait(&colsb[bi], ph);
-      if (L > 1) {
-        bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
-        bulk_commit();
-        bulk_wait_all();
-        fence_proxy_async_global();
-      }
-      st_release_s32(a.prog_full + s, m + 1);
-      BCW_TRACE(s, m, 6);
-      mbar_arrive(&empty[bi]);
-    }
-  }
-  // ============================== compute warps ==============================
-  const int r = (warp % RW) * 32 + lane, hg = warp / RW, j0 = hg * CPT;
-  auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NTH) : "memory"); };
-  double tau = 0.0;
-  for (uint32_t it = 0;; ++it) {
-    const int bi = it & 1;
-    const unsigned ph = (it >> 1) & 1u;
-    mbar_wait(&full[bi], ph);
-    const int64_t s = info_s[bi];
-    if (s < 0) {
-      if (tid == 0) mbar_arrive(&col0b[bi]);   // wake the STORE warp so it can see the end
-      return;
-    }
-    const int64_t m = info_m[bi];
-    if (tid == 0) BCW_TRACE(s, m, 0);
-    const int64_t off = bc_offset(n, b, s);
-    const int64_t r0 = s + 1 + m * b;
-    const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-    const int L = (int)(r1 - r0 + 1);
-    const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
-    const int L2 = (int)(r2 - r1);
-    double* win = sm + bi * wsz;
-    double* v = vb + (m & 1) * B;
-    double* vn = vb + ((m & 1) ^ 1) * B;
-    if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
-      const double* col = colb + bi * ldab + 1;
-      double sig = 0.0;
-      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
-      sig = warp_sum(sig);
-      const House hh = make_house(col[0], sig);
-      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
-      if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
-      tau = hh.tau;
-      cbar();
-    }
-    const bool active = r < L + L2;
-    const bool isO = r >= L && active;
-    const int lo_base = j0 * lda1 + r;
-    const int hi_base = r * lda1 + j0;
-    double e[CPT];
-#pragma unroll
-    for (int jj = 0; jj < CPT; ++jj) {
-      const int j = j0 + jj;
-      e[jj] = win[j <= r ? lo_base + jj * lda1 : hi_base + jj];
-    }
-    if (tau != 0.0) {
-      double acc0 = 0.0, acc1 = 0.0;
-#pragma unroll
-      for (int jj = 0; jj < CPT; jj += 2) {
-        acc0 = fma(e[jj], v[j0 + jj], acc0);
-        acc1 = fma(e[jj + 1], v[j0 + jj + 1], acc1);
-      }
-      part[hg * 2 * B + r] = acc0 + acc1;
-      if (tid == 0) BCW_TRACE(s, m, 10);
-      cbar();
-      if (tid == 0) BCW_TRACE(s, m, 11);
-      if (tid < 2 * B) {
-        double acc = 0.0;
-#pragma unroll
-        for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + tid];
-        pyv[tid] = (tid >= L) ? acc : tau * acc;
-      }
-      cbar();
-      if (tid == 0) BCW_TRACE(s, m, 12);
-      double pv = 0.0;
-      for (int i = lane; i < L; i += 32) pv += pyv[i] * v[i];
-      pv = warp_sum(pv);
-      const double hp = 0.5 * tau * pv;
-      if (isO) {
-        const double ty = tau * pyv[r];
-#pragma unroll
-        for (int jj = 0; jj < CPT; ++jj) e[jj] = fma(-ty, v[j0 + jj], e[jj]);
-      } else {
-        const double vr = r < L ? v[r] : 0.0;
-        const double wr = r < L ? fma(-hp, vr, pyv[r]) : 0.0;
-#pragma unroll
-        for (int jj = 0; jj < CPT; ++jj) {
-          const double vj = v[j0 + jj];
-          const double wj = fma(-hp, vj, pyv[j0 + jj]);
-          e[jj] = fma(-wr, vj, fma(-vr, wj, e[jj]));
-        }
-      }
-    }
-#pragma unroll
-    for (int jj = 0; jj < CPT; ++jj) {
-      const int j = j0 + jj;
-      if (active && j < L && j <= r) win[lo_base + jj * lda1] = e[jj];
-    }
-    cbar();
-    if (tid == 0) BCW_TRACE(s, m, 13);
-    double tau_next = 0.0;
-    House h2;
-    h2.beta = 0.0;
-    h2.tau = 0.0;
-    h2.scale = 0.0;
-    if (L2 > 0) {
-      double sg = 0.0;
-      for (int i = 1 + lane; i < L2; i += 32) sg = fma(win[L + i], win[L + i], sg);
-      sg = warp_sum(sg);
-      h2 = make_house(win[L], sg);
-      tau_next = h2.tau;
-      if (tid < B) vn[tid] = tid < L2 ? (tid == 0 ? 1.0 : h2.scale * win[L + tid]) : 0.0;
-    }
-    if (L2 > 0 && h2.tau != 0.0 && L > 1) {
-      const double x0 = 1 + lane < L2 ? win[L + 1 + lane] : 0.0;
-      const double x1 = 33 + lane < L2 ? win[L + 33 + lane] : 0.0;
-      double c[CPW];
-#pragma unroll
-      for (int q = 0; q < CPW; ++q) {
-        const int j = warp + q * NW;
-        double acc = 0.0;
-        if (j >= 1 && j < L) {
-          const int ob = j * lda1 + L;
-          if (1 + lane < L2) acc = x0 * win[ob + 1 + lane];
-          if (33 + lane < L2) acc = fma(x1, win[ob + 33 + lane], acc);
-        }
-        c[q] = acc;
-      }
-      {
-        int qbase = 0;
-#pragma unroll
-        for (int o = 16, K = CPW; K > 1; o >>= 1, K >>= 1) {
-          const bool up = (lane & o) != 0;
-#pragma unroll
-          for (int i = 0; i < K / 2; ++i) {
-            const double send = up ? c[i] : c[i + K / 2];
-            const double keep = up ? c[i + K / 2] : c[i];
-            c[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
-          }
-          if (up) qbase += K / 2;
-        }
-        constexpr int LV = CPW == 4 ? 2 : 3;
-        double f = c[0];
-#pragma unroll
-        for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
-        if ((lane & ((32 >> LV) - 1)) == 0) {
-          const int j = warp + qbase * NW;
-          if (j >= 1 && j < L) zv[j] = fma(h2.scale, f, win[j * lda1 + L]);
-        }
-      }
-    }
-    cbar();   // all reads of the raw O(:, 0) done; zv ready
-    if (tid == 0) BCW_TRACE(s, m, 14);
-    if (L2 > 0 && tid < L2) win[L + tid] = tid == 0 ? h2.beta : 0.0;
-    fence_proxy_async_smem();
-    cbar();
-    if (tid == 0) BCW_TRACE(s, m, 15);
-    if (tid == 0) {
-      BCW_TRACE(s, m, 1);
-      mbar_arrive(&col0b[bi]);   // column 0 final -> STORE publishes it
-    }
-    if (L2 > 0 && h2.tau != 0.0 && isO) {
-      const double vni = vn[r - L];
-      const double tv = h2.tau * vni;
-#pragma unroll
-      for (int jj = 0; jj < CPT; ++jj) {
-        const int j = j0 + jj;
-        if (j >= 1 && j < L) win[lo_base + jj * lda1] = fma(-tv, zv[j], e[jj]);
-      }
-    }
-    fence_proxy_async_smem();
-    if (a.V2) {
-      double* vd = a.V2 + (off + m) * a.vs;
-      for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
-      if (tid == 0) a.tau2[off + m] = tau;
-    }
-    cbar();
-    if (tid == 0) {
-      BCW_TRACE(s, m, 2);
-      mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
-    }
-    tau = tau_next;
-  }
-}
-
 // ---- v6: warp-specialized chase with a short column-0 path (default for b <= 64) ------------------------
-// Same roles, window mapping and step arithmetic as bc_ws_kernel, reorganised around the chain that bounds
-// the chase (Delta per sweep = step period + link, link = predecessor's column 0 -> our column 0):
+// NTH compute threads (named barrier 1) + a LOAD warp + two STORE warps; no compute warp ever waits on global
+// memory.  The step window M = [D; O] ((L+L2) x L) is held in registers, one row slice per thread (a warp covers
+// 32 consecutive rows of one column group, so every compact-window access is bank-conflict free).
+//   LOAD  (lane 0): claims sweeps (atomic ticket), and for every step fills a window buffer by bulk copies
+//         completing on mbarriers (expect_tx): columns 0..L-2 once the predecessor sweep's prog_full reached
+//         m+1, the last column once its prog reached min(m+2, nprev) (R9, lag 2), plus column s at a sweep's
+//         step 0.  It runs one step ahead (prefetch) and only waits on the predecessor sweep and on the
+//         buffer's empty barrier.
+//   STORE0/STORE1 (lane 0 each): publish column 0 (prog) and columns 1..L-1 (prog_full), then free the buffer.
+//         They never wait on another CTA, so publication cannot be held up by this CTA's own prefetch.
+// Step/sweep ids travel with the buffer (info[buf]); s < 0 terminates all roles.  The design is organised
+// around the chain that bounds the chase (Delta per sweep = step period + link, link = predecessor's
+// column 0 -> our column 0):
 //   * the last window column (sweep s-1's freshly published column 0) lands on its own mbarrier (lastb);
 //     it contributes to one row of D v (the diagonal D(L-1,L-1)) and to every row of O v, so the body
 //     matvec (columns 0..L-2) and its cross-group reduction run while it is in flight;
@@ -902,7 +345,7 @@ __global__ void __launch_bounds__(NTH + 64, 1) bc_ws_kernel(BcArgs a) {
 //   * the per-sweep counters sit one 32-byte sector apart (a.fs) and are polled without back-off (one lane
 //     per CTA).
 // All sums run in a fixed order (the last-column term is added after the body, z is summed by fixed
-// butterflies): bitwise reproducible and independent of scheduling, though not bitwise equal to bc_ws_kernel.
+// butterflies): bitwise reproducible and independent of scheduling (tests: serialised-vs-parallel, R9).
 __device__ __forceinline__ void wait_geq_spin(const int* p, int need) {
   while (ld_relaxed_s32(p) < need) {
   }
@@ -1075,6 +518,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
           continue;
         }
         if (s > 0) {
+          if (m == 0 && a.serial) wait_geq_spin(a.prog_full + (s - 1) * a.fs, (int)nprev);
           if (m == 0) wait_geq_opt(a.prog + (s - 1) * a.fs, 1, a.opt & 4);
           wait_geq_opt(a.prog_full + (s - 1) * a.fs, (int)(m + 1), a.opt & 4);
         }
@@ -1492,287 +936,6 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   if constexpr (CL) cl_sync_all();   // no CTA leaves while a peer may still copy into / signal its shared memory
 }
 
-// ---- row-per-thread chase (experimental, TRID_BC_FORCE=4; measured slower: see DESIGN.md sec. 5) ---------------------------------------------------------
-// One compute thread per window row (2B threads: row r of [D; O], all L <= B columns in registers), plus the
-// LOAD and STORE warps of bc_ws_kernel.  A row's matvec needs no cross-thread reduction, so the path from
-// "last column arrived" to "column 0 published" is: one FMA (the body matvec is done while the last column
-// is in flight), one warp-sum + named barrier (p^T v), the column-0 update, one warp-sum + barrier (|x|^2),
-// the reflector, the stores of column 0 and one barrier before the st.release.  The remaining work (full
-// two-sided update, z = vn^T O by transposed warp butterflies, left application, write-back, V2) follows.
-template <int B>
-__global__ void __launch_bounds__(2 * B + 64, 1) bc_row_kernel(BcArgs a) {
-  constexpr int NT = 2 * B;           // compute threads = window rows
-  constexpr int NWc = NT / 32;        // compute warps
-  extern __shared__ __align__(16) double sm[];
-  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int lda1 = ldab - 1;
-  const int64_t n = a.n;
-  const int wsz = B * ldab;
-  double* colb = sm + 2 * wsz;        // 2 x ldab: column s of a sweep's step 0, per buffer
-  double* vb = colb + 2 * ldab;       // 2 x B   (v / vn)
-  double* pyv = vb + 2 * B;           // 2B      p (D rows) | y (O rows)
-  double* zs = pyv + 2 * B;           // NWc x B z partials
-  double* wred = zs + NWc * B;        // 2 x NWc warp partials (p^T v, |x|^2) + 2 (alpha)
-  __shared__ __align__(8) uint64_t full[2], lastb[2], empty[2], colsb[2];
-  __shared__ int64_t info_s[2];
-  __shared__ int info_m[2];
-  if (tid == 0) {
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&full[i], 1);
-      mbar_init(&lastb[i], 1);
-      mbar_init(&empty[i], 1);
-      mbar_init(&colsb[i], 1);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncthreads();
-
-  if (warp == NWc) {
-    // ============================== LOAD warp (as bc_ws_kernel) ==============================
-    if (lane != 0) return;
-    uint32_t it = 0;
-    for (;;) {
-      const int64_t s = (int64_t)atomicAdd(a.ticket, 1u);
-      const bool done = s > n - 3;
-      const int64_t nst = done ? 1 : bc_steps(n, b, s);
-      const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
-      for (int64_t m = 0; m < nst; ++m, ++it) {
-        const int bi = it & 1;
-        if (it >= 2) mbar_wait(&empty[bi], ((it >> 1) - 1) & 1u);
-        if (done) {
-          info_s[bi] = -1;
-          mbar_arrive(&full[bi]);
-          return;
-        }
-        info_s[bi] = s;
-        info_m[bi] = (int)m;
-        BCW_TRACE(s, m, 7);
-        const int64_t r0 = s + 1 + m * b;
-        const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-        const int L = (int)(r1 - r0 + 1);
-        double* win = sm + bi * wsz;
-        mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
-        mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
-        if (s > 0) {
-          if (m == 0) wait_geq(a.prog + (s - 1), 1);
-          wait_geq(a.prog_full + (s - 1), (int)(m + 1));
-        }
-        BCW_TRACE(s, m, 8);
-        fence_proxy_async_global();
-        if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
-        if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
-        if (s > 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev) ? m + 2 : nprev));
-        BCW_TRACE(s, m, 9);
-        fence_proxy_async_global();
-        bulk_g2s(win + (L - 1) * ldab, a.band + (r0 + L - 1) * ldab, (unsigned)(ldab * 8), &lastb[bi]);
-      }
-    }
-  }
-  if (warp == NWc + 1) {
-    // ============================== STORE warp: columns 1..L-1 ==============================
-    if (lane != 0) return;
-    for (uint32_t it = 0;; ++it) {
-      const int bi = it & 1;
-      const unsigned ph = (it >> 1) & 1u;
-      mbar_wait(&colsb[bi], ph);
-      const int64_t s = info_s[bi];
-      if (s < 0) return;
-      const int m = info_m[bi];
-      const int64_t r0 = s + 1 + (int64_t)m * b;
-      const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
-      const int L = (int)(r1 - r0 + 1);
-      double* win = sm + bi * wsz;
-      BCW_TRACE(s, m, 3);
-      if (L > 1) {
-        bulk_s2g(a.band + (r0 + 1) * ldab, win + ldab, (unsigned)((L - 1) * ldab * 8));
-        bulk_commit();
-        bulk_wait_all();
-        fence_proxy_async_global();
-      }
-      st_release_s32(a.prog_full + s, m + 1);
-      BCW_TRACE(s, m, 6);
-      mbar_arrive(&empty[bi]);
-    }
-  }
-  // ============================== compute threads: one window row each ==============================
-  auto cbar = [] { asm volatile("bar.sync 1, %0;\n" ::"n"(NT) : "memory"); };
-  const int r = tid;
-  double tau = 0.0;
-  int64_t off = 0;
-  for (uint32_t it = 0;; ++it) {
-    const int bi = it & 1;
-    const unsigned ph = (it >> 1) & 1u;
-    mbar_wait(&full[bi], ph);
-    const int64_t s = info_s[bi];
-    if (s < 0) {
-      if (tid == 0) mbar_arrive(&colsb[bi]);
-      return;
-    }
-    const int m = info_m[bi];
-    if (tid == 0) BCW_TRACE(s, m, 0);
-    const int64_t r0 = s + 1 + (int64_t)m * b;
-    const int64_t r1 = (s + ((int64_t)m + 1) * b < n - 1) ? s + ((int64_t)m + 1) * b : n - 1;
-    const int L = (int)(r1 - r0 + 1);
-    const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
-    const int L2 = (int)(r2 - r1);
-    double* win = sm + bi * wsz;
-    double* v = vb + (m & 1) * B;
-    double* vn = vb + ((m & 1) ^ 1) * B;
-    if (m == 0) {   // the reflector annihilating column s below its first subdiagonal (from colb)
-      off = bc_offset(n, b, s);
-      const double* col = colb + bi * ldab + 1;
-      double sig = 0.0;
-      for (int i = 1 + lane; i < L; i += 32) sig = fma(col[i], col[i], sig);
-      sig = warp_sum(sig);
-      const House hh = make_house(col[0], sig);
-      if (tid < B) v[tid] = tid == 0 ? 1.0 : (tid < L ? hh.scale * col[tid] : 0.0);
-      if (tid == 0) __stcg(a.band + s * ldab + 1, hh.beta);   // e_s (the rest of column s is dead)
-      tau = hh.tau;
-      cbar();
-    }
-    const bool active = r < L + L2;
-    const bool isD = r < L;
-    // ---- row r of [D; O] into registers; element (r, j) lives at win[j*lda1 + r] for j <= r (lower D and
-    // all of O) and at win[r*lda1 + j] for j > r (upper D = column r).  Only (r >= L-1, j = L-1) is in the
-    // separately loaded last column.
-    double e[B];
-    double acc0 = 0.0, acc1 = 0.0;
-#pragma unroll
-    for (int j = 0; j < B; ++j) {
-      double x = 0.0;
-      if (active && j < L && !(j == L - 1 && r >= L - 1)) x = win[j <= r ? j * lda1 + r : r * lda1 + j];
-      e[j] = x;
-      if (j & 1) acc1 = fma(x, v[j], acc1);
-      else acc0 = fma(x, v[j], acc0);
-    }
-    mbar_wait(&lastb[bi], ph);
-    if (tid == 0) BCW_TRACE(s, m, 10);
-    if (active && r >= L - 1) {
-#pragma unroll
-      for (int j = 0; j < B; ++j)
-        if (j == L - 1) {
-          e[j] = win[j * lda1 + r];
-          acc0 = fma(e[j], v[j], acc0);
-        }
-    }
-    const double vr = isD ? v[r] : 0.0;
-    const double raw0 = r < ldab ? win[r] : 0.0;   // column 0 (for rows past the window: untouched band)
-    double pr = 0.0, hp = 0.0, wr = 0.0;
-    if (tau != 0.0) {
-      pr = isD ? tau * (acc0 + acc1) : (acc0 + acc1);   // p_r = tau (D v)_r  |  y_r = (O v)_r
-      if (active) pyv[r] = pr;
-      double t = isD ? pr * vr : 0.0;
-      t = warp_sum(t);
-      if (lane == 0) wred[warp] = t;
-      cbar();
-      double pv = 0.0;
-#pragma unroll
-      for (int w = 0; w < NWc; ++w) pv += wred[w];
-      hp = 0.5 * tau * pv;
-      wr = fma(-hp, vr, pr);   // w_r = p_r - 1/2 tau (p^T v) v_r
-    }
-    if (tid == 0) BCW_TRACE(s, m, 11);
-    // ---- column 0 of the updated window, the next reflector from x = O(:, 0), publish column 0
-    double x0 = e[0];
-    if (tau != 0.0) {
-      if (isD) {
-        const double w0 = fma(-hp, v[0], pyv[0]);
-        x0 = fma(-wr, v[0], fma(-vr, w0, x0));
-      } else if (active) {
-        x0 = fma(-tau * pr, v[0], x0);
-      }
-    }
-    {
-      double t = (active && r > L) ? x0 * x0 : 0.0;
-      t = warp_sum(t);
-      if (lane == 0) wred[NWc + warp] = t;
-      if (r == L) wred[2 * NWc] = x0;
-    }
-    cbar();
-    House h2;
-    h2.beta = 0.0;
-    h2.tau = 0.0;
-    h2.scale = 0.0;
-    if (L2 > 0) {
-      double sg = 0.0;
-#pragma unroll
-      for (int w = 0; w < NWc; ++w) sg += wred[NWc + w];
-      h2 = make_house(wred[2 * NWc], sg);
-    }
-    if (r < ldab) {
-      const double outv = isD ? x0 : (active ? (r == L ? h2.beta : 0.0) : raw0);
-      __stcg(a.band + r0 * ldab + r, outv);
-    }
-    if (tid == 0) BCW_TRACE(s, m, 12);
-    cbar();
-    if (tid == 0) {
-      st_release_s32(a.prog + s, m + 1);   // cumulative over the compute threads' stores (bar.sync above)
-      BCW_TRACE(s, m, 1);
-      BCW_TRACE(s, m, 5);
-    }
-    // ---- the rest of the two-sided update (D) and the right update of the bulge (O)
-    if (tau != 0.0) {
-      if (isD) {
-#pragma unroll
-        for (int j = 0; j < B; ++j) {
-          const double vj = v[j];
-          const double wj = fma(-hp, vj, pyv[j]);
-          e[j] = fma(-wr, vj, fma(-vr, wj, e[j]));
-        }
-      } else if (active) {
-        const double ty = tau * pr;
-#pragma unroll
-        for (int j = 0; j < B; ++j) e[j] = fma(-ty, v[j], e[j]);
-      }
-    }
-    // e[0] now equals x0 (same arithmetic); next reflector vn (rows L..L+L2-1)
-    const bool isO = active && !isD;
-    const double vnr = isO ? (r == L ? 1.0 : h2.scale * e[0]) : 0.0;
-    if (r >= L && r - L < B) vn[r - L] = vnr;
-    // ---- write back columns 1..L-1 (lower D, all of O)
-    if (active) {
-#pragma unroll
-      for (int j = 1; j < B; ++j)
-        if (j < L && j <= r) win[j * lda1 + r] = e[j];
-    }
-    cbar();
-    if (tid == 0) BCW_TRACE(s, m, 13);
-    // ---- z_j = vn^T O(:, j), j >= 1 (thread j walks column j of O), then left-apply to O(:, 1:)
-    if (L2 > 0 && h2.tau != 0.0) {
-      if (r >= 1 && r < L) {
-        const double* oc = win + r * lda1 + L;   // O(i, r) = oc[i]
-        double z0 = 0.0, z1 = 0.0;
-        int i = 0;
-        for (; i + 1 < L2; i += 2) {
-          z0 = fma(vn[i], oc[i], z0);
-          z1 = fma(vn[i + 1], oc[i + 1], z1);
-        }
-        if (i < L2) z0 = fma(vn[i], oc[i], z0);
-        zs[r] = z0 + z1;
-      }
-      cbar();
-      if (isO) {
-        const double tv = h2.tau * vnr;
-#pragma unroll
-        for (int j = 1; j < B; ++j)
-          if (j < L) win[j * lda1 + r] = fma(-tv, zs[j], e[j]);
-      }
-    }
-    fence_proxy_async_smem();
-    if (a.V2) {
-      double* vd = a.V2 + (off + m) * a.vs;
-      for (int i = tid; i < a.vs; i += NT) vd[i] = i < L ? v[i] : 0.0;
-      if (tid == 0) a.tau2[off + m] = tau;
-    }
-    cbar();
-    if (tid == 0) {
-      BCW_TRACE(s, m, 2);
-      mbar_arrive(&colsb[bi]);   // columns 1..L-1 final -> STORE
-    }
-    tau = h2.tau;
-  }
-}
-
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
   const size_t flags = sizeof(int) * (size_t)(2 * n + 128) * BC_FLAG_STRIDE;
@@ -1792,13 +955,12 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   const int ldab = bc_ldab(n, beff);
   double* band = (double*)work;
   const size_t band_bytes = ((sizeof(double) * (size_t)n * ldab + 255) / 256) * 256;
-  // per-sweep counters: BC_FLAG_STRIDE ints apart for bc_v6 (no two sweeps' counters in one 32-byte sector),
-  // packed (stride 1) for the older kernels; the region is sized for the strided layout
-  const char* forcev = getenv("TRID_BC_FORCE");
+  // per-sweep counters: one 32-byte sector apart for bc_v6 (no two sweeps' counters share a sector), packed
+  // (stride 1) for bc_kernel (b > 64); the region is sized for the widest layout (BC_FLAG_STRIDE)
   const char* fse = getenv("TRID_BC_FS");
   int fsv = fse ? atoi(fse) : 8;
   if (fsv < 1 || fsv > BC_FLAG_STRIDE) fsv = 8;
-  const int fs = (beff <= 64 && (!forcev || forcev[0] == '6' || forcev[0] == '7')) ? fsv : 1;
+  const int fs = beff <= 64 ? fsv : 1;
   int* prog = (int*)((char*)work + band_bytes);
   int* prog_full = prog + (n + 32) * fs;
   unsigned* ticket = (unsigned*)(prog_full + (n + 32) * fs);
@@ -1808,7 +970,7 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   {
     int64_t total = n * (int64_t)ldab;
     int blocks = (int)((total + 255) / 256);
-    if (blocks > 8 * kNumSMsB200 * 4) blocks = 8 * kNumSMsB200 * 4;
+    if (blocks > 32 * num_sms()) blocks = 32 * num_sms();
     band_pack_kernel<<<blocks, 256, 0, st>>>(n, beff, ldab, X, cs, band);
     count_launches(1);
     cudaError_t err = cudaGetLastError();
@@ -1830,94 +992,64 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
     a.ticket = ticket;
     a.trace = tr ? trace : nullptr;
     a.trace_sweep = tr ? atoll(tr) : -1;
+    // TRID_BC_SERIAL=1 (debug/tests): ONE CTA, and a sweep starts only after its predecessor stored every step:
+    // the sweep-major order of the oracle (O2b), run by the same kernel.  Its output must equal the pipelined
+    // chase's bit for bit (R9: lag 2 reads exactly what sweep-major order reads).
+    const char* se = getenv("TRID_BC_SERIAL");
+    const bool serial = se && se[0] == '1';
+    a.serial = serial ? 1 : 0;
+    const int64_t max_grid = serial ? 1 : (n - 2);
     int occ = 1;
     if (beff <= 64) {
-      // default: bc_v6_kernel (warp-specialized, short column-0 path, 1 CTA/SM).  TRID_BC_FORCE (debug/tests):
-      // "1" the single-buffer 2-CTA/SM bc_fast_kernel, "2" the double-buffered bc_fast_kernel, "3" bc_ws_kernel,
-      // "4" bc_row_kernel.
+      // bc_v6_kernel (warp-specialized, short column-0 path, 1 CTA/SM).  TRID_BC_FORCE=7 (A/B, tests): the same
+      // kernel in CTA clusters with DSMEM forwarding between consecutive sweeps (measured slower).
       const int B = beff <= 32 ? 32 : 64;
       const char* force = getenv("TRID_BC_FORCE");
-      const int variant = force ? force[0] - '0' : 6;
-      if (variant == 6 || variant == 7) {
-        const int nth = B == 32 ? 256 : 512;
-        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 4 * (size_t)ldab + 2 * B + 2 * B + B + 16 +
-                                              (size_t)(nth / (2 * B)) * 2 * B + 2 * B + (2 * B / 32) * B + 8);
-        const void* fn6 = B == 32 ? (const void*)bc_v6_kernel<32, 256, false> : (const void*)bc_v6_kernel<64, 512, false>;
-        const void* fn7 = B == 32 ? (const void*)bc_v6_kernel<32, 256, true> : (const void*)bc_v6_kernel<64, 512, true>;
-        bool launched = false;
-        if (variant == 7) {
-          // clusters of C (env TRID_BC_CLUSTER, default 2) sized to the co-resident cluster count
-          const char* ce = getenv("TRID_BC_CLUSTER");
-          const int C = ce ? atoi(ce) : 2;
-          cudaFuncSetAttribute(fn7, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-          if (C > 8) cudaFuncSetAttribute(fn7, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-          cudaLaunchConfig_t cfg = {};
-          cfg.blockDim = dim3((unsigned)(nth + 96));
-          cfg.dynamicSmemBytes = smem;
-          cfg.stream = st;
-          cudaLaunchAttribute at[1];
-          at[0].id = cudaLaunchAttributeClusterDimension;
-          at[0].val.clusterDim.x = (unsigned)C;
-          at[0].val.clusterDim.y = 1;
-          at[0].val.clusterDim.z = 1;
-          cfg.attrs = at;
-          cfg.numAttrs = 1;
-          cfg.gridDim = dim3((unsigned)(C * 40));
-          int nc = 0;
-          if (C >= 2 && cudaOccupancyMaxActiveClusters(&nc, fn7, &cfg) == cudaSuccess && nc >= 1) {
-            int64_t ncl = nc;
-            const int64_t need = (n - 2 + C - 1) / C;   // clusters with at least one sweep
-            if (ncl > need) ncl = need;
-            cfg.gridDim = dim3((unsigned)(ncl * C));
-            cudaError_t le = B == 32 ? cudaLaunchKernelEx(&cfg, bc_v6_kernel<32, 256, true>, a)
-                                     : cudaLaunchKernelEx(&cfg, bc_v6_kernel<64, 512, true>, a);
-            if (le != cudaSuccess) return le;
-            launched = true;
-          } else {
-            (void)cudaGetLastError();
-          }
+      const bool cluster = force && force[0] == '7' && !serial;
+      const int nth = B == 32 ? 256 : 512;
+      const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 4 * (size_t)ldab + 2 * B + 2 * B + B + 16 +
+                                            (size_t)(nth / (2 * B)) * 2 * B + 2 * B + (2 * B / 32) * B + 8);
+      const void* fn6 = B == 32 ? (const void*)bc_v6_kernel<32, 256, false> : (const void*)bc_v6_kernel<64, 512, false>;
+      const void* fn7 = B == 32 ? (const void*)bc_v6_kernel<32, 256, true> : (const void*)bc_v6_kernel<64, 512, true>;
+      bool launched = false;
+      if (cluster) {
+        // clusters of C (env TRID_BC_CLUSTER, default 2) sized to the co-resident cluster count
+        const char* ce = getenv("TRID_BC_CLUSTER");
+        const int C = ce ? atoi(ce) : 2;
+        cudaFuncSetAttribute(fn7, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (C > 8) cudaFuncSetAttribute(fn7, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        cudaLaunchConfig_t cfg = {};
+        cfg.blockDim = dim3((unsigned)(nth + 96));
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = (unsigned)C;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cfg.gridDim = dim3((unsigned)(C * 40));
+        int nc = 0;
+        if (C >= 2 && cudaOccupancyMaxActiveClusters(&nc, fn7, &cfg) == cudaSuccess && nc >= 1) {
+          int64_t ncl = nc;
+          const int64_t need = (n - 2 + C - 1) / C;   // clusters with at least one sweep
+          if (ncl > need) ncl = need;
+          cfg.gridDim = dim3((unsigned)(ncl * C));
+          cudaError_t le = B == 32 ? cudaLaunchKernelEx(&cfg, bc_v6_kernel<32, 256, true>, a)
+                                   : cudaLaunchKernelEx(&cfg, bc_v6_kernel<64, 512, true>, a);
+          if (le != cudaSuccess) return le;
+          launched = true;
+        } else {
+          (void)cudaGetLastError();
         }
-        if (!launched) {
-          cudaFuncSetAttribute(fn6, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-          int64_t grid = kNumSMsB200;
-          if (grid > n - 2) grid = n - 2;
-          if (B == 32) bc_v6_kernel<32, 256, false><<<(unsigned)grid, 256 + 96, smem, st>>>(a);
-          else bc_v6_kernel<64, 512, false><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
-        }
-      } else if (variant == 4) {
-        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B +
-                                              (size_t)(2 * B / 32) * B + 2 * (2 * B / 32) + 8);
-        const void* fn = B == 32 ? (const void*)bc_row_kernel<32> : (const void*)bc_row_kernel<64>;
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        int64_t grid = kNumSMsB200;
-        if (grid > n - 2) grid = n - 2;
-        if (B == 32) bc_row_kernel<32><<<(unsigned)grid, 64 + 64, smem, st>>>(a);
-        else bc_row_kernel<64><<<(unsigned)grid, 128 + 64, smem, st>>>(a);
-      } else if (variant == 3) {
-        const int nth = B == 32 ? 256 : 512;
-        const size_t smem = sizeof(double) * (2 * (size_t)B * ldab + 2 * (size_t)ldab + 2 * B + 2 * B + B +
-                                              (size_t)(nth / (2 * B)) * 2 * B + 8);
-        const void* fn = B == 32 ? (const void*)bc_ws_kernel<32, 256> : (const void*)bc_ws_kernel<64, 512>;
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        int64_t grid = kNumSMsB200;
-        if (grid > n - 2) grid = n - 2;
-        if (B == 32) bc_ws_kernel<32, 256><<<(unsigned)grid, 256 + 64, smem, st>>>(a);
-        else bc_ws_kernel<64, 512><<<(unsigned)grid, 512 + 64, smem, st>>>(a);
-      } else {
-        const bool two = B == 64 && variant == 1;
-        const int nbuf = two ? 1 : 2;
-        const int nth = B == 32 ? 256 : (two ? 256 : 512);
-        const size_t smem = sizeof(double) * (nbuf * (size_t)B * ldab + 2 * B + 2 * B + B + 4 * 2 * B + 8);
-        const void* fn = B == 32 ? (const void*)bc_fast_kernel<32, 256, 2>
-                                 : (two ? (const void*)bc_fast_kernel<64, 256, 1> : (const void*)bc_fast_kernel<64, 512, 2>);
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, nth, smem);
-        if (occ < 1) occ = 1;
-        int64_t grid = (int64_t)kNumSMsB200 * occ;
-        if (grid > n - 2) grid = n - 2;
-        if (B == 32) bc_fast_kernel<32, 256, 2><<<(unsigned)grid, 256, smem, st>>>(a);
-        else if (two) bc_fast_kernel<64, 256, 1><<<(unsigned)grid, 256, smem, st>>>(a);
-        else bc_fast_kernel<64, 512, 2><<<(unsigned)grid, 512, smem, st>>>(a);
+      }
+      if (!launched) {
+        cudaFuncSetAttribute(fn6, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int64_t grid = num_sms();
+        if (grid > max_grid) grid = max_grid;
+        if (B == 32) bc_v6_kernel<32, 256, false><<<(unsigned)grid, 256 + 96, smem, st>>>(a);
+        else bc_v6_kernel<64, 512, false><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
       }
     } else {
       const size_t vec = sizeof(double) * (size_t)(5 * beff + 2 * BC_NT + 8);
@@ -1932,8 +1064,8 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<false>, BC_NT, smem);
       }
       if (occ < 1) occ = 1;
-      int64_t grid = (int64_t)kNumSMsB200 * occ;
-      if (grid > n - 2) grid = n - 2;
+      int64_t grid = (int64_t)num_sms() * occ;
+      if (grid > max_grid) grid = max_grid;
       if (use_sm) bc_kernel<true><<<(unsigned)grid, BC_NT, smem, st>>>(a);
       else bc_kernel<false><<<(unsigned)grid, BC_NT, smem, st>>>(a);
     }
@@ -1943,7 +1075,7 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   }
   {
     int blocks = (int)((n + 255) / 256);
-    if (blocks > 4 * kNumSMsB200) blocks = 4 * kNumSMsB200;
+    if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
     band_extract_kernel<<<blocks, 256, 0, st>>>(n, ldab, band, d, e);
     count_launches(1);
     return cudaGetLastError();

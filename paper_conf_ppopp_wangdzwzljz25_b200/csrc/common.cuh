@@ -6,13 +6,48 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ != 1000)
 #error "libtrid is written for sm_100a only"
 #endif
 
 namespace trid {
 
-constexpr int kNumSMsB200 = 148;
+constexpr int kNumSMsB200 = 148;   // B200 SM count: upper bound for grid-sized workspaces (partials, barriers)
+
+// ---- host: per-device cached attributes (thread-safe: libtrid is driven from several host threads by the
+// local multi-GPU ranks).  A racing first call may query twice; both store the same value.
+constexpr int kMaxDevices = 64;
+inline int cur_device() {
+  int d = 0;
+  if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= kMaxDevices) d = 0;
+  return d;
+}
+// SMs of the current device, capped at kNumSMsB200 (workspaces are sized for at most that many CTAs).
+inline int num_sms() {
+  static std::atomic<int> cache[kMaxDevices];
+  const int d = cur_device();
+  int v = cache[d].load(std::memory_order_relaxed);
+  if (v == 0) {
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d) != cudaSuccess || v < 1) v = kNumSMsB200;
+    if (v > kNumSMsB200) v = kNumSMsB200;
+    cache[d].store(v, std::memory_order_relaxed);
+  }
+  return v;
+}
+// Idempotent per-device setup (e.g. cudaFuncSetAttribute): runs f() until it succeeds once on this device.
+struct DeviceOnce {
+  std::atomic<unsigned long long> done{0};
+  template <class F>
+  cudaError_t operator()(F&& f) {
+    const unsigned long long bit = 1ull << cur_device();
+    if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+    const cudaError_t e = f();
+    if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+    return e;
+  }
+};
 
 // D(16x8) += A(16x8) * B(8x8), fp64.  Fragment layout (verified on B200, tools/microbench_fp64.cu):
 //   g = lane>>2, t = lane&3;  a[i] = A[g + 8*(i&1)][t + 4*(i>>1)];  b[i] = B[t + 4*i][g];

@@ -6,8 +6,7 @@
 //     Fig. 7: independent square tiles, reorderable)
 //   * the next-panel update                                                    (Alg. 1 l.8-12)
 //   * W = Y T, corrections and Z = X - 1/2 Y (W^T X)                            (Eq. (1))
-//   * the SYMM X = A W of the Z builder (symm_kernel: row strip + transposed column strip per row
-//     block, so the lower-stored trailing matrix is read without atomics; deterministic split-K).
+// (the SYMM X = A W of the Z builder runs on the warp-specialized engine, gemm_ws.cu)
 // Padded smem strides (4 mod 16 doubles) keep 64-bit DMMA fragment loads bank-conflict free.
 #include "common.cuh"
 #include "gemm.cuh"
@@ -259,13 +258,12 @@ template <int BM, int BN, int WGM, int WGN, int OPA, int OPB>
 static cudaError_t launch_tile(const GemmArgs& a, cudaStream_t st) {
   constexpr int NT = WGM * WGN * 32;
   constexpr size_t smem = sizeof(double) * STAGES * (ATile<BM, OPA>::ELEMS + BTile<BN, OPB>::ELEMS);
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BM, BN, WGM, WGN, OPA, OPB>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
+  static DeviceOnce attr;
+  cudaError_t e0 = attr([&] {
+    return cudaFuncSetAttribute(gemm_kernel<BM, BN, WGM, WGN, OPA, OPB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)smem);
+  });
+  if (e0 != cudaSuccess) return e0;
   const int64_t tm = (a.M + BM - 1) / BM, tn = (a.N + BN - 1) / BN;
   dim3 grid;
   GemmArgs b = a;
@@ -310,7 +308,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
   if (e != cudaSuccess || a.splits == 1 || a.sem) return e;
   int64_t total = a.M * a.N;
   int blocks = (int)((total + 127) / 128);   // small outputs (b x b, k x b): spread over many SMs
-  if (blocks > 4 * kNumSMsB200 * 8) blocks = 4 * kNumSMsB200 * 8;
+  if (blocks > 4 * num_sms() * 8) blocks = 4 * num_sms() * 8;
   reduce_partials_kernel<<<blocks, 128, 0, st>>>(a);
   count_launches(1);
   return cudaGetLastError();
@@ -319,7 +317,7 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st) {
 int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems) {
   const int bm = tile == TILE_128x64 ? 128 : 64, bn = tile == TILE_128x128 ? 128 : 64;
   const int64_t tiles = ((M + bm - 1) / bm) * ((N + bn - 1) / bn);
-  const int64_t target = 2 * kNumSMsB200;
+  const int64_t target = 2 * kNumSMsB200;   // fixed: the split count decides the summation order
   int64_t s = (target + tiles - 1) / tiles;
   const int64_t maxk = (K + 255) / 256;  // keep >= 256 of K per split
   if (s > maxk) s = maxk;
@@ -327,120 +325,6 @@ int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elem
   if (s < 1) s = 1;
   if (s > 128) s = 128;
   return (int)s;
-}
-
-// ------------------------------------------------------------------------------------------------
-// SYMM: X[r0:r0+BM, c0:c0+BN] = sum_k Asym(r, k) W(k, c) over the CTA's K chunk.
-//   phase 1 (row strip):    Asym(r, k) = A(r, k)   for k <= r   (k in [k0, min(k1, r0+BM)))
-//   phase 2 (column strip): Asym(r, k) = A(k, r)   for k >  r   (k in [max(k0, r0), k1))
-// Every CTA owns whole output tiles -> no atomics; split-K partials are reduced in fixed order.
-struct SymmArgs {
-  int64_t m, w;
-  const double* A;
-  int64_t lda;
-  const double* W;
-  int64_t ldw;
-  double* X;
-  int64_t ldx;
-  int64_t chunk;
-  int nchunk;
-  double* part;
-  int64_t part_stride;
-};
-
-constexpr int SY_BM = 128, SY_BN = 64, SY_WGM = 2, SY_WGN = 2;
-
-__global__ void __launch_bounds__(SY_WGM* SY_WGN * 32, 2) symm_kernel(SymmArgs a) {
-  constexpr int WTM = SY_BM / SY_WGM, WTN = SY_BN / SY_WGN;
-  constexpr int MT = WTM / 16, NTL = WTN / 8;
-  extern __shared__ __align__(16) double smem[];
-  const int64_t r0 = (int64_t)blockIdx.x * SY_BM, c0 = (int64_t)blockIdx.y * SY_BN;
-  const int z = blockIdx.z;
-  const int64_t k0 = (int64_t)z * a.chunk;
-  const int64_t k1 = (k0 + a.chunk < a.m) ? k0 + a.chunk : a.m;
-  double acc[MT][NTL][4];
-#pragma unroll
-  for (int i = 0; i < MT; ++i)
-#pragma unroll
-    for (int j = 0; j < NTL; ++j)
-#pragma unroll
-      for (int q = 0; q < 4; ++q) acc[i][j][q] = 0.0;
-  {
-    const int64_t e1 = (k1 < r0 + SY_BM) ? k1 : r0 + SY_BM;
-    mainloop<SY_BM, SY_BN, SY_WGM, SY_WGN, OP_N, OP_N, 1>(acc, smem, a.A, a.lda, a.W, a.ldw, r0, c0, a.m, a.w, k0, e1);
-    const int64_t s2 = (k0 > r0) ? k0 : r0;
-    mainloop<SY_BM, SY_BN, SY_WGM, SY_WGN, OP_T, OP_N, 2>(acc, smem, a.A, a.lda, a.W, a.ldw, r0, c0, a.m, a.w, s2, k1);
-  }
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int wm = warp % SY_WGM, wn = warp / SY_WGM;
-  const int g = lane >> 2, t = lane & 3;
-#pragma unroll
-  for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-    for (int nt = 0; nt < NTL; ++nt)
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int64_t r = r0 + wm * WTM + mt * 16 + g + (i >= 2 ? 8 : 0);
-        const int64_t c = c0 + wn * WTN + nt * 8 + 2 * t + (i & 1);
-        if (r < a.m && c < a.w) {
-          if (a.nchunk > 1) a.part[z * a.part_stride + r + c * a.m] = acc[mt][nt][i];
-          else a.X[r + c * a.ldx] = acc[mt][nt][i];
-        }
-      }
-}
-
-static int symm_nchunk(int64_t m, int64_t w) {
-  const int64_t blocks = ((m + SY_BM - 1) / SY_BM) * ((w + SY_BN - 1) / SY_BN);
-  const int64_t target = 3 * kNumSMsB200;  // ~3 CTAs per SM in flight for balance
-  int64_t c = (target + blocks - 1) / blocks;
-  const int64_t maxc = (m + 1023) / 1024;  // >= 1024 strip columns per chunk
-  if (c > maxc) c = maxc;
-  if (c > 32) c = 32;
-  if (c < 1) c = 1;
-  return (int)c;
-}
-
-int64_t symm_part_elems(int64_t m, int64_t w) {
-  int c = symm_nchunk(m, w);
-  return c > 1 ? (int64_t)c * m * w : 0;
-}
-
-cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw,
-                       double* X, int64_t ldx, double* part, int64_t part_elems, cudaStream_t st) {
-  if (m <= 0 || w <= 0) return cudaSuccess;
-  constexpr size_t smem =
-      sizeof(double) * STAGES *
-      ((ATile<SY_BM, OP_N>::ELEMS > ATile<SY_BM, OP_T>::ELEMS ? ATile<SY_BM, OP_N>::ELEMS : ATile<SY_BM, OP_T>::ELEMS) +
-       BTile<SY_BN, OP_N>::ELEMS);
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(symm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
-  SymmArgs a;
-  a.m = m; a.w = w; a.A = A; a.lda = lda; a.W = W; a.ldw = ldw; a.X = X; a.ldx = ldx;
-  int nc = symm_nchunk(m, w);
-  if ((int64_t)nc * m * w > part_elems) nc = 1;
-  a.nchunk = nc;
-  a.chunk = (((m + nc - 1) / nc) + BK - 1) / BK * BK;
-  a.nchunk = (int)((m + a.chunk - 1) / a.chunk);
-  a.part = part;
-  a.part_stride = m * w;
-  dim3 grid((unsigned)((m + SY_BM - 1) / SY_BM), (unsigned)((w + SY_BN - 1) / SY_BN), (unsigned)a.nchunk);
-  symm_kernel<<<grid, SY_WGM * SY_WGN * 32, smem, st>>>(a);
-  count_launches(1);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess || a.nchunk == 1) return e;
-  GemmArgs r;
-  r.M = m; r.N = w; r.alpha = 1.0; r.beta = 0.0; r.C = X; r.ldc = ldx;
-  r.splits = a.nchunk; r.part = part; r.part_ld = m; r.part_stride = m * w;
-  int64_t total = m * w;
-  int blocks = (int)((total + 255) / 256);
-  if (blocks > 16 * kNumSMsB200) blocks = 16 * kNumSMsB200;
-  reduce_partials_kernel<<<blocks, 256, 0, st>>>(r);
-  count_launches(1);
-  return cudaGetLastError();
 }
 
 }  // namespace trid

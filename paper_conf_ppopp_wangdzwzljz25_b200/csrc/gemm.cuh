@@ -61,12 +61,6 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st);
 // Choose a split count so the grid fills the machine for a tall reduction (K >> M, N).
 int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems);
 
-// X = Asym * W (m x w), Asym lower-referenced, ld lda.  Split-K over the strip when the row-block grid
-// is too small; partials need symm_part_elems() doubles.
-cudaError_t symm_lower(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw,
-                       double* X, int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);
-int64_t symm_part_elems(int64_t m, int64_t w);
-
 // Warp-specialized persistent engine (gemm_ws.cu): op(A) = A only; tiles 128x128 (N > 64) / 128x64.
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
 int64_t symm_ws_splits(int64_t m, int64_t w);

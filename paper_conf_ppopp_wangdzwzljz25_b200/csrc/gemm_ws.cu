@@ -471,19 +471,18 @@ __global__ void ws_reduce_kernel(int64_t M, int64_t N, int splits, const double*
 template <int BM, int BN, int CWM, int CWN, int OPB, bool MG = false>
 static cudaError_t launch(WsArgs& a, cudaStream_t st) {
   using C = Cfg<BM, BN>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(ws_kernel<BM, BN, CWM, CWN, OPB, MG>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
+  static DeviceOnce attr;
+  cudaError_t e0 = attr([] {
+    return cudaFuncSetAttribute(ws_kernel<BM, BN, CWM, CWN, OPB, MG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)C::SMEM);
+  });
+  if (e0 != cudaSuccess) return e0;
   a.tiles_m = (int)((a.M + BM - 1) / BM);
   a.tiles_n = (int)((a.N + BN - 1) / BN);
   if (a.tri && BM != BN) a.tri = 0;
   const int64_t tiles = a.tri ? (int64_t)a.tiles_m * (a.tiles_m + 1) / 2 : (int64_t)a.tiles_m * a.tiles_n;
   a.units = tiles * a.splits;
-  int64_t grid = a.units < kNumSMsB200 ? a.units : kNumSMsB200;
+  int64_t grid = a.units < num_sms() ? a.units : num_sms();
   if (grid < 1) return cudaSuccess;
   ws_kernel<BM, BN, CWM, CWN, OPB, MG><<<(unsigned)grid, (CWM * CWN + NPW) * 32, C::SMEM, st>>>(a);
   count_launches(1);
@@ -491,7 +490,7 @@ static cudaError_t launch(WsArgs& a, cudaStream_t st) {
   if (e != cudaSuccess || a.splits == 1) return e;
   int64_t total = a.M * a.N;
   int blocks = (int)((total + 255) / 256);
-  if (blocks > 16 * kNumSMsB200) blocks = 16 * kNumSMsB200;
+  if (blocks > 16 * num_sms()) blocks = 16 * num_sms();
   ws_reduce_kernel<<<blocks, 256, 0, st>>>(a.M, a.N, a.splits, a.part, a.part_ld, a.part_stride, a.alpha, a.beta,
                                            a.Cin, a.ldcin, a.C, a.ldc, a.lower, a.diag_off);
   count_launches(1);
@@ -535,7 +534,7 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
 // ~3 waves of the persistent grid, >= 256 of K per split, <= 16 splits.  Partials: splits * M * N doubles.
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {
   const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
-  int64_t sp = (3 * kNumSMsB200 + tiles - 1) / tiles;
+  int64_t sp = (3 * kNumSMsB200 + tiles - 1) / tiles;   // fixed (not the device's): sizes workspaces, fixes sums
   const int64_t maxs = K / 256;
   if (sp > maxs) sp = maxs;
   if (sp > 16) sp = 16;

@@ -135,7 +135,7 @@ cudaError_t launch_sum(double* dst, const std::vector<void*>& src, int g, int64_
   SumPtrs s{};
   for (int q = 0; q < g; ++q) s.p[q] = (const double*)src[q];
   int blocks = (int)((count + 255) / 256);
-  if (blocks > 8 * kNumSMsB200) blocks = 8 * kNumSMsB200;
+  if (blocks > 8 * num_sms()) blocks = 8 * num_sms();
   if (blocks < 1) blocks = 1;
   sum_ptrs_kernel<<<blocks, 256, 0, st>>>(dst, s, g, count);
   count_launches(1);
@@ -261,7 +261,7 @@ __global__ void band_scatter_kernel(double* AB, int64_t ldab, int64_t n, int b, 
 
 int grid_for(int64_t total) {
   int64_t blocks = (total + 255) / 256;
-  if (blocks > 8 * kNumSMsB200) blocks = 8 * kNumSMsB200;
+  if (blocks > 8 * num_sms()) blocks = 8 * num_sms();
   return blocks < 1 ? 1 : (int)blocks;
 }
 

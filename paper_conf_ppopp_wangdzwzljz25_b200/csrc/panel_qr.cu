@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(PQ_NT, 1) panel_qr_kernel(PanelArgs a) {
 
 static int panel_grid(int64_t m) {
   int64_t G = (m + 63) / 64;
-  if (G > kNumSMsB200) G = kNumSMsB200;
+  if (G > num_sms()) G = num_sms();   // 1 CTA/SM (launch bounds, shared memory): co-resident for the grid barrier
   if (G < 1) G = 1;
   return (int)G;
 }
@@ -229,12 +229,11 @@ cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, doub
   }
   a.t_smem = smem + tsz <= kMaxSmem ? 1 : 0;
   if (a.t_smem) smem += tsz;
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(panel_qr_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
-    if (e != cudaSuccess) return e;
-    attr_done = true;
-  }
+  static DeviceOnce attr;
+  cudaError_t e0 = attr([&] {
+    return cudaFuncSetAttribute(panel_qr_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
+  });
+  if (e0 != cudaSuccess) return e0;
   cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned), st);
   if (e != cudaSuccess) return e;
   void* args[] = {&a};

@@ -289,9 +289,51 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
 
 size_t panel_reg_gpart_bytes(int w) { return sizeof(double) * 2 * PR_MAXNC * 2 * (size_t)w; }
 
+static size_t panel_reg_smem(int w) {
+  return sizeof(double) * (size_t)(2 * 32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
+}
+static const void* panel_reg_fn(int w) {
+  return w == 16 ? (const void*)panel_reg_kernel<2>
+                 : (w == 32 ? (const void*)panel_reg_kernel<4> : (const void*)panel_reg_kernel<8>);
+}
+// Co-resident 4-CTA clusters of the kernel for width w on the current device (cached per device and width;
+// a racing first query stores the same value twice).  0 if the query fails (the caller then takes the general
+// panel kernel).
+static int panel_reg_max_clusters(int w) {
+  static std::atomic<int> cache[kMaxDevices][3];
+  const int wi = w == 16 ? 0 : (w == 32 ? 1 : 2);
+  const int d = cur_device();
+  int nc = cache[d][wi].load(std::memory_order_relaxed);
+  if (nc != 0) return nc < 0 ? 0 : nc;
+  const size_t smem = panel_reg_smem(w);
+  const void* fn = panel_reg_fn(w);
+  nc = -1;
+  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) == cudaSuccess) {
+    cudaLaunchConfig_t q = {};
+    q.gridDim = dim3(PR_CL * PR_MAXNC);
+    q.blockDim = dim3(PR_NT);
+    q.dynamicSmemBytes = smem;
+    cudaLaunchAttribute qa[1];
+    qa[0].id = cudaLaunchAttributeClusterDimension;
+    qa[0].val.clusterDim.x = PR_CL;
+    qa[0].val.clusterDim.y = 1;
+    qa[0].val.clusterDim.z = 1;
+    q.attrs = qa;
+    q.numAttrs = 1;
+    int v = 0;
+    if (cudaOccupancyMaxActiveClusters(&v, fn, &q) == cudaSuccess && v >= 1) nc = v > PR_MAXNC ? PR_MAXNC : v;
+  }
+  (void)cudaGetLastError();
+  cache[d][wi].store(nc, std::memory_order_relaxed);
+  return nc < 0 ? 0 : nc;
+}
+
 bool panel_reg_supported(int64_t m, int w) {
-  // 33 co-resident clusters of 4 (GPC packing on B200, 1 CTA/SM) x 256 rows per CTA
-  return (w == 16 || w == 32 || w == 64) && m <= (int64_t)PR_CL * 33 * 32 * PR_RL && m >= 1;
+  // every CTA holds <= 32 * PR_RL rows in registers, and the grid is limited to co-resident clusters (33 of 4
+  // on an idle B200: m <= 33792); otherwise (fewer SMs, MPS limits, taller panels) the general kernel runs
+  if (!(w == 16 || w == 32 || w == 64) || m < 1) return false;
+  const int nc = panel_reg_max_clusters(w);
+  return nc >= 1 && m <= (int64_t)PR_CL * nc * 32 * PR_RL;
 }
 
 cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
@@ -305,33 +347,13 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
     a.trace = (tr && atoll(tr) == m) ? (long long*)(gpart + 2 * (size_t)kNumSMsB200 * 2 * w + 2 * 2 * (size_t)w)
                                      : nullptr;
   }
-  const size_t smem = sizeof(double) * (size_t)(2 * 32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
-  // co-resident clusters of 8 (a cluster must fit in one GPC): query once per kernel instantiation
-  static int max_clusters[3] = {0, 0, 0};
-  const int wi = w == 16 ? 0 : (w == 32 ? 1 : 2);
-  const void* fn = w == 16 ? (const void*)panel_reg_kernel<2>
-                            : (w == 32 ? (const void*)panel_reg_kernel<4> : (const void*)panel_reg_kernel<8>);
-  if (!max_clusters[wi]) {
-    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaLaunchConfig_t q = {};
-    q.gridDim = dim3(PR_CL * PR_MAXNC);
-    q.blockDim = dim3(PR_NT);
-    q.dynamicSmemBytes = smem;
-    cudaLaunchAttribute qa[1];
-    qa[0].id = cudaLaunchAttributeClusterDimension;
-    qa[0].val.clusterDim.x = PR_CL;
-    qa[0].val.clusterDim.y = 1;
-    qa[0].val.clusterDim.z = 1;
-    q.attrs = qa;
-    q.numAttrs = 1;
-    int nc = 0;
-    if (cudaOccupancyMaxActiveClusters(&nc, fn, &q) != cudaSuccess || nc < 1) nc = 1;
-    max_clusters[wi] = nc > PR_MAXNC ? PR_MAXNC : nc;
-  }
+  const size_t smem = panel_reg_smem(w);
+  const int maxc = panel_reg_max_clusters(w);
+  if (maxc < 1) return cudaErrorInvalidConfiguration;   // caller checks panel_reg_supported
   // as few rows per CTA as possible within the co-resident clusters
   int64_t G = (m + 63) / 64;
   G = (G + PR_CL - 1) / PR_CL * PR_CL;
-  if (G > (int64_t)PR_CL * max_clusters[wi]) G = (int64_t)PR_CL * max_clusters[wi];
+  if (G > (int64_t)PR_CL * maxc) G = (int64_t)PR_CL * maxc;
   if (G < PR_CL) G = PR_CL;
   a.rows = (int)((m + G - 1) / G);
   if (a.rows > 32 * PR_RL) return cudaErrorInvalidConfiguration;   // caller checks panel_reg_supported
@@ -350,17 +372,26 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   attr[1].id = cudaLaunchAttributeCooperative;
   attr[1].val.cooperative = 1;
   cfg.attrs = attr;
-  // The cooperative attribute guarantees co-residency for the grid barrier.  ncu cannot replay a
-  // cooperative cluster launch, so profiling runs set TRID_PANEL_NOCOOP=1 (the grid fits in one wave:
-  // G <= 4 x max co-resident clusters, so on an otherwise idle GPU every CTA is resident anyway).
+  // The cooperative attribute guarantees co-residency for the grid barrier.  Profilers may refuse a cooperative
+  // cluster launch (plain ncu does); then, and with TRID_PANEL_NOCOOP=1, the grid is launched without it: it fits
+  // in one wave (G <= 4 x co-resident clusters), so on an otherwise idle GPU every CTA is resident anyway.
   static const bool nocoop = getenv("TRID_PANEL_NOCOOP") != nullptr;
   cfg.numAttrs = nocoop ? 1 : 2;
   count_launches(1);
-  switch (w) {
-    case 16: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<2>, a);
-    case 32: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<4>, a);
-    default: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<8>, a);
+  auto launch = [&]() -> cudaError_t {
+    switch (w) {
+      case 16: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<2>, a);
+      case 32: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<4>, a);
+      default: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<8>, a);
+    }
+  };
+  e = launch();
+  if (e != cudaSuccess && cfg.numAttrs == 2) {
+    (void)cudaGetLastError();
+    cfg.numAttrs = 1;
+    e = launch();
   }
+  return e;
 }
 
 }  // namespace trid

@@ -4,7 +4,7 @@ Q cannot be formed at n >= 8192, so:
   * G3 on prescribed-spectrum inputs (trid_gen.clustered_symmetric: the 1-2-1 Toeplitz spectrum in closed
     form, or 32 tight clusters), eigenvalues of T sampled one by one with the oracle's Sturm count
     (bisection to full precision), against the known eigenvalues: within 1e-12 ||A||_2;
-  * G1/G2 with Hutchinson probes through the returned reflectors (tests/qapply.py): <= 1e-14;
+  * G1/G2 with 16 Hutchinson probes through the returned reflectors (tests/qapply.py): <= 1e-14;
   * the stage split is checked too: the band after stage 1 has the input's spectrum (sampled)."""
 import numpy as np
 import pytest
@@ -54,7 +54,26 @@ def test_fullsize_gates(n, b, nb, k, kind, seed, dev):
     idx = np.unique(np.concatenate([[0, n - 1], rng.integers(0, n, 62)]))
     w = sampled_eigs(dn, en, idx)
     assert np.max(np.abs(w - lam[idx])) <= 1e-12 * norm2
-    g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b, p=4)
+    g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b, p=16)
+    assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
+
+
+def test_timed_input_gates(dev):
+    """The exact input bench.py times (configs[2]: n = 32768 random symmetric, seed 3001, b = 64, nb = 16,
+    k = 1024) in the bench's launch configuration: G1/G2 with 16 Hutchinson probes through the returned
+    reflectors, and G3 for 64 sampled eigenvalues of T against cuSOLVER syevd (torch.linalg.eigvalsh) of A."""
+    n, b, nb, k = 32768, 64, 16, 1024
+    A = trid_gen.random_symmetric(n, 3001, device="cuda:0")
+    lam = torch.linalg.eigvalsh(A).cpu().numpy()
+    A0 = A.clone()
+    d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=nb, k=k)
+    torch.cuda.synchronize()
+    norm2 = float(np.max(np.abs(lam)))
+    rng = np.random.default_rng(3001)
+    idx = np.unique(np.concatenate([[0, n - 1], rng.integers(0, n, 62)]))
+    w = sampled_eigs(d.cpu().numpy(), e.cpu().numpy(), idx)
+    assert np.max(np.abs(w - lam[idx])) <= 1e-12 * norm2
+    g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b, p=16)
     assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
 
 

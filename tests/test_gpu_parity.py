@@ -132,22 +132,39 @@ def test_bulge_chase_parity(n, b, dev):
     assert np.max(np.abs(V2.cpu().numpy() - V_o), initial=0) <= 1e-9
 
 
-@pytest.mark.parametrize("variant", ["1", "2", "3", "4", "6", "7"])
+@pytest.mark.parametrize("variant", ["6", "7"])
 def test_bulge_chase_b64_variants(variant, dev, monkeypatch):
-    """Every B=64 chase kernel (1: bc_fast 2 CTAs/SM single buffer, 2: bc_fast double buffer, 3: warp-specialized
-    bc_ws, 4: row-per-thread bc_row, 6: bc_v6 (default), 7: bc_v6 in CTA clusters with DSMEM forwarding) against
-    the oracle, bitwise reproducible."""
+    """The B=64 chase (6: bc_v6 (default), 7: bc_v6 in CTA clusters with DSMEM forwarding) against the oracle
+    (both the Alg. 2 grouping O2b and the R7 grouping O2c), bitwise reproducible."""
     monkeypatch.setenv("TRID_BC_FORCE", variant)
     n, b = 700, 64
     Bm = band_from_lower(trid_gen.random_symmetric_np(n, 99), b)
     d_o, e_o, V_o, t_o = oracle.bc_naive(Bm, b)
+    d7, e7, V7, t7 = oracle.bc_r7(Bm, b)
     d, e, V2, tau2 = trid.bulge_chase(to_dev(Bm), b)
     tol = 64 * n * U * np.linalg.norm(Bm)
-    assert np.max(np.abs(d.cpu().numpy() - d_o)) <= tol
-    assert np.max(np.abs(e.cpu().numpy() - e_o)) <= tol
-    assert np.max(np.abs(V2.cpu().numpy() - V_o)) <= 1e-9
+    for dr, er, Vr in ((d_o, e_o, V_o), (d7, e7, V7)):
+        assert np.max(np.abs(d.cpu().numpy() - dr)) <= tol
+        assert np.max(np.abs(e.cpu().numpy() - er)) <= tol
+        assert np.max(np.abs(V2.cpu().numpy() - Vr)) <= 1e-9
     r1 = [x.clone() for x in trid.bulge_chase(to_dev(Bm), b)]
     for x, y in zip(r1, (d, e, V2, tau2)):
+        assert torch.equal(x, y)
+
+
+@pytest.mark.parametrize("n,b", [(700, 32), (700, 64), (700, 128), (3000, 32), (3000, 64), (3000, 128), (2001, 48),
+                                 (12000, 32), (12000, 64), (12000, 128), (1500, 256)])
+def test_bulge_chase_serial_equals_parallel_bitwise(n, b, dev, monkeypatch):
+    """R9 and include/trid.h's promise: the pipelined chase (148 persistent CTAs, lag-2 progress counters) is bit
+    for bit the sweep-major chase.  TRID_BC_SERIAL=1 runs the same kernel on ONE CTA, starting a sweep only after
+    its predecessor stored every step (the oracle's order, O2b/O2c with lag 0); the oracle pins the lag rule
+    itself (tests/test_oracle.py::test_bc_lag_rule_r9)."""
+    Bm = band_from_lower(trid_gen.random_symmetric_np(n, 17 + n + b), b)
+    Ad = to_dev(Bm)
+    par = [x.clone() for x in trid.bulge_chase(Ad, b)]
+    monkeypatch.setenv("TRID_BC_SERIAL", "1")
+    ser = trid.bulge_chase(Ad, b)
+    for x, y in zip(par, ser):
         assert torch.equal(x, y)
 
 

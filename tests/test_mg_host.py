@@ -91,3 +91,21 @@ def test_gloo_two_rank_partition_and_id_exchange():
     for rank, ok_cover, ok_id, tmax, cnts in res:
         assert ok_cover and ok_id and tmax == 2.0
         assert cnts == [trid.mg_local_cols(n, cb, world, r) for r in range(world)]
+
+
+def test_bench_gpus_flag_spawns_ranks():
+    """bench.py --gpus N without a launcher re-runs itself under torch.distributed.run with N ranks (gloo dry run on
+    CPU: the rank plumbing the driver's multi-GPU bench uses), and refuses a --gpus / WORLD_SIZE mismatch."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--dry-run"],
+                         capture_output=True, text=True, timeout=300, env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    line = json.loads([x for x in out.stdout.splitlines() if x.startswith("{")][-1])
+    assert line["world_size"] == 2 and sorted(r[0] for r in line["ranks"]) == [0, 1]
+    bad = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--dry-run"],
+                         capture_output=True, text=True, timeout=120, env={**env, "WORLD_SIZE": "1"})
+    assert bad.returncode == 2

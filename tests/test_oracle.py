@@ -277,6 +277,47 @@ def test_bc_similarity_and_spectrum(n, b):
     assert np.all((tau2 == 0) | ((tau2 >= 1) & (tau2 <= 2)))
 
 
+@pytest.mark.parametrize("n,b", [(64, 8), (200, 8), (256, 32), (300, 17), (130, 64), (100, 2), (50, 100)])
+def test_bc_r7_grouping_equals_alg2_and_is_a_similarity(n, b):
+    """O2c (R7 grouping: the next reflector is generated and left-applied inside the step, lower triangle only)
+    computes O2b's reflectors and T up to rounding (amplified by the forward sensitivity of T, R15: a
+    diagnostic bound), and is itself an orthogonal similarity (pinned by the gates with its own reflectors, not
+    by O2b) with O2b's spectrum."""
+    B = band_from_lower(rand_sym(n, 3 + n), min(b, n - 1))
+    d, e, V2, tau2 = oracle.bc_naive(B, b)
+    d7, e7, V7, t7 = oracle.bc_r7(B, b)
+    tol = 1e-9 * np.linalg.norm(B)
+    assert np.max(np.abs(d - d7)) <= tol and np.max(np.abs(e - e7), initial=0) <= tol
+    assert np.max(np.abs(V2 - V7), initial=0) <= 1e-7 and np.max(np.abs(tau2 - t7), initial=0) <= 1e-7
+    w, w7 = oracle.sturm_eig(d, e), oracle.sturm_eig(d7, e7)
+    assert np.max(np.abs(w - w7)) <= 1e-12 * np.linalg.norm(B, 2)
+    Q2 = oracle.form_q(n, b, None, None, V7, t7)
+    g1, g2 = gates(B, Q2, d7, e7)
+    assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
+
+
+@pytest.mark.parametrize("n,b", [(200, 8), (256, 32), (300, 17), (130, 64), (100, 2)])
+def test_bc_lag_rule_r9(n, b):
+    """Reading R9: the sweeps pipelined in the wavefront order (slot t runs step t - lag*s
+    of every sweep, later sweeps first).
+      * R7 grouping (the GPU kernels' footprint: a step owns its columns R_m): lag 2 and lag 3 reproduce the
+        sweep-major result bit for bit; lag 1 is wrong (O(1) differences).
+      * Alg. 2's grouping (the left application of H_m to B_ol inside step m): lag 3 is bitwise
+        ("after the first three bulges"); lag 1 is wrong."""
+    B = band_from_lower(rand_sym(n, 3 + n), b)
+    ref7 = oracle.bc_r7(B, b, 0)
+    for lag in (2, 3):
+        got = oracle.bc_r7(B, b, lag)
+        assert all(np.array_equal(x, y) for x, y in zip(ref7, got)), lag
+    bad = oracle.bc_r7(B, b, 1)
+    assert np.max(np.abs(bad[0] - ref7[0])) > 1e-3
+    ref2 = oracle.bc_naive(B, b)
+    got3 = oracle.bc_wavefront(B, b, 3)
+    assert all(np.array_equal(x, y) for x, y in zip(ref2, got3))
+    bad2 = oracle.bc_wavefront(B, b, 1)
+    assert np.max(np.abs(bad2[0] - ref2[0])) > 1e-3
+
+
 def test_bc_noop_cases_bitwise():
     n = 30
     T = trid_gen.toeplitz121(n) + np.diag(np.linspace(0, 1, n))
