@@ -416,7 +416,7 @@ def main():
     value = flop * args.steps / (ms * 1e-3) / 1e12   # one matrix per step for every N (strong scaling)
     per = {c: (v[0] / args.steps, v[1] / args.steps) for c, v in stages.items()}
     t_bc = per["bulge_chase"][0]
-    t_sbr = sum(v[0] for c, v in per.items() if c != "bulge_chase")
+    t_sbr = sum(per[c][0] for c in trid.SBR_CLASSES)
 
     # roofline: the dominant DBBR contraction (largest time share) against the measured FP64 DMMA peak
     fl = dbbr_flops(n, b, k)

@@ -101,6 +101,41 @@ int trid_sytrd_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, d
                       double* tau1, double* V2, double* tau2, void* dwork, size_t dwork_bytes,
                       cudaStream_t stream);
 
+/* ---- eigenvalues of T (the eigenvalues-only EVD of P:446-448) ------------------------
+ * trid_stebz: w[0..n) = the eigenvalues of T = tridiag(e, d, e) in ascending order, by Sturm-sequence bisection
+ * (LAPACK dstebz/dlaebz definition: count of negative pivots of T - xI with the pivmin guard, Gershgorin start,
+ * stop at width <= 2 eps max(|lo|,|hi|) + pivmin; the gate G3's definition).  d[n], e[n-1], w[n] device arrays;
+ * d/e are not modified.  dwork: trid_stebz_bufsize bytes.  Accuracy: each w[k] is within 2 eps |w[k]| + pivmin
+ * of an exact eigenvalue of T (bisection on exact Sturm counts; Kahan's count is backward stable). */
+int trid_stebz_bufsize(int64_t n, size_t* dwork_bytes);
+int trid_stebz(int64_t n, const double* d, const double* e, double* w, void* dwork, size_t dwork_bytes,
+               cudaStream_t stream);
+
+/* trid_syevals_2stage: eigenvalues of the symmetric A (lower triangle, overwritten as by trid_sytrd_2stage) by
+ * DBBR + eigenvalues-only bulge chasing (no V2) + trid_stebz; w[n] ascending.  dwork: trid_syevals_2stage_bufsize
+ * bytes (holds d, e, tau1 and the stage workspaces).  Argument meanings as trid_sytrd_2stage. */
+int trid_syevals_2stage_bufsize(int64_t n, int b, int nb, int k, size_t* dwork_bytes);
+int trid_syevals_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* w, void* dwork,
+                        size_t dwork_bytes, cudaStream_t stream);
+
+/* ---- back-transformations: eigenvectors of A from those of T -------------------------
+ * trid_sbr_backtransform: C <- Q1 C (trans = 0) or Q1^T C (trans = 1) for the n x ncols matrix C (ld ldc), Q1 from
+ * the SBR vectors below A's band and tau1 as left by trid_sbr_dbbr / trid_sytrd_2stage (b, A, lda, tau1 exactly as
+ * passed there).  Method: sec. 4.3 Alg. 3 and sec. 5.3: the per-panel W blocks are merged
+ * recursively, W = [W1 | W2 - W1 Y1^T W2], into groups of k reflector columns (k = 0 -> 2048; else k >= b,
+ * k % b == 0), each applied as one block reflector with DMMA contractions.  A and tau1 are not modified.
+ * dwork: trid_sbr_backtransform_bufsize bytes (2 n k + k ncols doubles plus small buffers). */
+int trid_sbr_backtransform_bufsize(int64_t n, int b, int k, int64_t ncols, size_t* dwork_bytes);
+int trid_sbr_backtransform(int64_t n, int b, int k, const double* A, int64_t lda, const double* tau1, int trans,
+                           int64_t ncols, double* C, int64_t ldc, void* dwork, size_t dwork_bytes, cudaStream_t stream);
+
+/* trid_bc_backtransform: C <- Q2 C (trans = 0) or Q2^T C (trans = 1), Q2 from V2/tau2 as returned by
+ * trid_bulge_chase (same n and b; R7 layout).  Blocks of consecutive sweeps are regrouped by step (only reflectors
+ * on disjoint rows are reordered: the product is Q2 exactly) and applied to 32-column slabs of C, one CTA each.
+ * No workspace.  V2/tau2 may be NULL only when the chase stores no reflector (n < 3 or b < 2). */
+int trid_bc_backtransform(int64_t n, int b, const double* V2, const double* tau2, int trans, int64_t ncols, double* C,
+                          int64_t ldc, cudaStream_t stream);
+
 /* ---- stage 2 from LAPACK lower band storage (dsbtrd-style input): AB[(i-j) + j*ldab] = B(i, j) for
  * 0 <= i-j <= b, ldab >= b+1 (the layout trid_band_gather produces).  Otherwise as trid_bulge_chase. */
 int trid_bulge_chase_band(int64_t n, int b, const double* AB, int64_t ldab, double* d, double* e, double* V2,
@@ -146,7 +181,8 @@ int trid_band_gather(trid_comm_t comm, int64_t n, int b, const double* A_local, 
  * those events and returns, per stage class, the summed elapsed milliseconds and the number of stage
  * instances; classes: 0 panel QR (a1/a2), 1 W = Y T, 2 SYMM X = A W (a3), 3 Z-builder corrections and
  * Z = X - 1/2 Y W^T X (a3), 4 next-panel update (a4), 5 deferred syr2k (a5), 6 bulge chase incl. band
- * pack and d/e extraction (a6/a7).  Either pointer may be NULL.  Process-global state (not reentrant).
+ * pack and d/e extraction (a6/a7), 7 Sturm bisection (trid_stebz), 8 SBR back-transformation, 9 BC
+ * back-transformation.  Either pointer may be NULL.  Process-global state (not reentrant).
  * trid_kernel_launches(): total number of CUDA kernels this library has launched in the process. */
 int trid_profile_begin(void);
 int trid_profile_end(double* ms, int64_t* calls, int nclass);

@@ -106,6 +106,8 @@ def lib():
         L.oracle_bc_naive.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, ctypes.c_int]
         L.oracle_bc_wavefront.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
         L.oracle_bc_r7.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
+        L.oracle_sbr_backtransform.argtypes = [_I, _I, _P, _I, _P, ctypes.c_int, _I, _P, _I]
+        L.oracle_bc_backtransform.argtypes = [_I, _I, _P, _P, ctypes.c_int, _I, _P, _I]
         L.oracle_form_q.argtypes = [_I, _I, _P, _I, _P, _P, _P, _P, _I]
         L.oracle_sturm_eig.argtypes = [_I, _P, _P, _P]
         L.oracle_sturm_count.restype = _I
@@ -246,6 +248,26 @@ def bc_r7(A, b, lag=0):
     tau2 = np.zeros(max(tot, 1))
     lib().oracle_bc_r7(n, b, _p(A), max(n, 1), _p(d), _p(e), _p(V2), _p(tau2), lag)
     return d, e, V2[: tot * b], tau2[:tot]
+
+
+def sbr_backtransform(A_sbr, tau1, b, C, trans=False):
+    """C <- Q1 C (or Q1^T C) from the SBR vectors below the band of A_sbr (sec. 4.3), one reflector at a time."""
+    A_sbr = _f(A_sbr)
+    C = _f(C)
+    n, ncols = C.shape
+    tau1 = np.ascontiguousarray(tau1, dtype=np.float64)
+    lib().oracle_sbr_backtransform(n, b, _p(A_sbr), max(n, 1), _p(tau1), 1 if trans else 0, ncols, _p(C), max(n, 1))
+    return C
+
+
+def bc_backtransform(V2, tau2, b, C, trans=False):
+    """C <- Q2 C (or Q2^T C) from the bulge-chasing reflectors (R7 layout), one reflector at a time."""
+    C = _f(C)
+    n, ncols = C.shape
+    V2 = np.ascontiguousarray(V2, dtype=np.float64)
+    tau2 = np.ascontiguousarray(tau2, dtype=np.float64)
+    lib().oracle_bc_backtransform(n, b, _p(V2), _p(tau2), 1 if trans else 0, ncols, _p(C), max(n, 1))
+    return C
 
 
 def form_q(n, b, A_sbr=None, tau1=None, V2=None, tau2=None):

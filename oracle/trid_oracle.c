@@ -517,6 +517,65 @@ void oracle_form_q(int64_t n, int64_t b, const double* A_sbr, int64_t lda, const
   free(v);
 }
 
+/* SBR back-transformation (sec. 4.3): C <- Q1 C (trans = 0) or Q1^T C
+ * (trans = 1), Q1 = H_0 H_1 ... H_{n-b-2} with H_c = I - tau1[c] v_c v_c^T, v_c = (1, A(c+b+1:n-1, c)) on rows
+ * c+b..n-1 (the layout trid_sbr_dbbr leaves).  The definition, one reflector at a time: Q1 C applies H_{n-b-2}
+ * first, Q1^T C applies H_0 first.  (The paper's Alg. 3 merges the W blocks into wider ones; that regrouping is
+ * the method, this is the result it must reach.)  C is n x ncols, column-major, ld ldc. */
+void oracle_sbr_backtransform(int64_t n, int64_t b, const double* A, int64_t lda, const double* tau1, int trans,
+                              int64_t ncols, double* C, int64_t ldc) {
+  if (n <= 0 || ncols <= 0) return;
+  double* v = zalloc((size_t)n);
+  const int64_t last = n - b - 2;
+  for (int64_t q = 0; q <= last; ++q) {
+    const int64_t c = trans ? q : last - q;
+    const double tau = tau1[c];
+    if (tau == 0.0) continue;
+    const int64_t o = c + b, L = n - o;
+    v[0] = 1.0;
+    for (int64_t r = 1; r < L; ++r) v[r] = AT(A, o + r, c, lda);
+    for (int64_t j = 0; j < ncols; ++j) {
+      double s = 0.0;
+      for (int64_t r = 0; r < L; ++r) s += v[r] * AT(C, o + r, j, ldc);
+      s *= tau;
+      for (int64_t r = 0; r < L; ++r) AT(C, o + r, j, ldc) -= s * v[r];
+    }
+  }
+  free(v);
+}
+
+/* BC back-transformation: C <- Q2 C (trans = 0) or Q2^T C (trans = 1),
+ * Q2 = prod over sweeps s (ascending) and steps m (ascending) of H_{s,m} = I - tau2 v v^T (the R7 layout of
+ * trid_bulge_chase: v at V2[(S(s)+m)*b], rows s+1+m*b .. min(s+(m+1)*b, n-1)).  The definition, one
+ * reflector at a time: Q2 C applies the last reflector first. */
+void oracle_bc_backtransform(int64_t n, int64_t b, const double* V2, const double* tau2, int trans, int64_t ncols,
+                             double* C, int64_t ldc) {
+  if (n < 3 || b < 2 || ncols <= 0) return;
+  const int64_t tot = oracle_bc_total_steps(n, b);
+  int64_t* sw = (int64_t*)calloc((size_t)tot, sizeof(int64_t));
+  int64_t* st = (int64_t*)calloc((size_t)tot, sizeof(int64_t));
+  if (!sw || !st) abort();
+  int64_t off = 0;
+  for (int64_t s = 0; s + 3 <= n; ++s)
+    for (int64_t m = 0; m < oracle_bc_steps(n, b, s); ++m, ++off) { sw[off] = s; st[off] = m; }
+  for (int64_t q = 0; q < tot; ++q) {
+    const int64_t i = trans ? q : tot - 1 - q;
+    const double tau = tau2[i];
+    if (tau == 0.0) continue;
+    const int64_t r0 = sw[i] + 1 + st[i] * b;
+    int64_t r1 = sw[i] + (st[i] + 1) * b; if (r1 > n - 1) r1 = n - 1;
+    const int64_t L = r1 - r0 + 1;
+    const double* v = &V2[i * b];
+    for (int64_t j = 0; j < ncols; ++j) {
+      double s = 0.0;
+      for (int64_t r = 0; r < L; ++r) s += v[r] * AT(C, r0 + r, j, ldc);
+      s *= tau;
+      for (int64_t r = 0; r < L; ++r) AT(C, r0 + r, j, ldc) -= s * v[r];
+    }
+  }
+  free(sw); free(st);
+}
+
 /* Sturm count: number of eigenvalues < x (LAPACK dlaebz-style pivot guard). */
 int64_t oracle_sturm_count(int64_t n, const double* d, const double* e, double x, double pivmin) {
   int64_t cnt = 0;

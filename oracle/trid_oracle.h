@@ -81,6 +81,15 @@ void oracle_bc_r7(int64_t n, int64_t b, const double* A, int64_t lda, double* d,
 void oracle_form_q(int64_t n, int64_t b, const double* A_sbr, int64_t lda, const double* tau1,
                    const double* V2, const double* tau2, double* Q, int64_t ldq);
 
+/* SBR back-transformation (sec. 4.3): C <- Q1 C (trans 0) or Q1^T C (trans 1), one reflector at
+ * a time (the definition the paper's Alg. 3 regroups).  C n x ncols. */
+void oracle_sbr_backtransform(int64_t n, int64_t b, const double* A, int64_t lda, const double* tau1, int trans,
+                              int64_t ncols, double* C, int64_t ldc);
+
+/* BC back-transformation: C <- Q2 C (trans 0) or Q2^T C (trans 1), one reflector at a time. */
+void oracle_bc_backtransform(int64_t n, int64_t b, const double* V2, const double* tau2, int trans, int64_t ncols,
+                             double* C, int64_t ldc);
+
 /* Eigenvalues of the symmetric tridiagonal T = tridiag(e, d, e) by Sturm-sequence bisection
  * (gate G3), ascending into w[n]. */
 void oracle_sturm_eig(int64_t n, const double* d, const double* e, double* w);

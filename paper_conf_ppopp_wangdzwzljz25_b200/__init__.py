@@ -61,6 +61,13 @@ def lib():
         L.trid_zy_bufsize.argtypes = [_I64, _INT, ctypes.POINTER(_SZ)]
         L.trid_zy.argtypes = [_I64, _INT, _P, _I64, _P, _I64, _P, _I64, _P, _I64, _P, _SZ, _P]
         L.trid_bulge_chase_band.argtypes = [_I64, _INT, _P, _I64, _P, _P, _P, _P, _P, _SZ, _P]
+        L.trid_sbr_backtransform_bufsize.argtypes = [_I64, _INT, _INT, _I64, ctypes.POINTER(_SZ)]
+        L.trid_sbr_backtransform.argtypes = [_I64, _INT, _INT, _P, _I64, _P, _INT, _I64, _P, _I64, _P, _SZ, _P]
+        L.trid_bc_backtransform.argtypes = [_I64, _INT, _P, _P, _INT, _I64, _P, _I64, _P]
+        L.trid_stebz_bufsize.argtypes = [_I64, ctypes.POINTER(_SZ)]
+        L.trid_stebz.argtypes = [_I64, _P, _P, _P, _P, _SZ, _P]
+        L.trid_syevals_2stage_bufsize.argtypes = [_I64, _INT, _INT, _INT, ctypes.POINTER(_SZ)]
+        L.trid_syevals_2stage.argtypes = [_I64, _P, _I64, _INT, _INT, _INT, _P, _P, _SZ, _P]
         L.trid_comm_unique_id.argtypes = [ctypes.c_char_p]
         L.trid_comm_init_nccl.argtypes = [ctypes.c_char_p, _INT, _INT, ctypes.POINTER(_P)]
         L.trid_comm_init_local.argtypes = [_INT, ctypes.POINTER(_P)]
@@ -80,7 +87,9 @@ def lib():
         L.trid_profile_end.restype = _INT
         L.trid_profile_end.argtypes = [_P, _P, _INT]
         L.trid_kernel_launches.restype = _I64
-        for name in ("trid_sbr_dbbr_bufsize", "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize",
+        for name in ("trid_sbr_backtransform_bufsize", "trid_sbr_backtransform", "trid_bc_backtransform",
+                     "trid_stebz_bufsize", "trid_stebz", "trid_syevals_2stage_bufsize", "trid_syevals_2stage",
+                     "trid_sbr_dbbr_bufsize", "trid_bulge_chase_bufsize", "trid_sytrd_2stage_bufsize",
                      "trid_sbr_dbbr", "trid_bulge_chase", "trid_sytrd_2stage", "trid_panel_qr_bufsize",
                      "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize", "trid_zy"):
             getattr(L, name).restype = _INT
@@ -93,9 +102,13 @@ EXPORTS = ("trid_status_string", "trid_last_error_string", "trid_version", "trid
            "trid_sytrd_2stage", "trid_panel_qr_bufsize", "trid_panel_qr", "trid_syr2k_lower", "trid_zy_bufsize",
            "trid_zy", "trid_profile_begin", "trid_profile_end", "trid_kernel_launches", "trid_bulge_chase_band",
            "trid_comm_unique_id", "trid_comm_init_nccl", "trid_comm_init_local", "trid_comm_destroy", "trid_comm_size",
-           "trid_comm_rank", "trid_mg_local_cols", "trid_sbr_dbbr_mg_bufsize", "trid_sbr_dbbr_mg", "trid_band_gather")
+           "trid_comm_rank", "trid_mg_local_cols", "trid_sbr_dbbr_mg_bufsize", "trid_sbr_dbbr_mg", "trid_band_gather",
+           "trid_stebz_bufsize", "trid_stebz", "trid_syevals_2stage_bufsize", "trid_syevals_2stage",
+           "trid_sbr_backtransform_bufsize", "trid_sbr_backtransform", "trid_bc_backtransform")
 
-PROF_CLASSES = ("panel_qr", "wy", "symm", "zy", "next_panel", "syr2k", "bulge_chase")
+PROF_CLASSES = ("panel_qr", "wy", "symm", "zy", "next_panel", "syr2k", "bulge_chase", "stebz", "sbr_backtransform",
+                "bc_backtransform")
+SBR_CLASSES = ("panel_qr", "wy", "symm", "zy", "next_panel", "syr2k")
 
 
 def profile_begin():
@@ -293,6 +306,57 @@ def bulge_chase_band(AB: torch.Tensor, n: int, b: int, want_vectors: bool = True
                                        tau2.data_ptr() if tau2 is not None else None,
                                        work.data_ptr(), work.numel(), _stream()), "trid_bulge_chase_band")
     return d[:n], e[: max(n - 1, 0)], (V2[:v2len] if V2 is not None else None), (tau2[:t2len] if tau2 is not None else None)
+
+
+# ------------------------------------------------------------------ back-transformations
+def sbr_backtransform(S: torch.Tensor, tau1: torch.Tensor, b: int, C: torch.Tensor, trans: bool = False, k: int = 0,
+                      work=None):
+    """C <- Q1 C (or Q1^T C) in place.  S: the storage tensor of A after stage 1 (its lower part holds the SBR
+    vectors); C: storage tensor of the column-major n x ncols matrix (shape (ncols, n))."""
+    n = S.shape[0]
+    ncols = C.shape[0]
+    out = _SZ()
+    _check(lib().trid_sbr_backtransform_bufsize(n, b, k, ncols, ctypes.byref(out)), "trid_sbr_backtransform_bufsize")
+    work = work if work is not None else _workspace(out.value, C.device)
+    _check(lib().trid_sbr_backtransform(n, b, k, _dev(S, "A"), _ld(S, n), _dev(tau1, "tau1"), 1 if trans else 0,
+                                        ncols, _dev(C, "C"), _ld(C, n), work.data_ptr(), work.numel(), _stream()),
+           "trid_sbr_backtransform")
+    return C
+
+
+def bc_backtransform(V2, tau2, n: int, b: int, C: torch.Tensor, trans: bool = False):
+    """C <- Q2 C (or Q2^T C) in place; C storage tensor of shape (ncols, n)."""
+    ncols = C.shape[0]
+    _check(lib().trid_bc_backtransform(n, b, V2.data_ptr() if V2 is not None else None,
+                                       tau2.data_ptr() if tau2 is not None else None, 1 if trans else 0, ncols,
+                                       _dev(C, "C"), _ld(C, n), _stream()), "trid_bc_backtransform")
+    return C
+
+
+# ------------------------------------------------------------------ eigenvalues (SURVEY 8(f) row 3)
+def stebz(d: torch.Tensor, e: torch.Tensor, w=None, work=None):
+    """Eigenvalues of tridiag(e, d, e), ascending (Sturm bisection on the GPU)."""
+    n = d.numel()
+    out = _SZ()
+    _check(lib().trid_stebz_bufsize(n, ctypes.byref(out)), "trid_stebz_bufsize")
+    w = w if w is not None else torch.empty(max(n, 1), dtype=torch.float64, device=d.device)
+    work = work if work is not None else _workspace(out.value, d.device)
+    _check(lib().trid_stebz(n, _dev(d, "d"), _dev(e, "e") if e.numel() else None, _dev(w, "w"), work.data_ptr(),
+                            work.numel(), _stream()), "trid_stebz")
+    return w[:n]
+
+
+def syevals_2stage(A: torch.Tensor, b: int, nb: int | None = None, k: int = 0, w=None, work=None):
+    """Eigenvalues of the symmetric A (overwritten) by DBBR + eigenvalues-only BC + Sturm bisection."""
+    n = A.shape[0]
+    nb = nb or b
+    out = _SZ()
+    _check(lib().trid_syevals_2stage_bufsize(n, b, nb, k, ctypes.byref(out)), "trid_syevals_2stage_bufsize")
+    w = w if w is not None else torch.empty(max(n, 1), dtype=torch.float64, device=A.device)
+    work = work if work is not None else _workspace(out.value, A.device)
+    _check(lib().trid_syevals_2stage(n, _dev(A, "A"), _ld(A, n), b, nb, k, _dev(w, "w"), work.data_ptr(),
+                                     work.numel(), _stream()), "trid_syevals_2stage")
+    return w[:n]
 
 
 # ------------------------------------------------------------------ multi-GPU stage 1 (DESIGN.md sec. 8)

@@ -24,6 +24,8 @@
 #include "panel.cuh"
 #include "prof.cuh"
 #include "driver.cuh"
+#include "eig.cuh"
+#include "backtrans.cuh"
 
 using namespace trid;
 
@@ -448,6 +450,131 @@ int trid_sytrd_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, d
   r = trid_sbr_dbbr(n, A, lda, b, nb, k, tau1, dwork, dwork_bytes, stream);
   if (r) return r;
   return trid_bulge_chase(n, b, A, lda, d, e, V2, tau2, dwork, dwork_bytes, stream);
+}
+
+int trid_stebz_bufsize(int64_t n, size_t* dwork_bytes) {
+  if (n < 0) return -1;
+  if (!dwork_bytes) return -2;
+  *dwork_bytes = stebz_work_bytes(n > 0 ? n : 1);
+  return TRID_SUCCESS;
+}
+
+int trid_stebz(int64_t n, const double* d, const double* e, double* w, void* dwork, size_t dwork_bytes,
+               cudaStream_t stream) {
+  if (n < 0) return -1;
+  if (n > 0 && !d) return -2;
+  if (n > 1 && !e) return -3;
+  if (n > 0 && !w) return -4;
+  if (n == 0) return TRID_SUCCESS;
+  if (!dwork) return -5;
+  if (dwork_bytes < stebz_work_bytes(n)) return TRID_ERR_WORKSPACE;
+  TRID_CUDA_TRY(stebz(n, d, e, w, dwork, stream));
+  return TRID_SUCCESS;
+}
+
+namespace {
+struct EigWork {
+  double *d, *e, *tau1;
+  void* inner;
+  size_t inner_bytes, bytes;
+};
+EigWork carve_eig(void* base, int64_t n, size_t inner) {
+  EigWork w;
+  Carver c(base);
+  w.d = c.take<double>((size_t)(n > 0 ? n : 1));
+  w.e = c.take<double>((size_t)(n > 1 ? n - 1 : 1));
+  w.tau1 = c.take<double>((size_t)(n > 0 ? n : 1));
+  w.inner = c.take<char>(inner);
+  w.inner_bytes = inner;
+  w.bytes = c.off;
+  return w;
+}
+}  // namespace
+
+int trid_syevals_2stage_bufsize(int64_t n, int b, int nb, int k, size_t* dwork_bytes) {
+  if (!dwork_bytes) return -5;
+  size_t a = 0;
+  int r = trid_sytrd_2stage_bufsize(n, b, nb, k, &a, nullptr, nullptr);
+  if (r) return r;
+  const size_t s = stebz_work_bytes(n > 0 ? n : 1);
+  *dwork_bytes = carve_eig(nullptr, n, a > s ? a : s).bytes;
+  return TRID_SUCCESS;
+}
+
+int trid_syevals_2stage(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* w, void* dwork,
+                        size_t dwork_bytes, cudaStream_t stream) {
+  int r = check_common(n, A, lda, b);
+  if (r) return r;
+  if (nb < 1 || nb > b || b % nb) return -5;
+  if (k != 0 && (k < b || k % b)) return -6;
+  if (n > 0 && !w) return -7;
+  size_t need = 0;
+  r = trid_syevals_2stage_bufsize(n, b, nb, k, &need);
+  if (r) return r;
+  if (n == 0) return TRID_SUCCESS;
+  if (!dwork) return -8;
+  if (dwork_bytes < need) return TRID_ERR_WORKSPACE;
+  size_t a = 0;
+  trid_sytrd_2stage_bufsize(n, b, nb, k, &a, nullptr, nullptr);
+  const size_t s = stebz_work_bytes(n);
+  EigWork ew = carve_eig(dwork, n, a > s ? a : s);
+  r = trid_sytrd_2stage(n, A, lda, b, nb, k, ew.d, ew.e, ew.tau1, nullptr, nullptr, ew.inner, ew.inner_bytes, stream);
+  if (r) return r;
+  {
+    ProfScope ps(PROF_EIG, stream);
+    TRID_CUDA_TRY(stebz(n, ew.d, ew.e, w, ew.inner, stream));
+  }
+  return TRID_SUCCESS;
+}
+
+int trid_sbr_backtransform_bufsize(int64_t n, int b, int k, int64_t ncols, size_t* dwork_bytes) {
+  if (n < 0) return -1;
+  if (b < 1) return -2;
+  if (k != 0 && (k < b || k % b)) return -3;
+  if (ncols < 0) return -4;
+  if (!dwork_bytes) return -5;
+  if (k == 0) k = sbr_bt_default_k(b);
+  *dwork_bytes = sbr_backtransform_work_bytes(n > 0 ? n : 1, b, k, ncols);
+  return TRID_SUCCESS;
+}
+
+int trid_sbr_backtransform(int64_t n, int b, int k, const double* A, int64_t lda, const double* tau1, int trans,
+                           int64_t ncols, double* C, int64_t ldc, void* dwork, size_t dwork_bytes, cudaStream_t stream) {
+  if (n < 0) return -1;
+  if (b < 1) return -2;
+  if (k != 0 && (k < b || k % b)) return -3;
+  if (n > 0 && !A) return -4;
+  if (lda < (n > 1 ? n : 1)) return -5;
+  if (n > 0 && !tau1) return -6;
+  if (trans != 0 && trans != 1) return -7;
+  if (ncols < 0) return -8;
+  if (n > 0 && ncols > 0 && !C) return -9;
+  if (ldc < (n > 1 ? n : 1)) return -10;
+  if (k == 0) k = sbr_bt_default_k(b);
+  if (n == 0 || ncols == 0) return TRID_SUCCESS;
+  if (!dwork) return -11;
+  if (dwork_bytes < sbr_backtransform_work_bytes(n, b, k, ncols)) return TRID_ERR_WORKSPACE;
+  ProfScope ps(PROF_SBR_BT, stream);
+  TRID_CUDA_TRY(sbr_backtransform(n, b, k, A, lda, tau1, trans, ncols, C, ldc, dwork, stream));
+  return TRID_SUCCESS;
+}
+
+int trid_bc_backtransform(int64_t n, int b, const double* V2, const double* tau2, int trans, int64_t ncols, double* C,
+                          int64_t ldc, cudaStream_t stream) {
+  if (n < 0) return -1;
+  if (b < 1) return -2;
+  const bool has = n >= 3 && b >= 2;   // otherwise the chase stored no reflector (Q2 = I)
+  if (has && !V2) return -3;
+  if (has && !tau2) return -4;
+  if (trans != 0 && trans != 1) return -5;
+  if (ncols < 0) return -6;
+  if (n > 0 && ncols > 0 && !C) return -7;
+  if (ldc < (n > 1 ? n : 1)) return -8;
+  if (b > TRID_MAX_B) return TRID_ERR_UNSUPPORTED;
+  if (!has || ncols == 0) return TRID_SUCCESS;
+  ProfScope ps(PROF_BC_BT, stream);
+  TRID_CUDA_TRY(bc_backtransform(n, b, V2, tau2, trans, ncols, C, ldc, stream));
+  return TRID_SUCCESS;
 }
 
 int trid_panel_qr_bufsize(int64_t m, int w, size_t* dwork_bytes) {

@@ -6,6 +6,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <stdlib.h>
+
 #include <atomic>
 
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ != 1000)
@@ -35,6 +37,14 @@ inline int num_sms() {
     cache[d].store(v, std::memory_order_relaxed);
   }
   return v;
+}
+// True when a CUDA profiler/injection tool (Nsight Compute) is attached: such tools may refuse cooperative
+// cluster launches, so the grid-barrier kernels then launch without the cooperative attribute (their grids are
+// sized to co-resident clusters and the profiler serialises kernels, so every CTA is resident anyway).
+inline bool profiler_attached() {
+  static const bool on = getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE") != nullptr ||
+                         getenv("NV_NSIGHT_INJECTION_PORT_BASE") != nullptr || getenv("TRID_PANEL_NOCOOP") != nullptr;
+  return on;
 }
 // Idempotent per-device setup (e.g. cudaFuncSetAttribute): runs f() until it succeeds once on this device.
 struct DeviceOnce {

@@ -1,0 +1,161 @@
+// eig.cu — eigenvalues of the symmetric tridiagonal T = tridiag(e, d, e) on the GPU by Sturm-sequence
+// bisection (the eigenvalues-only EVD of P:446-448 without MAGMA; the gate G3 of
+// north_star uses the same definition).
+//
+// Method (plain definition, as LAPACK dstebz/dlaebz): the number of eigenvalues of T below x equals the
+// number of negative pivots q_i of the LDL^T factorisation of T - x I,
+//     q_0 = d_0 - x,   q_i = d_i - x - e_{i-1}^2 / q_{i-1},
+// with |q| < pivmin replaced by -pivmin (pivmin = DBL_MIN * max(1, max e^2)).  Eigenvalue k (ascending) is the
+// limit of bisection on [gl, gu] (Gershgorin bounds widened by 2 eps |.| + 2 pivmin) keeping count(lo) <= k <
+// count(hi), stopped when hi - lo <= 2 eps max(|lo|, |hi|) + pivmin.
+//
+// B200 design: the count is a sequential recurrence with one IEEE division per element, so the kernel is
+// latency-bound per eigenvalue and throughput-bound over all of them: ONE thread per eigenvalue, every thread
+// of a CTA walks the same d_i / e_i^2 in lockstep out of a shared-memory tile (one global read per element per
+// CTA instead of per thread), 128 threads per CTA so n = 32768 fills 256 CTAs (1.7 per SM).  The bounds come
+// from one small reduction kernel (min/max are exact, so the order does not matter).  Every operation is the
+// plain expression above in the same order with IEEE division (no FMA can contract it): the results equal a
+// serial implementation of the same definition bit for bit.
+#include "common.cuh"
+#include "eig.cuh"
+#include "prof.cuh"
+
+#include <float.h>
+
+namespace trid {
+
+constexpr int EIG_NT = 128;    // threads (eigenvalues) per CTA of the bisection kernel
+constexpr int EIG_TILE = 1024; // d / e^2 elements staged per shared-memory tile
+
+// bounds[0] = gl, bounds[1] = gu, bounds[2] = pivmin (widened as in the header comment); one CTA.
+__global__ void __launch_bounds__(1024) sturm_bounds_kernel(int64_t n, const double* d, const double* e,
+                                                            double* bounds) {
+  __shared__ double s_lo[32], s_hi[32], s_e2[32];
+  double lo = d[0], hi = d[0], em = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const double r = (i > 0 ? fabs(e[i - 1]) : 0.0) + (i + 1 < n ? fabs(e[i]) : 0.0);
+    lo = fmin(lo, d[i] - r);
+    hi = fmax(hi, d[i] + r);
+    if (i + 1 < n) em = fmax(em, e[i] * e[i]);
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    lo = fmin(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+    hi = fmax(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+    em = fmax(em, __shfl_xor_sync(0xffffffffu, em, o));
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) {
+    s_lo[w] = lo;
+    s_hi[w] = hi;
+    s_e2[w] = em;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const int nw = (blockDim.x + 31) / 32;
+    for (int q = 1; q < nw; ++q) {
+      lo = fmin(lo, s_lo[q]);
+      hi = fmax(hi, s_hi[q]);
+      em = fmax(em, s_e2[q]);
+    }
+    lo = fmin(lo, s_lo[0]);
+    hi = fmax(hi, s_hi[0]);
+    em = fmax(em, s_e2[0]);
+    const double pivmin = DBL_MIN * (em > 1.0 ? em : 1.0);
+    const double scale = fabs(lo) > fabs(hi) ? fabs(lo) : fabs(hi);
+    bounds[0] = lo - (2.0 * DBL_EPSILON * scale + 2.0 * pivmin + 1e-300);
+    bounds[1] = hi + (2.0 * DBL_EPSILON * scale + 2.0 * pivmin + 1e-300);
+    bounds[2] = pivmin;
+  }
+}
+
+// e2[i] = e[i]^2 (exact product, computed once instead of once per bisection step)
+__global__ void square_kernel(int64_t n1, const double* e, double* e2) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1; i += (int64_t)gridDim.x * blockDim.x)
+    e2[i] = e[i] * e[i];
+}
+
+// One thread per eigenvalue index k = blockIdx.x * EIG_NT + threadIdx.x.  All threads of the CTA run the same
+// number of bisection steps (a thread whose interval converged keeps its result and idles through the count),
+// so the CTA walks the shared tiles together.
+__global__ void __launch_bounds__(EIG_NT) sturm_bisect_kernel(int64_t n, const double* __restrict__ d,
+                                                              const double* __restrict__ e2,
+                                                              const double* __restrict__ bounds, double* w) {
+  __shared__ double sd[EIG_TILE], se[EIG_TILE];
+  __shared__ int s_active;
+  const int64_t k = (int64_t)blockIdx.x * EIG_NT + threadIdx.x;
+  const double pivmin = bounds[2];
+  double lo = bounds[0], hi = bounds[1];
+  bool active = k < n;
+  for (int it = 0; it < 256; ++it) {
+    double mid = 0.0;
+    if (active) {
+      const double tol = 2.0 * DBL_EPSILON * (fabs(lo) > fabs(hi) ? fabs(lo) : fabs(hi)) + pivmin;
+      if (hi - lo <= tol) {
+        active = false;
+      } else {
+        mid = 0.5 * (lo + hi);
+        if (mid <= lo || mid >= hi) active = false;
+      }
+    }
+    if (threadIdx.x == 0) s_active = 0;
+    __syncthreads();
+    if (active) s_active = 1;
+    __syncthreads();
+    if (!s_active) break;
+    // Sturm count of T - mid I
+    int64_t cnt = 0;
+    double q = 1.0;
+    for (int64_t t0 = 0; t0 < n; t0 += EIG_TILE) {
+      const int len = (int)((n - t0) < EIG_TILE ? (n - t0) : EIG_TILE);
+      __syncthreads();
+      for (int i = threadIdx.x; i < len; i += EIG_NT) {
+        sd[i] = d[t0 + i];
+        se[i] = (t0 + i > 0) ? e2[t0 + i - 1] : 0.0;
+      }
+      __syncthreads();
+      if (active) {
+        int i = 0;
+        if (t0 == 0) {
+          q = sd[0] - mid;
+          if (fabs(q) < pivmin) q = -pivmin;
+          if (q < 0) ++cnt;
+          i = 1;
+        }
+        for (; i < len; ++i) {
+          q = sd[i] - mid - se[i] / q;
+          if (fabs(q) < pivmin) q = -pivmin;
+          if (q < 0) ++cnt;
+        }
+      }
+    }
+    if (active) {
+      if (cnt > k) hi = mid;
+      else lo = mid;
+    }
+  }
+  if (k < n) w[k] = 0.5 * (lo + hi);
+}
+
+size_t stebz_work_bytes(int64_t n) {
+  return ((sizeof(double) * (size_t)(n > 1 ? n - 1 : 1) + 255) / 256) * 256 + 256;
+}
+
+cudaError_t stebz(int64_t n, const double* d, const double* e, double* w, void* work, cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  double* e2 = (double*)work;
+  double* bounds = (double*)((char*)work + ((sizeof(double) * (size_t)(n > 1 ? n - 1 : 1) + 255) / 256) * 256);
+  if (n > 1) {
+    int blocks = (int)((n - 1 + 255) / 256);
+    if (blocks > 4 * num_sms()) blocks = 4 * num_sms();
+    square_kernel<<<blocks, 256, 0, st>>>(n - 1, e, e2);
+    count_launches(1);
+  }
+  sturm_bounds_kernel<<<1, 1024, 0, st>>>(n, d, e, bounds);
+  count_launches(1);
+  const int64_t grid = (n + EIG_NT - 1) / EIG_NT;
+  sturm_bisect_kernel<<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w);
+  count_launches(1);
+  return cudaGetLastError();
+}
+
+}  // namespace trid

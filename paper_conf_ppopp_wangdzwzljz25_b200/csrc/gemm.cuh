@@ -61,8 +61,9 @@ cudaError_t gemm(GemmArgs a, int opA, int opB, int tile, cudaStream_t st);
 // Choose a split count so the grid fills the machine for a tall reduction (K >> M, N).
 int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elems);
 
-// Warp-specialized persistent engine (gemm_ws.cu): op(A) = A only; tiles 128x128 (N > 64) / 128x64.
+// Warp-specialized persistent engine (gemm_ws.cu): tiles 128x128 (N > 64) / 128x64.  gemm_ws: op(A) = A.
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
+cudaError_t gemm_ws_op(GemmArgs a, int opA, int opB, cudaStream_t st);
 int64_t symm_ws_splits(int64_t m, int64_t w);
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K);
 int64_t symm_ws_part_elems(int64_t m, int64_t w);

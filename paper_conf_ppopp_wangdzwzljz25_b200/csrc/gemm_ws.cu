@@ -49,6 +49,7 @@ struct Seg {
 
 struct WsArgs {
   int64_t M, N;
+  int opa;                  // GEMM segments: OP_N (A is M x K) / OP_T (A is K x M)
   int opb;                  // OP_N / OP_T for every segment
   int nseg;                 // GEMM: 1 or 2 segments over the split's K range
   const double* A[2];
@@ -176,8 +177,8 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
     kb1 = b0 * BK;
     ke1 = (e * BK < a.K[1]) ? e * BK : a.K[1];
   }
-  const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, OP_N, 0, 0, 0};
-  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, OP_N, 0, 0, 0};
+  const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, a.opa, 0, 0, 0};
+  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, a.opa, 0, 0, 0};
   if (ke0 > kb0) {
     s0 = g0;
     s1 = g1;
@@ -501,12 +502,14 @@ static bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 
 }  // namespace ws
 
-// C = alpha * sum_seg A_seg op(B_seg) + beta * Cin with op(A) = A (m-inner); tile 128x128 (wide N) or
-// 128x64 (N <= 64).  Same semantics as gemm() for opA == OP_N.
-cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
+// C = alpha * sum_seg op(A_seg) op(B_seg) + beta * Cin; tile 128x128 (wide N) or 128x64 (N <= 64).  Same
+// semantics as gemm().
+cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) { return gemm_ws_op(g, OP_N, opB, st); }
+
+cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   if (g.M <= 0 || g.N <= 0) return cudaSuccess;
   ws::WsArgs a{};
-  a.M = g.M; a.N = g.N; a.opb = opB; a.nseg = g.nseg;
+  a.M = g.M; a.N = g.N; a.opa = opA; a.opb = opB; a.nseg = g.nseg;
   bool v16 = true;
   for (int i = 0; i < 2; ++i) {
     a.A[i] = g.A[i]; a.B[i] = g.B[i]; a.lda[i] = g.lda[i]; a.ldb[i] = g.ldb[i]; a.K[i] = g.K[i];
@@ -521,7 +524,7 @@ cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) {
   if (a.mg_g > 1 && (a.tri || (a.lower && a.splits > 1) || a.mg_cb < 1)) return cudaErrorInvalidValue;
   a.part = g.part; a.part_ld = g.part_ld; a.part_stride = g.part_stride;
   if (a.mg_g > 1) {   // multi-GPU column map (only the lower-masked syr2k of mg.cu uses it)
-    if (opB != OP_T) return cudaErrorInvalidValue;
+    if (opB != OP_T || opA != OP_N) return cudaErrorInvalidValue;
     return g.N <= 64 ? ws::launch<128, 64, 4, 2, OP_T, true>(a, st) : ws::launch<128, 128, 4, 2, OP_T, true>(a, st);
   }
   if (g.N <= 64) {

@@ -372,11 +372,11 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   attr[1].id = cudaLaunchAttributeCooperative;
   attr[1].val.cooperative = 1;
   cfg.attrs = attr;
-  // The cooperative attribute guarantees co-residency for the grid barrier.  Profilers may refuse a cooperative
-  // cluster launch (plain ncu does); then, and with TRID_PANEL_NOCOOP=1, the grid is launched without it: it fits
-  // in one wave (G <= 4 x co-resident clusters), so on an otherwise idle GPU every CTA is resident anyway.
-  static const bool nocoop = getenv("TRID_PANEL_NOCOOP") != nullptr;
-  cfg.numAttrs = nocoop ? 1 : 2;
+  // The cooperative attribute guarantees co-residency for the grid barrier.  Nsight Compute aborts the
+  // application on a cooperative cluster launch; under it (and with TRID_PANEL_NOCOOP=1) the grid is launched
+  // without the attribute: it fits in one wave (G <= 4 x co-resident clusters) and the profiler serialises
+  // kernels, so every CTA is resident anyway.  A refused cooperative launch is retried the same way.
+  cfg.numAttrs = profiler_attached() ? 1 : 2;
   count_launches(1);
   auto launch = [&]() -> cudaError_t {
     switch (w) {

@@ -14,7 +14,10 @@ enum ProfClass {
   PROF_NEXT = 4,    // a4 next-panel update
   PROF_SYR2K = 5,   // a5 deferred syr2k
   PROF_BC = 6,      // a6+a7 band pack, bulge chase, d/e extraction
-  PROF_NCLASS = 7
+  PROF_EIG = 7,     // f3 Sturm bisection of T
+  PROF_SBR_BT = 8,  // f1 SBR back-transformation (C <- Q1 C)
+  PROF_BC_BT = 9,   // f2 BC back-transformation (C <- Q2 C)
+  PROF_NCLASS = 10
 };
 
 void prof_mark(int cls, bool begin, cudaStream_t st);

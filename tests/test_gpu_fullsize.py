@@ -61,10 +61,17 @@ def test_fullsize_gates(n, b, nb, k, kind, seed, dev):
 def test_timed_input_gates(dev):
     """The exact input bench.py times (configs[2]: n = 32768 random symmetric, seed 3001, b = 64, nb = 16,
     k = 1024) in the bench's launch configuration: G1/G2 with 16 Hutchinson probes through the returned
-    reflectors, and G3 for 64 sampled eigenvalues of T against cuSOLVER syevd (torch.linalg.eigvalsh) of A."""
+    reflectors, and G3 for 64 sampled eigenvalues of T (oracle Sturm count) and all n (trid_stebz) against MAGMA's
+    dsyevd of A (torch.linalg.eigvalsh)."""
     n, b, nb, k = 32768, 64, 16, 1024
     A = trid_gen.random_symmetric(n, 3001, device="cuda:0")
-    lam = torch.linalg.eigvalsh(A).cpu().numpy()
+    # cuSOLVER's syevd rejects n = 32768 (32-bit workspace query); MAGMA's hybrid dsyevd takes it (~90 s)
+    prev = torch.backends.cuda.preferred_linalg_library()
+    try:
+        torch.backends.cuda.preferred_linalg_library("magma")
+        lam = torch.linalg.eigvalsh(A).cpu().numpy()
+    finally:
+        torch.backends.cuda.preferred_linalg_library(prev)
     A0 = A.clone()
     d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=nb, k=k)
     torch.cuda.synchronize()
@@ -73,6 +80,9 @@ def test_timed_input_gates(dev):
     idx = np.unique(np.concatenate([[0, n - 1], rng.integers(0, n, 62)]))
     w = sampled_eigs(d.cpu().numpy(), e.cpu().numpy(), idx)
     assert np.max(np.abs(w - lam[idx])) <= 1e-12 * norm2
+    # all n eigenvalues of T by the GPU bisection (trid_stebz) against syevd
+    wall = trid.stebz(d, e).cpu().numpy()
+    assert np.max(np.abs(wall - lam)) <= 1e-12 * norm2
     g1, g2 = probe_gates(A0, A, d, e, tau1, V2, tau2, b, p=16)
     assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
 

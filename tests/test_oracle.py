@@ -330,6 +330,38 @@ def test_bc_noop_cases_bitwise():
     assert np.array_equal(d, np.arange(n)) and np.all(e == 0.0)
 
 
+# ---------------------------------------------------------------------------- back-transformations
+@pytest.mark.parametrize("n,b,k", [(96, 8, 32), (130, 16, None), (64, 4, 16)])
+def test_sbr_backtransform_pins(n, b, k):
+    """C <- Q1 C: with C = I it is Q1 as formed by right multiplication in form_q (a different loop order); Q1^T
+    undoes Q1; and Q1^T A Q1 is the band stage 1 produced (sec. 4.3)."""
+    A = rand_sym(n, 900 + n)
+    Aout, tau1 = oracle.dbbr(A, b, k) if k else oracle.sbr_naive(A, b)
+    Q1 = oracle.sbr_backtransform(Aout, tau1, b, np.eye(n))
+    assert np.max(np.abs(Q1 - oracle.form_q(n, b, Aout, tau1))) <= 1e-14 * n
+    C = np.random.default_rng(n).uniform(-1, 1, (n, 7))
+    back = oracle.sbr_backtransform(Aout, tau1, b, oracle.sbr_backtransform(Aout, tau1, b, C), trans=True)
+    assert np.max(np.abs(back - C)) <= 1e-14 * n
+    Bt = oracle.sbr_backtransform(Aout, tau1, b, oracle.sbr_backtransform(Aout, tau1, b, A, trans=True).T, trans=True)
+    assert np.max(np.abs(Bt - band_from_lower(Aout, b))) <= 64 * n * EPS * np.linalg.norm(A)
+
+
+@pytest.mark.parametrize("n,b", [(64, 8), (100, 7), (50, 2), (40, 64)])
+def test_bc_backtransform_pins(n, b):
+    """C <- Q2 C: with C = I it is form_q's Q2; Q2^T undoes Q2; Q2^T B Q2 = T (the chase's own output)."""
+    B = band_from_lower(rand_sym(n, 2 * n + b), min(b, n - 1))
+    d, e, V2, tau2 = oracle.bc_naive(B, b)
+    if b >= n - 1 or V2 is None or len(V2) == 0:
+        return
+    Q2 = oracle.bc_backtransform(V2, tau2, b, np.eye(n))
+    assert np.max(np.abs(Q2 - oracle.form_q(n, b, None, None, V2, tau2))) <= 1e-14 * n
+    C = np.random.default_rng(n).uniform(-1, 1, (n, 5))
+    back = oracle.bc_backtransform(V2, tau2, b, oracle.bc_backtransform(V2, tau2, b, C), trans=True)
+    assert np.max(np.abs(back - C)) <= 1e-14 * n
+    T = oracle.bc_backtransform(V2, tau2, b, oracle.bc_backtransform(V2, tau2, b, B, trans=True).T, trans=True)
+    assert np.max(np.abs(T - tridiag(d, e))) <= 64 * n * EPS * np.linalg.norm(B)
+
+
 # ---------------------------------------------------------------------------- the whole method (G1-G3)
 @pytest.mark.parametrize("k", [None, 32, 64, 128, 256])
 def test_two_stage_gates_n256(k):
