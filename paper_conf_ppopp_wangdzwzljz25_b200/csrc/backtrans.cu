@@ -224,9 +224,8 @@ template <int QR>
 __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int nb, const double* __restrict__ V2,
                                                         const double* __restrict__ tau2, int trans, int64_t ncols,
                                                         double* C, int64_t ldc) {
-  constexpr int RW = 8 * QR;
-  extern __shared__ __align__(16) double sv[];   // nb x (b + RW) staged reflectors (zero padded), nb taus
-  double* stau = sv + (size_t)nb * (b + RW);
+  extern __shared__ __align__(16) double sv[];   // nb x b staged reflectors (zero padded to b), nb taus
+  double* stau = sv + (size_t)nb * b;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rg = lane >> 2, cl = lane & 3;
   const int64_t col = (int64_t)blockIdx.x * BT_COLS + warp * 4 + cl;
@@ -234,7 +233,7 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   double* Cc = C + (colok ? col : 0) * ldc;
   const int64_t nsw = n - 2;   // sweeps 0 .. n-3
   const int64_t nblk = (nsw + nb - 1) / nb;
-  const int vstride = b + RW;   // staged vector j at sv + j*vstride + RW: v index i at row offset (s-s0) + i
+  const int vstride = b;   // staged vector j at sv + j*b: its entry i sits at window row j + i
   for (int64_t bi = 0; bi < nblk; ++bi) {
     const int64_t blk = trans ? bi : nblk - 1 - bi;
     const int64_t s0 = blk * nb;
@@ -246,11 +245,9 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
       // stage the group's reflectors: vector of sweep s0+j (if step m exists) and its tau
       __syncthreads();
       for (int idx = threadIdx.x; idx < nbb * vstride; idx += BT_NT) {
-        const int j = idx / vstride, i = idx - j * vstride - RW;
+        const int j = idx / vstride, i = idx - j * vstride;
         const int64_t s = s0 + j;
-        double v = 0.0;
-        if (i >= 0 && m < bt_steps(n, b, s)) v = V2[(bt_offset(n, b, s) + m) * b + i];
-        sv[idx] = v;
+        sv[idx] = m < bt_steps(n, b, s) ? V2[(bt_offset(n, b, s) + m) * b + i] : 0.0;
       }
       for (int j = threadIdx.x; j < nbb; j += BT_NT) {
         const int64_t s = s0 + j;
@@ -269,25 +266,26 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         const int j = trans ? jj : nbb - 1 - jj;
         const double tau = stau[j];
         if (tau == 0.0) continue;
-        // v entry for window row rg*QR + q is vector index (rg*QR + q) - j
-        const double* vj = sv + (size_t)j * vstride + RW - j + rg * QR;
-        double d = 0.0;
+        // v entry for window row rg*QR + q is vector index (rg*QR + q) - j (zero outside [0, b)); the shared load
+        // index is clamped so it never leaves the staged vector
+        const double* vj = sv + (size_t)j * vstride;
+        const int base = rg * QR - j;
+        double vv[QR];
 #pragma unroll
         for (int q = 0; q < QR; ++q) {
-          const int wr = rg * QR + q - j;
-          const double vq = (wr >= 0 && wr < b) ? vj[q] : 0.0;
-          d = fma(vq, x[q], d);
+          const int wr = base + q;
+          const int wc = wr < 0 ? 0 : (wr >= b ? b - 1 : wr);
+          vv[q] = (wr >= 0 && wr < b) ? vj[wc] : 0.0;
         }
+        double d = 0.0;
+#pragma unroll
+        for (int q = 0; q < QR; ++q) d = fma(vv[q], x[q], d);
         d += __shfl_xor_sync(0xffffffffu, d, 4);
         d += __shfl_xor_sync(0xffffffffu, d, 8);
         d += __shfl_xor_sync(0xffffffffu, d, 16);
         const double td = tau * d;
 #pragma unroll
-        for (int q = 0; q < QR; ++q) {
-          const int wr = rg * QR + q - j;
-          const double vq = (wr >= 0 && wr < b) ? vj[q] : 0.0;
-          x[q] = fma(-td, vq, x[q]);
-        }
+        for (int q = 0; q < QR; ++q) x[q] = fma(-td, vv[q], x[q]);
       }
 #pragma unroll
       for (int q = 0; q < QR; ++q) {
@@ -299,17 +297,20 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
 }
 
 int bc_bt_nb(int b) {
-  // window 8*QR rows >= b + nb - 1 with QR = 16 (b <= 64) or 32 (b <= 128) or 64 (b <= 256)
+  // window 8*QR rows >= b + nb - 1 with QR = 16 (b <= 64) or 32 (b <= 128) or 64 (b <= 256); the nb staged vectors
+  // (nb * b doubles) fit in 200 KB of shared memory
   const int rw = b <= 64 ? 128 : (b <= 128 ? 256 : 512);
-  return rw - b + 1 < 1 ? 1 : rw - b + 1;
+  int nb = rw - b + 1;
+  const int cap = (int)(200 * 1024 / (8 * (size_t)b)) - 1;
+  if (nb > cap) nb = cap;
+  return nb < 1 ? 1 : nb;
 }
 
 cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* tau2, int trans, int64_t ncols,
                              double* C, int64_t ldc, cudaStream_t st) {
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
-  const int rw = b <= 64 ? 128 : (b <= 128 ? 256 : 512);
-  const size_t smem = sizeof(double) * ((size_t)nb * (b + rw) + nb);
+  const size_t smem = sizeof(double) * ((size_t)nb * b + nb);
   const int64_t grid = (ncols + BT_COLS - 1) / BT_COLS;
   const void* fn = b <= 64 ? (const void*)bc_bt_kernel<16> : (b <= 128 ? (const void*)bc_bt_kernel<32>
                                                                        : (const void*)bc_bt_kernel<64>);
