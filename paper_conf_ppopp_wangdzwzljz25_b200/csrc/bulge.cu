@@ -466,7 +466,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       mbar_init(&lastb[i], 1);
       mbar_init(&empty[i], 1);
       mbar_init(&col0b[i], 2 * B);
-      mbar_init(&colsb[i], 1);
+      mbar_init(&colsb[i], (a.opt & 8) ? NW : 1);
       mbar_init(&c0done[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -651,7 +651,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
     const int64_t s = info_s[bi];
     if (s < 0) {
       if (c0path) mbar_arrive(&col0b[bi]);   // wake the STORE warps so they can see the end
-      if (tid == 0) mbar_arrive(&colsb[bi]);
+      if ((a.opt & 8) ? lane == 0 : tid == 0) mbar_arrive(&colsb[bi]);
       return;
     }
     const int64_t m = info_m[bi];
@@ -918,10 +918,20 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       for (int i = tid; i < a.vs; i += NTH) vd[i] = i < L ? v[i] : 0.0;
       if (tid == 0) a.tau2[off + m] = tau;
     }
-    cbar();   // (4) columns 1..L-1 final
-    if (tid == 0) {
-      BCW_TRACE(s, m, 2);
-      mbar_arrive(&colsb[bi]);   // -> STORE1
+    if (a.opt & 8) {
+      // per-warp hand-off (TRID_BC_OPT bit 8): each warp releases its own stores of this step to STORE1 (colsb
+      // counts the NW compute warps), so warps that finished early start the next step's body matvec while the
+      // O-row warps finish the left application; the next step's first CTA barrier still orders every shared
+      // scratch reuse
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&colsb[bi]);
+      if (tid == 0) BCW_TRACE(s, m, 2);
+    } else {
+      cbar();   // (4) columns 1..L-1 final
+      if (tid == 0) {
+        BCW_TRACE(s, m, 2);
+        mbar_arrive(&colsb[bi]);   // -> STORE1
+      }
     }
     };
     if (Lx == B && L2x == B) step(std::true_type{});
