@@ -874,7 +874,14 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
     } else if (lane < CPT) {
       zp[(warp % RW) * B + j0 + lane] = 0.0;
     }
-    cbar();   // (3) z partials, vn
+    if (FULL && RW == 4 && (a.opt & 16)) {
+      // (3') full windows: z_j of column group hg needs only the partials of its own two O-row warps (rows
+      // L..L+L2-1), so those 64 threads meet on the group's named barrier and the D-row warps go on (TRID_BC_OPT
+      // bit 16, with bit 8)
+      if (isO) asm volatile("bar.sync %0, %1;\n" ::"r"(3 + hg), "n"(2 * 32) : "memory");
+    } else {
+      cbar();   // (3) z partials, vn
+    }
     if (tid == 0) BCW_TRACE(s, m, 13);
     if (FULL && isO) {
       // full window: the O rows are the last two row-warps of the group (the others' partials are zero, and
