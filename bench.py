@@ -32,6 +32,11 @@ CONFIGS = {
                    desc="n=32768 random symmetric FP64, b=64, nb=16, k=1024 on 1xB200"),
     "n32768b128": dict(n=32768, b=128, nb=16, k=1024, seed=3001,
                        desc="n=32768 random symmetric FP64, b=128, nb=16, k=1024 on 1xB200"),
+    "n49152": dict(n=49152, b=64, nb=16, k=1024, seed=4001, kind="clusters",
+                   desc="n=49152 clustered-spectrum symmetric FP64 (32 clusters), b=64, nb=16, k=1024"),
+    **{f"n16384b{bb}": dict(n=16384, b=bb, nb=min(16, bb), k=1024, seed=5001,
+                            desc=f"n=16384 random symmetric FP64, b={bb}, nb={min(16, bb)}, k=1024 (band sweep)")
+       for bb in (32, 64, 128, 256)},
 }
 
 
@@ -342,7 +347,10 @@ def main():
     want = not args.eig_only
     stream = torch.cuda.current_stream()
     if ws == 1:
-        A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
+        if cfg.get("kind"):
+            A0, _ = trid_gen.clustered_symmetric(n, cfg["seed"], kind=cfg["kind"], device=dev)
+        else:
+            A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
         A = torch.empty_like(A0)
         nbytes, v2len, t2len = trid.sytrd_2stage_bufsize(n, b, nb, k)
         work = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)

@@ -182,7 +182,7 @@ def test_bulge_chase_cluster_forwarding_bitwise(n, b, cl, dev, monkeypatch):
         assert torch.equal(x, y)
 
 
-@pytest.mark.parametrize("env", [("TRID_BC_FS", "1"), ("TRID_BC_FS", "32"), ("TRID_BC_OPT", "1"), ("TRID_BC_OPT", "2"),
+@pytest.mark.parametrize("env", [("TRID_BC_FS", "1"), ("TRID_BC_FS", "32"), ("TRID_BC_OPT", "0"), ("TRID_BC_OPT", "1"), ("TRID_BC_OPT", "2"), ("TRID_BC_OPT", "8"), ("TRID_BC_OPT", "31"),
                                  ("TRID_BC_OPT", "4"), ("TRID_BC_OPT", "7")])
 def test_bulge_chase_handoff_options_bitwise(env, dev, monkeypatch):
     """Counter layout (TRID_BC_FS) and hand-off options (TRID_BC_OPT) change only how data and progress move
