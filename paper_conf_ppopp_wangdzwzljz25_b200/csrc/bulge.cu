@@ -24,7 +24,6 @@
 
 namespace trid {
 
-constexpr int BC_NT = 256;
 constexpr int BC_FLAG_STRIDE = 32;   // workspace room per counter (ints); bc_v6 uses 8 (one sector) unless TRID_BC_FS
 
 struct BcArgs {
@@ -97,215 +96,6 @@ __global__ void band_extract_kernel(int64_t n, int ldab, const double* band, dou
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     d[i] = band[i * ldab];
     if (i + 1 < n) e[i] = band[i * ldab + 1];
-  }
-}
-
-// ---- the chase ---------------------------------------------------------------------------------
-// Window of step (s, m): compact columns r0 .. r0+L-1 (each ldab doubles: rows c .. c+ldab-1).
-//   D = B_d  (L x L symmetric):  D(i,j) = C[j*ldab + i-j] (i >= j)
-//   O = B_od (L2 x L, the block below, where the bulge appears):  O(i,j) = C[j*ldab + L+i-j]
-template <bool SM>
-struct CWin {
-  double* C;
-  int ldab, L;
-  __device__ __forceinline__ double ld(int off) const {
-    if constexpr (SM) return C[off];
-    else return __ldcg(C + off);
-  }
-  __device__ __forceinline__ void st(int off, double v) const {
-    if constexpr (SM) C[off] = v;
-    else __stcg(C + off, v);
-  }
-  __device__ __forceinline__ int dof(int i, int j) const { return i >= j ? j * ldab + (i - j) : i * ldab + (j - i); }
-  __device__ __forceinline__ int oof(int i, int j) const { return j * ldab + L + i - j; }
-};
-
-// Window load: 16-byte cp.async (all copies of a thread in flight at once, no registers held).
-__device__ __forceinline__ void load_span(double* dst, const double* src, int count) {
-  const int n2 = count >> 1;
-  for (int i = threadIdx.x; i < n2; i += BC_NT) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst + 2 * i);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src + 2 * i) : "memory");
-  }
-  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
-}
-// Window store: 16-byte st.global.cg (fire and forget).
-__device__ __forceinline__ void store_span(double* dst, const double* src, int count) {
-  const int n2 = count >> 1;
-  const double2* s2 = reinterpret_cast<const double2*>(src);
-  double2* d2 = reinterpret_cast<double2*>(dst);
-  for (int i = threadIdx.x; i < n2; i += BC_NT) __stcg(d2 + i, s2[i]);
-}
-
-template <bool SM>
-__global__ void __launch_bounds__(BC_NT, 3) bc_kernel(BcArgs a) {
-  extern __shared__ __align__(16) double sm[];
-  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31;
-  const int64_t n = a.n;
-  double* win = sm;
-  double* vec = SM ? sm + (size_t)b * ldab : sm;
-  double* v = vec;               // b   reflector of this step
-  double* vn = v + b;            // b   reflector of the next step
-  double* p = vn + b;            // b   tau * D v
-  double* y = p + b;             // b   O v
-  double* z = y + b;             // b   vn^T O
-  double* scratch = z + b;       // 2 * BC_NT partial sums
-  __shared__ int64_t s_sweep;
-
-  for (;;) {
-    if (tid == 0) s_sweep = (int64_t)atomicAdd(a.ticket, 1u);
-    __syncthreads();
-    const int64_t s = s_sweep;
-    __syncthreads();
-    if (s > n - 3) return;
-    const int64_t nst = bc_steps(n, b, s);
-    const int64_t off = bc_offset(n, b, s);
-    const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
-    double tau = 0.0;
-    for (int64_t m = 0; m < nst; ++m) {
-      const int64_t r0 = s + 1 + m * b;
-      const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
-      const int L = (int)(r1 - r0 + 1);
-      const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
-      const int L2 = (int)(r2 - r1);
-      // ---- lag-2 dependency (R9): sweep s-1 must have completed step m+1
-      if (s > 0) {
-        if (tid == 0) {
-          const int need = (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev);
-          wait_geq(a.prog + (s - 1), need);
-        }
-        __syncthreads();
-      }
-      // ---- step 0: the reflector annihilating column s below its first subdiagonal
-      if (m == 0) {
-        double* col = a.band + s * a.ldab + 1;
-        double sig = 0.0;
-        for (int i = 1 + lane; i < L; i += 32) {
-          const double x = __ldcg(col + i);
-          sig += x * x;
-        }
-        sig = warp_sum(sig);  // every warp computes the same value in the same order
-        const House h = make_house(__ldcg(col), sig);
-        __syncthreads();      // all reads of column s done before it is overwritten
-        for (int i = tid; i < L; i += BC_NT) {
-          v[i] = i == 0 ? 1.0 : h.scale * __ldcg(col + i);
-        }
-        __syncthreads();
-        for (int i = tid; i < L; i += BC_NT) __stcg(col + i, i == 0 ? h.beta : 0.0);
-        tau = h.tau;
-      }
-      CWin<SM> W;
-      W.ldab = ldab;
-      W.L = L;
-      if constexpr (SM) {
-        W.C = win;
-        load_span(win, a.band + r0 * ldab, L * ldab);
-      } else {
-        W.C = a.band + r0 * ldab;
-      }
-      __syncthreads();
-      // ---- two-sided on B_d and right-apply to B_od (the bulge), from ONE pass of matvecs
-      if (tau != 0.0) {
-        const int R = L + L2;
-        const int q = R < BC_NT ? BC_NT / R : 1;
-        for (int task = tid; task < R * q; task += BC_NT) {
-          const int i = task % R, c = task / R;
-          double acc = 0.0;
-          if (i < L) {
-            for (int j = c; j < L; j += q) acc += W.ld(W.dof(i, j)) * v[j];
-          } else {
-            for (int j = c; j < L; j += q) acc += W.ld(W.oof(i - L, j)) * v[j];
-          }
-          scratch[c * R + i] = acc;
-        }
-        __syncthreads();
-        for (int i = tid; i < R; i += BC_NT) {
-          double acc = 0.0;
-          for (int c = 0; c < q; ++c) acc += scratch[c * R + i];
-          if (i < L) p[i] = tau * acc;
-          else y[i - L] = acc;
-        }
-        __syncthreads();
-        double pv = 0.0;  // p^T v, per warp (identical in every warp)
-        for (int i = lane; i < L; i += 32) pv += p[i] * v[i];
-        pv = warp_sum(pv);
-        const double hp = 0.5 * tau * pv;
-        // D -= v w^T + w v^T (lower), w = p - 1/2 tau (p^T v) v;   O -= tau (O v) v^T
-        const int nd = L * L, no = L2 * L;
-        for (int idx = tid; idx < nd + no; idx += BC_NT) {
-          if (idx < nd) {
-            const int i = idx % L, j = idx / L;
-            if (i >= j) {
-              const double wi = p[i] - hp * v[i], wj = p[j] - hp * v[j];
-              const int o = j * ldab + (i - j);
-              W.st(o, W.ld(o) - (v[i] * wj + wi * v[j]));
-            }
-          } else {
-            const int k = idx - nd, i = k % L2, j = k / L2;
-            const int o = W.oof(i, j);
-            W.st(o, W.ld(o) - tau * y[i] * v[j]);
-          }
-        }
-        __syncthreads();
-      }
-      // ---- next reflector from the bulge's first column; left-apply to O(:, 1:)
-      double tau_next = 0.0;
-      if (L2 > 0) {
-        double sig = 0.0;
-        for (int i = 1 + lane; i < L2; i += 32) {
-          const double x = W.ld(W.oof(i, 0));
-          sig += x * x;
-        }
-        sig = warp_sum(sig);
-        const House h = make_house(W.ld(W.oof(0, 0)), sig);
-        tau_next = h.tau;
-        if (h.tau != 0.0 && L > 1) {
-          const int C = L - 1;
-          const int q = C < BC_NT ? BC_NT / C : 1;
-          for (int task = tid; task < C * q; task += BC_NT) {
-            const int j = 1 + task % C, c = task / C;
-            double acc = 0.0;
-            for (int i = c; i < L2; i += q) {
-              const double vi = i == 0 ? 1.0 : h.scale * W.ld(W.oof(i, 0));
-              acc += vi * W.ld(W.oof(i, j));
-            }
-            scratch[c * C + (j - 1)] = acc;
-          }
-          __syncthreads();
-          for (int j = tid; j < C; j += BC_NT) {
-            double acc = 0.0;
-            for (int c = 0; c < q; ++c) acc += scratch[c * C + j];
-            z[j + 1] = acc;
-          }
-          __syncthreads();
-          for (int idx = tid; idx < L2 * C; idx += BC_NT) {
-            const int i = idx % L2, j = 1 + idx / L2;
-            const double vi = i == 0 ? 1.0 : h.scale * W.ld(W.oof(i, 0));
-            const int o = W.oof(i, j);
-            W.st(o, W.ld(o) - h.tau * vi * z[j]);
-          }
-        }
-        __syncthreads();  // every read of O(:, 0) is done
-        for (int i = tid; i < L2; i += BC_NT) {
-          const int o = W.oof(i, 0);
-          vn[i] = i == 0 ? 1.0 : h.scale * W.ld(o);
-          W.st(o, i == 0 ? h.beta : 0.0);
-        }
-      }
-      __syncthreads();
-      // ---- write back, store the reflector of this step, publish progress
-      if constexpr (SM) store_span(a.band + r0 * ldab, win, L * ldab);
-      if (a.V2) {
-        double* vd = a.V2 + (off + m) * a.vs;
-        for (int i = tid; i < a.vs; i += BC_NT) vd[i] = i < L ? v[i] : 0.0;
-        if (tid == 0) a.tau2[off + m] = tau;
-      }
-      __syncthreads();
-      if (tid == 0) st_release_s32(a.prog + s, (int)(m + 1));  // cumulative over the CTA's stores (bar.sync above)
-      for (int i = tid; i < L2; i += BC_NT) v[i] = vn[i];
-      tau = tau_next;
-      __syncthreads();
-    }
   }
 }
 
@@ -955,6 +745,248 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
   if constexpr (CL) cl_sync_all();   // no CTA leaves while a peer may still copy into / signal its shared memory
 }
 
+
+// ---- wide-band chase (64 < b <= 256) ----------------------------------------------------------------------------------
+// The b <= 64 register-resident design does not scale: at b = 128 a step window ([D; O], 2b rows x b columns) is
+// 197 KB even when only its stored part is kept, at b = 256 it is 788 KB.  Here a step's window lives in shared
+// memory as a TRAPEZOID: window column j holds only its rows j .. 2b-1 (the lower triangle of D and the whole
+// bulge block O), 2b - j doubles rounded up to even, packed one after the other (16-byte aligned columns, loaded and
+// stored with 16-byte cp.async / st.global.cg by all threads).  For b > 128 the window is split by columns over a
+// cluster of CS = 4 CTAs (balanced by stored size, <= 197 KB each) that cooperate on one sweep through DSMEM:
+//   1. every CTA forms the partial matvec [D; O] v over its columns for all 2b rows (the lower part of D row-wise,
+//      the mirrored upper part as a column dot, both from its own columns), writes it to shared memory;
+//   2. cluster barrier; every CTA sums the CS partials in rank order (DSMEM loads): identical p = tau D v, y = O v;
+//   3. rank-2 update of D and right update of O on its own columns;
+//   4. the CTA owning window column 0 forms the next reflector from O(:, 0) and broadcasts it (DSMEM stores);
+//      cluster barrier;
+//   5. z_j = vn^T O(:, j) and the left update on its own columns; store back; cluster barrier; rank 0 publishes.
+// Sweeps are claimed from the atomic ticket and pipelined at lag 2 on per-sweep counters (R9) as in bc_v6.  All sums
+// run in a fixed order: bitwise reproducible, independent of scheduling (serial-vs-parallel test).
+constexpr int BW_NT = 512;
+struct BwPart {
+  int c[5];   // window columns [c[q], c[q+1]) belong to cluster rank q
+};
+
+// offset (doubles) of window column j in the packed trapezoid, columns of 2b - j rows rounded up to even
+__host__ __device__ __forceinline__ int bw_coff(int b, int j) { return 2 * b * j - j * (j - 1) / 2 + j / 2; }
+
+template <int CS>
+__device__ __forceinline__ double* bw_peer(double* p, unsigned rank) {
+  if constexpr (CS == 1) {
+    return p;
+  } else {
+    // generic address of the same variable in the shared memory of cluster rank `rank`
+    double* r;
+    asm volatile("mapa.u64 %0, %1, %2;\n" : "=l"(r) : "l"(p), "r"(rank));
+    return r;
+  }
+}
+template <int CS>
+__device__ __forceinline__ void bw_csync() {
+  if constexpr (CS == 1) __syncthreads();
+  else cl_sync_all();
+}
+
+template <int CS>
+__global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part) {
+  extern __shared__ __align__(16) double sm[];
+  constexpr int NW = BW_NT / 32;
+  const int b = a.b, ldab = a.ldab, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t n = a.n;
+  const unsigned q = CS > 1 ? cl_rank() : 0u;
+  const int cbeg = part.c[q], cend = part.c[q + 1];
+  const int base_off = bw_coff(b, cbeg);
+  const int H2 = 2 * b;
+  // shared layout: vb[2][b] | prt[2b] | pf[2b] | w[b] | colv[b] | scal[16] | window
+  double* vb = sm;
+  double* prt = vb + 2 * b;
+  double* pf = prt + H2;
+  double* wv = pf + H2;
+  double* colv = wv + b;
+  double* scal = colv + b;   // 0 pv, 1..3 reflector of column s (beta, tau, scale), 4..6 next reflector
+  double* win = scal + 16;
+  __shared__ int64_t s_sweep;
+  auto W = [&](int i, int j) -> double& { return win[bw_coff(b, j) - base_off + (i - j)]; };   // i >= j, j mine
+  for (int64_t sweep_i = 0;; ++sweep_i) {
+    if (q == 0 && tid == 0) {
+      const int64_t s0 = (int64_t)atomicAdd(a.ticket, 1u);
+      if constexpr (CS == 1) {
+        s_sweep = s0;
+      } else {
+        for (unsigned r = 0; r < CS; ++r) *reinterpret_cast<int64_t*>(bw_peer<CS>((double*)&s_sweep, r)) = s0;
+      }
+    }
+    bw_csync<CS>();
+    const int64_t s = s_sweep;
+    bw_csync<CS>();
+    if (s > n - 3) return;
+    const int64_t nst = bc_steps(n, b, s);
+    const int64_t off = bc_offset(n, b, s);
+    const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
+    double tau = 0.0;
+    for (int64_t m = 0; m < nst; ++m) {
+      double* v = vb + (m & 1) * b;
+      double* vn = vb + ((m & 1) ^ 1) * b;
+      const int64_t r0 = s + 1 + m * b;
+      const int64_t r1 = (s + (m + 1) * b < n - 1) ? s + (m + 1) * b : n - 1;
+      const int L = (int)(r1 - r0 + 1);
+      const int64_t r2 = (r1 + b < n - 1) ? r1 + b : n - 1;
+      const int L2 = (int)(r2 - r1);
+      const int H = L + L2;
+      const int je = cend < L ? cend : L;   // my window columns [cbeg, je)
+      // ---- lag-2 dependency (R9): sweep s-1 has completed step m+1 (serial mode: all of its steps)
+      if (s > 0) {
+        if (tid == 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev));
+        __syncthreads();
+      }
+      // ---- load my window columns (rows j .. H-1 of column j: offsets 0 .. H-1-j)
+      for (int j = cbeg; j < je; ++j) {
+        const int len = H - j, len2 = len >> 1;
+        double* dst = &W(j, j);
+        const double* src = a.band + (r0 + j) * ldab;
+        for (int i = tid; i < len2; i += BW_NT) {
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(dst + 2 * i)), "l"(src + 2 * i)
+                       : "memory");
+        }
+        if ((len & 1) && tid == BW_NT - 1) dst[len - 1] = __ldcg(src + len - 1);
+      }
+      asm volatile("cp.async.commit_group;\n" ::: "memory");
+      // ---- step 0: the reflector annihilating column s below its first subdiagonal (every CTA, same bits)
+      if (m == 0) {
+        for (int i = tid; i < L; i += BW_NT) colv[i] = __ldcg(a.band + s * ldab + 1 + i);
+        __syncthreads();
+        if (warp == 0) {
+          double sg = 0.0;
+          for (int i = 1 + lane; i < L; i += 32) sg = fma(colv[i], colv[i], sg);
+          sg = warp_sum(sg);
+          if (lane == 0) {
+            const House h = make_house(colv[0], sg);
+            scal[1] = h.beta;
+            scal[2] = h.tau;
+            scal[3] = h.scale;
+            if (q == 0) __stcg(a.band + s * ldab + 1, h.beta);   // e_s (the rest of column s is dead)
+          }
+        }
+        __syncthreads();
+        for (int i = tid; i < b; i += BW_NT) v[i] = i == 0 ? 1.0 : (i < L ? scal[3] * colv[i] : 0.0);
+        tau = scal[2];
+      }
+      asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+      __syncthreads();
+      // ---- 1. partial matvec [D; O] v over my columns, all H rows
+      if (tau != 0.0) {
+        for (int i = tid; i < H2; i += BW_NT) {
+          double acc = 0.0;
+          if (i < H) {
+            const int jt = je < i + 1 ? je : i + 1;   // lower part of D (and all of O): columns j <= i
+            for (int j = cbeg; j < jt; ++j) acc = fma(W(i, j), v[j], acc);
+          }
+          prt[i] = acc;
+        }
+        __syncthreads();
+        // mirrored upper part of D for my columns c: sum_{j > c, j < L} D(j, c) v_j (a column dot, one warp)
+        for (int c = cbeg + warp; c < je; c += NW) {
+          double acc = 0.0;
+          for (int j = c + 1 + lane; j < L; j += 32) acc = fma(W(j, c), v[j], acc);
+          acc = warp_sum(acc);
+          if (lane == 0) prt[c] += acc;
+        }
+        bw_csync<CS>();   // (1) partials of every CTA complete
+        // ---- 2. p = tau D v, y = O v: the CS partials summed in rank order
+        for (int i = tid; i < H; i += BW_NT) {
+          double acc = 0.0;
+#pragma unroll
+          for (unsigned r = 0; r < CS; ++r) acc += *bw_peer<CS>(prt + i, r);
+          pf[i] = i < L ? tau * acc : acc;
+        }
+        __syncthreads();
+        if (warp == 0) {
+          double pv = 0.0;
+          for (int i = lane; i < L; i += 32) pv = fma(pf[i], v[i], pv);
+          pv = warp_sum(pv);
+          if (lane == 0) scal[0] = pv;
+        }
+        __syncthreads();
+        const double hp = 0.5 * tau * scal[0];
+        for (int i = tid; i < L; i += BW_NT) wv[i] = fma(-hp, v[i], pf[i]);
+        __syncthreads();
+        // ---- 3. D -= v w^T + w v^T (lower, my columns), O -= tau y v^T (my columns)
+        for (int j = cbeg; j < je; ++j) {
+          const double vj = v[j], wj = wv[j], tvj = tau * vj;
+          for (int i = j + tid; i < H; i += BW_NT) {
+            double& x = W(i, j);
+            if (i < L) x = fma(-wv[i], vj, fma(-v[i], wj, x));
+            else x = fma(-pf[i], tvj, x);
+          }
+        }
+      }
+      // ---- 4. the next reflector from O(:, 0) (window column 0: rank 0), broadcast
+      double taun = 0.0;
+      if (L2 > 0) {
+        __syncthreads();
+        if (q == 0) {
+          if (warp == 0) {
+            double sg = 0.0;
+            for (int i = 1 + lane; i < L2; i += 32) {
+              const double x = W(L + i, 0);
+              sg = fma(x, x, sg);
+            }
+            sg = warp_sum(sg);
+            if (lane == 0) {
+              const House h = make_house(W(L, 0), sg);
+              for (unsigned r = 0; r < CS; ++r) {
+                double* sc = bw_peer<CS>(scal, r);
+                sc[4] = h.beta;
+                sc[5] = h.tau;
+                sc[6] = h.scale;
+              }
+            }
+          }
+          __syncthreads();
+          const double hs = scal[6];
+          for (int i = tid; i < b; i += BW_NT) {
+            const double x = i < L2 ? (i == 0 ? 1.0 : hs * W(L + i, 0)) : 0.0;
+#pragma unroll
+            for (unsigned r = 0; r < CS; ++r) bw_peer<CS>(vn, r)[i] = x;
+          }
+          __syncthreads();
+          for (int i = tid; i < L2; i += BW_NT) W(L + i, 0) = i == 0 ? scal[4] : 0.0;
+        }
+        bw_csync<CS>();   // (2) vn and its scalars everywhere
+        taun = scal[5];
+        // ---- 5. O(:, j) -= taun vn (vn^T O(:, j)) for my columns j >= 1
+        if (taun != 0.0) {
+          const int j1 = cbeg > 1 ? cbeg : 1;
+          for (int c = j1 + warp; c < je; c += NW) {
+            double acc = 0.0;
+            for (int i = lane; i < L2; i += 32) acc = fma(vn[i], W(L + i, c), acc);
+            acc = warp_sum(acc);
+            const double tz = taun * acc;
+            for (int i = lane; i < L2; i += 32) W(L + i, c) = fma(-tz, vn[i], W(L + i, c));
+          }
+        }
+      }
+      __syncthreads();
+      // ---- store my columns back, the reflector of this step, publish
+      for (int j = cbeg; j < je; ++j) {
+        const int len = H - j, len2 = len >> 1;
+        const double2* srcp = reinterpret_cast<const double2*>(&W(j, j));
+        double2* dst = reinterpret_cast<double2*>(a.band + (r0 + j) * ldab);
+        for (int i = tid; i < len2; i += BW_NT) __stcg(dst + i, srcp[i]);
+        if ((len & 1) && tid == BW_NT - 1) __stcg(a.band + (r0 + j) * ldab + len - 1, W(H - 1, j));
+      }
+      if (q == 0 && a.V2) {
+        double* vd = a.V2 + (off + m) * a.vs;
+        for (int i = tid; i < a.vs; i += BW_NT) vd[i] = i < L ? v[i] : 0.0;
+        if (tid == 0) a.tau2[off + m] = tau;
+      }
+      bw_csync<CS>();   // (3) every CTA's stores of this step issued (ordered before the release below)
+      if (q == 0 && tid == 0) st_release_s32(a.prog + s, (int)(m + 1));
+      tau = taun;
+    }
+  }
+}
+
 size_t bc_work_bytes(int64_t n, int b) {
   const size_t band = sizeof(double) * (size_t)n * bc_ldab(n, b);
   const size_t flags = sizeof(int) * (size_t)(2 * n + 128) * BC_FLAG_STRIDE;
@@ -1071,22 +1103,52 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
         else bc_v6_kernel<64, 512, false><<<(unsigned)grid, 512 + 96, smem, st>>>(a);
       }
     } else {
-      const size_t vec = sizeof(double) * (size_t)(5 * beff + 2 * BC_NT + 8);
-      const size_t winb = sizeof(double) * (size_t)beff * ldab;
-      const bool use_sm = vec + winb <= 200 * 1024;
-      const size_t smem = use_sm ? vec + winb : vec;
-      if (use_sm) {
-        cudaFuncSetAttribute(bc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<true>, BC_NT, smem);
-      } else {
-        cudaFuncSetAttribute(bc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bc_kernel<false>, BC_NT, smem);
+      // 64 < b <= 256: bc_wide_kernel, one CTA per sweep (b <= 128) or a cluster of 4 (b > 128)
+      const int CS = beff <= 128 ? 1 : 4;
+      BwPart part{};
+      const int total = bw_coff(beff, beff);
+      part.c[0] = 0;
+      for (int q = 1; q < CS; ++q) {
+        int j = part.c[q - 1];
+        while (j < beff && bw_coff(beff, j) < (int)((int64_t)total * q / CS)) ++j;
+        part.c[q] = j;
       }
-      if (occ < 1) occ = 1;
-      int64_t grid = (int64_t)num_sms() * occ;
-      if (grid > max_grid) grid = max_grid;
-      if (use_sm) bc_kernel<true><<<(unsigned)grid, BC_NT, smem, st>>>(a);
-      else bc_kernel<false><<<(unsigned)grid, BC_NT, smem, st>>>(a);
+      part.c[CS] = beff;
+      int maxw = 0;
+      for (int q = 0; q < CS; ++q) {
+        const int w = bw_coff(beff, part.c[q + 1]) - bw_coff(beff, part.c[q]);
+        if (w > maxw) maxw = w;
+      }
+      const size_t smem = sizeof(double) * ((size_t)2 * beff + 4 * (size_t)beff + 2 * (size_t)beff + 16 + maxw);
+      if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
+      const void* fn = CS == 1 ? (const void*)bc_wide_kernel<1> : (const void*)bc_wide_kernel<4>;
+      cudaError_t e2 = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e2 != cudaSuccess) return e2;
+      if (CS == 1) {
+        int64_t grid = num_sms();
+        if (grid > max_grid) grid = max_grid;
+        bc_wide_kernel<1><<<(unsigned)grid, BW_NT, smem, st>>>(a, part);
+      } else {
+        cudaLaunchConfig_t cfg = {};
+        cfg.blockDim = dim3(BW_NT);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = (unsigned)CS;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cfg.gridDim = dim3((unsigned)(CS * 37));
+        int nc = 0;
+        if (cudaOccupancyMaxActiveClusters(&nc, fn, &cfg) != cudaSuccess || nc < 1) return cudaErrorInvalidConfiguration;
+        int64_t ncl = nc;
+        if (ncl > max_grid) ncl = max_grid;
+        cfg.gridDim = dim3((unsigned)(ncl * CS));
+        e2 = cudaLaunchKernelEx(&cfg, bc_wide_kernel<4>, a, part);
+        if (e2 != cudaSuccess) return e2;
+      }
     }
     count_launches(1);
     err = cudaGetLastError();
