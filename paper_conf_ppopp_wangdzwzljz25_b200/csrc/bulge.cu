@@ -770,16 +770,22 @@ struct BwPart {
 // offset (doubles) of window column j in the packed trapezoid, columns of 2b - j rows rounded up to even
 __host__ __device__ __forceinline__ int bw_coff(int b, int j) { return 2 * b * j - j * (j - 1) / 2 + j / 2; }
 
+// DSMEM access to the same shared variable in cluster rank `rank` (shared::cluster addresses from mapa); CS == 1:
+// plain shared memory
 template <int CS>
-__device__ __forceinline__ double* bw_peer(double* p, unsigned rank) {
+__device__ __forceinline__ double bw_ld(const double* p, unsigned rank) {
   if constexpr (CS == 1) {
-    return p;
+    return *p;
   } else {
-    // generic address of the same variable in the shared memory of cluster rank `rank`
-    double* r;
-    asm volatile("mapa.u64 %0, %1, %2;\n" : "=l"(r) : "l"(p), "r"(rank));
-    return r;
+    double v;
+    asm volatile("ld.shared::cluster.f64 %0, [%1];\n" : "=d"(v) : "r"(cl_mapa(p, rank)) : "memory");
+    return v;
   }
+}
+template <int CS>
+__device__ __forceinline__ void bw_st(double* p, unsigned rank, double v) {
+  if constexpr (CS == 1) *p = v;
+  else asm volatile("st.shared::cluster.f64 [%0], %1;\n" ::"r"(cl_mapa(p, rank)), "d"(v) : "memory");
 }
 template <int CS>
 __device__ __forceinline__ void bw_csync() {
@@ -795,29 +801,30 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
   const int64_t n = a.n;
   const unsigned q = CS > 1 ? cl_rank() : 0u;
   const int cbeg = part.c[q], cend = part.c[q + 1];
-  const int base_off = bw_coff(b, cbeg);
   const int H2 = 2 * b;
-  // shared layout: vb[2][b] | prt[2b] | pf[2b] | w[b] | colv[b] | scal[16] | window
+  // shared layout: vb[2][b] | prt[2][2b] | pf[2b] | w[b] | colv[b] | scal[16] | sweep[2] | cofs[b] (ints) | window
   double* vb = sm;
-  double* prt = vb + 2 * b;
-  double* pf = prt + H2;
+  double* prt = vb + 2 * b;   // [0, 2b): this CTA's partial matvec; [2b, 4b): the second half-row partial
+  double* pf = prt + 2 * H2;
   double* wv = pf + H2;
   double* colv = wv + b;
   double* scal = colv + b;   // 0 pv, 1..3 reflector of column s (beta, tau, scale), 4..6 next reflector
-  double* win = scal + 16;
-  __shared__ int64_t s_sweep;
-  auto W = [&](int i, int j) -> double& { return win[bw_coff(b, j) - base_off + (i - j)]; };   // i >= j, j mine
-  for (int64_t sweep_i = 0;; ++sweep_i) {
+  double* swp = scal + 16;   // the claimed sweep (as a double-sized slot)
+  int* cofs = reinterpret_cast<int*>(swp + 2);
+  double* win = sm + ((10 * b + 18 + (b + 1) / 2 + 1) & ~1);   // 16-byte aligned, past cofs
+  // window element (i, j), i >= j, of my column j: win[cofs[j] + i]
+  for (int j = tid; j < b; j += BW_NT) cofs[j] = (j >= cbeg && j < cend) ? bw_coff(b, j) - bw_coff(b, cbeg) - j : 0;
+  __syncthreads();
+  // threads per window row in the matvec (b <= 128: two, each over half of my columns)
+  const int tpr = BW_NT / H2 >= 2 ? 2 : 1;
+  const int jmid = cbeg + (cend - cbeg + 1) / 2;
+  for (;;) {
     if (q == 0 && tid == 0) {
-      const int64_t s0 = (int64_t)atomicAdd(a.ticket, 1u);
-      if constexpr (CS == 1) {
-        s_sweep = s0;
-      } else {
-        for (unsigned r = 0; r < CS; ++r) *reinterpret_cast<int64_t*>(bw_peer<CS>((double*)&s_sweep, r)) = s0;
-      }
+      const double s0 = (double)atomicAdd(a.ticket, 1u);   // exact (< 2^53)
+      for (unsigned r = 0; r < CS; ++r) bw_st<CS>(swp, r, s0);
     }
     bw_csync<CS>();
-    const int64_t s = s_sweep;
+    const int64_t s = (int64_t)swp[0];
     bw_csync<CS>();
     if (s > n - 3) return;
     const int64_t nst = bc_steps(n, b, s);
@@ -834,21 +841,21 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       const int L2 = (int)(r2 - r1);
       const int H = L + L2;
       const int je = cend < L ? cend : L;   // my window columns [cbeg, je)
+      const double* gw = a.band + r0 * ldab;   // window column j at gw + j*ldab (rows j.. at offsets 0..)
       // ---- lag-2 dependency (R9): sweep s-1 has completed step m+1 (serial mode: all of its steps)
       if (s > 0) {
         if (tid == 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev));
         __syncthreads();
       }
-      // ---- load my window columns (rows j .. H-1 of column j: offsets 0 .. H-1-j)
-      for (int j = cbeg; j < je; ++j) {
+      // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j)
+      for (int j = cbeg + warp; j < je; j += NW) {
         const int len = H - j, len2 = len >> 1;
-        double* dst = &W(j, j);
-        const double* src = a.band + (r0 + j) * ldab;
-        for (int i = tid; i < len2; i += BW_NT) {
+        double* dst = win + cofs[j] + j;
+        const double* src = gw + (int64_t)j * ldab;
+        for (int i = lane; i < len2; i += 32)
           asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(dst + 2 * i)), "l"(src + 2 * i)
                        : "memory");
-        }
-        if ((len & 1) && tid == BW_NT - 1) dst[len - 1] = __ldcg(src + len - 1);
+        if ((len & 1) && lane == 0) dst[len - 1] = __ldcg(src + len - 1);
       }
       asm volatile("cp.async.commit_group;\n" ::: "memory");
       // ---- step 0: the reflector annihilating column s below its first subdiagonal (every CTA, same bits)
@@ -875,19 +882,28 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       __syncthreads();
       // ---- 1. partial matvec [D; O] v over my columns, all H rows
       if (tau != 0.0) {
-        for (int i = tid; i < H2; i += BW_NT) {
-          double acc = 0.0;
-          if (i < H) {
-            const int jt = je < i + 1 ? je : i + 1;   // lower part of D (and all of O): columns j <= i
-            for (int j = cbeg; j < jt; ++j) acc = fma(W(i, j), v[j], acc);
+        {
+          const int i = tid % H2, h = tid / H2;   // row i, half h (tpr == 2) of my columns
+          if (h < tpr) {
+            double acc = 0.0;
+            if (i < H) {
+              const int jlo = tpr == 2 ? (h ? jmid : cbeg) : cbeg;
+              int jhi = tpr == 2 ? (h ? je : (jmid < je ? jmid : je)) : je;
+              if (jhi > i + 1) jhi = i + 1;   // lower part of D (and all of O): columns j <= i
+              for (int j = jlo; j < jhi; ++j) acc = fma(win[cofs[j] + i], v[j], acc);
+            }
+            prt[h * H2 + i] = acc;
           }
-          prt[i] = acc;
         }
+        __syncthreads();
+        if (tpr == 2)
+          for (int i = tid; i < H2; i += BW_NT) prt[i] += prt[H2 + i];
         __syncthreads();
         // mirrored upper part of D for my columns c: sum_{j > c, j < L} D(j, c) v_j (a column dot, one warp)
         for (int c = cbeg + warp; c < je; c += NW) {
+          const double* col = win + cofs[c];
           double acc = 0.0;
-          for (int j = c + 1 + lane; j < L; j += 32) acc = fma(W(j, c), v[j], acc);
+          for (int j = c + 1 + lane; j < L; j += 32) acc = fma(col[j], v[j], acc);
           acc = warp_sum(acc);
           if (lane == 0) prt[c] += acc;
         }
@@ -896,7 +912,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         for (int i = tid; i < H; i += BW_NT) {
           double acc = 0.0;
 #pragma unroll
-          for (unsigned r = 0; r < CS; ++r) acc += *bw_peer<CS>(prt + i, r);
+          for (unsigned r = 0; r < CS; ++r) acc += bw_ld<CS>(prt + i, r);
           pf[i] = i < L ? tau * acc : acc;
         }
         __syncthreads();
@@ -910,14 +926,13 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         const double hp = 0.5 * tau * scal[0];
         for (int i = tid; i < L; i += BW_NT) wv[i] = fma(-hp, v[i], pf[i]);
         __syncthreads();
-        // ---- 3. D -= v w^T + w v^T (lower, my columns), O -= tau y v^T (my columns)
-        for (int j = cbeg; j < je; ++j) {
+        // ---- 3. D -= v w^T + w v^T (lower, my columns), O -= tau y v^T (my columns); one warp per column
+        for (int j = cbeg + warp; j < je; j += NW) {
+          double* col = win + cofs[j];
           const double vj = v[j], wj = wv[j], tvj = tau * vj;
-          for (int i = j + tid; i < H; i += BW_NT) {
-            double& x = W(i, j);
-            if (i < L) x = fma(-wv[i], vj, fma(-v[i], wj, x));
-            else x = fma(-pf[i], tvj, x);
-          }
+          int i = j + lane;
+          for (; i < L; i += 32) col[i] = fma(-wv[i], vj, fma(-v[i], wj, col[i]));
+          for (; i < H; i += 32) col[i] = fma(-pf[i], tvj, col[i]);
         }
       }
       // ---- 4. the next reflector from O(:, 0) (window column 0: rank 0), broadcast
@@ -925,32 +940,29 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       if (L2 > 0) {
         __syncthreads();
         if (q == 0) {
+          double* c0 = win + cofs[0];
           if (warp == 0) {
             double sg = 0.0;
-            for (int i = 1 + lane; i < L2; i += 32) {
-              const double x = W(L + i, 0);
-              sg = fma(x, x, sg);
-            }
+            for (int i = 1 + lane; i < L2; i += 32) sg = fma(c0[L + i], c0[L + i], sg);
             sg = warp_sum(sg);
             if (lane == 0) {
-              const House h = make_house(W(L, 0), sg);
+              const House h = make_house(c0[L], sg);
               for (unsigned r = 0; r < CS; ++r) {
-                double* sc = bw_peer<CS>(scal, r);
-                sc[4] = h.beta;
-                sc[5] = h.tau;
-                sc[6] = h.scale;
+                bw_st<CS>(scal + 4, r, h.beta);
+                bw_st<CS>(scal + 5, r, h.tau);
+                bw_st<CS>(scal + 6, r, h.scale);
               }
             }
           }
           __syncthreads();
           const double hs = scal[6];
           for (int i = tid; i < b; i += BW_NT) {
-            const double x = i < L2 ? (i == 0 ? 1.0 : hs * W(L + i, 0)) : 0.0;
+            const double x = i < L2 ? (i == 0 ? 1.0 : hs * c0[L + i]) : 0.0;
 #pragma unroll
-            for (unsigned r = 0; r < CS; ++r) bw_peer<CS>(vn, r)[i] = x;
+            for (unsigned r = 0; r < CS; ++r) bw_st<CS>(vn + i, r, x);
           }
           __syncthreads();
-          for (int i = tid; i < L2; i += BW_NT) W(L + i, 0) = i == 0 ? scal[4] : 0.0;
+          for (int i = tid; i < L2; i += BW_NT) c0[L + i] = i == 0 ? scal[4] : 0.0;
         }
         bw_csync<CS>();   // (2) vn and its scalars everywhere
         taun = scal[5];
@@ -958,22 +970,24 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (taun != 0.0) {
           const int j1 = cbeg > 1 ? cbeg : 1;
           for (int c = j1 + warp; c < je; c += NW) {
+            double* col = win + cofs[c] + L;
             double acc = 0.0;
-            for (int i = lane; i < L2; i += 32) acc = fma(vn[i], W(L + i, c), acc);
+            for (int i = lane; i < L2; i += 32) acc = fma(vn[i], col[i], acc);
             acc = warp_sum(acc);
             const double tz = taun * acc;
-            for (int i = lane; i < L2; i += 32) W(L + i, c) = fma(-tz, vn[i], W(L + i, c));
+            for (int i = lane; i < L2; i += 32) col[i] = fma(-tz, vn[i], col[i]);
           }
         }
       }
       __syncthreads();
-      // ---- store my columns back, the reflector of this step, publish
-      for (int j = cbeg; j < je; ++j) {
+      // ---- store my columns back (one warp per column), the reflector of this step, publish
+      for (int j = cbeg + warp; j < je; j += NW) {
         const int len = H - j, len2 = len >> 1;
-        const double2* srcp = reinterpret_cast<const double2*>(&W(j, j));
-        double2* dst = reinterpret_cast<double2*>(a.band + (r0 + j) * ldab);
-        for (int i = tid; i < len2; i += BW_NT) __stcg(dst + i, srcp[i]);
-        if ((len & 1) && tid == BW_NT - 1) __stcg(a.band + (r0 + j) * ldab + len - 1, W(H - 1, j));
+        const double* srcp = win + cofs[j] + j;
+        double* dst = a.band + (r0 + j) * ldab;
+        for (int i = lane; i < len2; i += 32)
+          __stcg(reinterpret_cast<double2*>(dst) + i, reinterpret_cast<const double2*>(srcp)[i]);
+        if ((len & 1) && lane == 0) __stcg(dst + len - 1, srcp[len - 1]);
       }
       if (q == 0 && a.V2) {
         double* vd = a.V2 + (off + m) * a.vs;
@@ -1104,7 +1118,11 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       }
     } else {
       // 64 < b <= 256: bc_wide_kernel, one CTA per sweep (b <= 128) or a cluster of 4 (b > 128)
-      const int CS = beff <= 128 ? 1 : 4;
+      int CS = beff <= 128 ? 1 : 4;
+      {
+        const char* ce = getenv("TRID_BC_WCS");   // debug/A-B: force the cluster split (1, 2 or 4)
+        if (ce && (atoi(ce) == 1 || atoi(ce) == 2 || atoi(ce) == 4)) CS = atoi(ce);
+      }
       BwPart part{};
       const int total = bw_coff(beff, beff);
       part.c[0] = 0;
@@ -1119,9 +1137,11 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
         const int w = bw_coff(beff, part.c[q + 1]) - bw_coff(beff, part.c[q]);
         if (w > maxw) maxw = w;
       }
-      const size_t smem = sizeof(double) * ((size_t)2 * beff + 4 * (size_t)beff + 2 * (size_t)beff + 16 + maxw);
+      // vb 2b | prt 4b | pf 2b | w b | colv b | scal 16 | sweep 2 | cofs (b ints) + pad | window
+      const size_t smem = sizeof(double) * ((size_t)((10 * beff + 18 + (beff + 1) / 2 + 1) & ~1) + maxw);
       if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
-      const void* fn = CS == 1 ? (const void*)bc_wide_kernel<1> : (const void*)bc_wide_kernel<4>;
+      const void* fn = CS == 1 ? (const void*)bc_wide_kernel<1>
+                               : (CS == 2 ? (const void*)bc_wide_kernel<2> : (const void*)bc_wide_kernel<4>);
       cudaError_t e2 = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       if (e2 != cudaSuccess) return e2;
       if (CS == 1) {
@@ -1146,7 +1166,8 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
         int64_t ncl = nc;
         if (ncl > max_grid) ncl = max_grid;
         cfg.gridDim = dim3((unsigned)(ncl * CS));
-        e2 = cudaLaunchKernelEx(&cfg, bc_wide_kernel<4>, a, part);
+        e2 = CS == 2 ? cudaLaunchKernelEx(&cfg, bc_wide_kernel<2>, a, part)
+                     : cudaLaunchKernelEx(&cfg, bc_wide_kernel<4>, a, part);
         if (e2 != cudaSuccess) return e2;
       }
     }
