@@ -847,6 +847,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (tid == 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev));
         __syncthreads();
       }
+      if (a.opt & 64) bw_csync<CS>();   // debug (TRID_BC_OPT): extra cluster barriers
       // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j)
       for (int j = cbeg + warp; j < je; j += NW) {
         const int len = H - j, len2 = len >> 1;
@@ -871,7 +872,6 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
             scal[1] = h.beta;
             scal[2] = h.tau;
             scal[3] = h.scale;
-            if (q == 0) __stcg(a.band + s * ldab + 1, h.beta);   // e_s (the rest of column s is dead)
           }
         }
         __syncthreads();
@@ -880,6 +880,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       }
       asm volatile("cp.async.wait_group 0;\n" ::: "memory");
       __syncthreads();
+      if (a.opt & 128) bw_csync<CS>();
       // ---- 1. partial matvec [D; O] v over my columns, all H rows
       if (tau != 0.0) {
         {
@@ -923,6 +924,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           if (lane == 0) scal[0] = pv;
         }
         __syncthreads();
+        if (a.opt & 512) bw_csync<CS>();
         const double hp = 0.5 * tau * scal[0];
         for (int i = tid; i < L; i += BW_NT) wv[i] = fma(-hp, v[i], pf[i]);
         __syncthreads();
@@ -980,6 +982,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         }
       }
       __syncthreads();
+      if (a.opt & 256) bw_csync<CS>();
       // ---- store my columns back (one warp per column), the reflector of this step, publish
       for (int j = cbeg + warp; j < je; j += NW) {
         const int len = H - j, len2 = len >> 1;
@@ -995,7 +998,11 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (tid == 0) a.tau2[off + m] = tau;
       }
       bw_csync<CS>();   // (3) every CTA's stores of this step issued (ordered before the release below)
-      if (q == 0 && tid == 0) st_release_s32(a.prog + s, (int)(m + 1));
+      if (q == 0 && tid == 0) {
+        // e_s (the rest of column s is dead): written only now, when every CTA of the cluster has read column s
+        if (m == 0) __stcg(a.band + s * ldab + 1, scal[1]);
+        st_release_s32(a.prog + s, (int)(m + 1));
+      }
       tau = taun;
     }
   }
