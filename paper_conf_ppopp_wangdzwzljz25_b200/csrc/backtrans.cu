@@ -72,30 +72,21 @@ __global__ void bt_tfactor_kernel(int b, int kg, const double* G, const double* 
   }
 }
 
+cudaError_t tfactor_from_gram(int b, int kg, const double* G, const double* tau, double* T, cudaStream_t st) {
+  const int np = (kg + b - 1) / b;
+  bt_tfactor_kernel<<<np, 128, 0, st>>>(b, kg, G, tau, T);
+  count_launches(1);
+  return cudaGetLastError();
+}
+
 namespace {
 size_t a256(size_t x) { return (x + 255) / 256 * 256; }
 
-int ws_splits(int64_t M, int64_t N, int64_t K, int64_t part_elems) {
-  const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
-  int64_t s = (3 * kNumSMsB200 + tiles - 1) / tiles;   // fixed count: deterministic summation order
-  const int64_t maxk = K / 256;
-  if (s > maxk) s = maxk;
-  if (s > 64) s = 64;
-  if (s > 1 && s * M * N > part_elems) s = part_elems / (M * N);
-  return s < 1 ? 1 : (int)s;
-}
-
-// C (M x N) = alpha op(A) op(B) + beta Cin on the DMMA engine, split-K when the output grid is small
+// C (M x N) = alpha op(A) op(B) + beta Cin on the DMMA engine (gemm_ws_mm, split-K when the grid is small)
 cudaError_t mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
                const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part, int64_t part_elems,
                cudaStream_t st) {
-  if (M <= 0 || N <= 0) return cudaSuccess;
-  GemmArgs g;
-  g.M = M; g.N = N; g.K[0] = K; g.A[0] = A; g.lda[0] = lda; g.B[0] = B; g.ldb[0] = ldb;
-  g.alpha = alpha; g.beta = beta; g.Cin = C; g.ldcin = ldc; g.C = C; g.ldc = ldc;
-  g.splits = ws_splits(M, N, K, part_elems);
-  g.part = part; g.part_ld = M; g.part_stride = M * N;
-  return gemm_ws_op(g, opA, opB, st);
+  return gemm_ws_mm(opA, opB, M, N, K, alpha, A, lda, B, ldb, beta, C, ldc, part, part_elems, st);
 }
 
 struct SbrBtWork {

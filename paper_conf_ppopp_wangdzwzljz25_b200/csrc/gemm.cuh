@@ -64,6 +64,10 @@ int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elem
 // Warp-specialized persistent engine (gemm_ws.cu): tiles 128x128 (N > 64) / 128x64.  gemm_ws: op(A) = A.
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
 cudaError_t gemm_ws_op(GemmArgs a, int opA, int opB, cudaStream_t st);
+// C (M x N) = alpha op(A) op(B) + beta Cin (ld lda/ldb/ldc), deterministic split-K over part (part_elems doubles)
+cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
+                       const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
+                       int64_t part_elems, cudaStream_t st);
 int64_t symm_ws_splits(int64_t m, int64_t w);
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K);
 int64_t symm_ws_part_elems(int64_t m, int64_t w);

@@ -533,6 +533,27 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 
+// C (M x N) = alpha op(A) op(B) + beta Cin with a fixed split-K count (deterministic sums) when the output grid is
+// small: ~3 waves of units, >= 256 of K per split, <= 64 splits, within part_elems partials.
+cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
+                       const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
+                       int64_t part_elems, cudaStream_t st) {
+  if (M <= 0 || N <= 0) return cudaSuccess;
+  const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
+  int64_t s = (3 * kNumSMsB200 + tiles - 1) / tiles;
+  const int64_t maxk = K / 256;
+  if (s > maxk) s = maxk;
+  if (s > 64) s = 64;
+  if (s > 1 && s * M * N > part_elems) s = part_elems / (M * N);
+  if (s < 1) s = 1;
+  GemmArgs g;
+  g.M = M; g.N = N; g.K[0] = K; g.A[0] = A; g.lda[0] = lda; g.B[0] = B; g.ldb[0] = ldb;
+  g.alpha = alpha; g.beta = beta; g.Cin = C; g.ldcin = ldc; g.C = C; g.ldc = ldc;
+  g.splits = (int)s;
+  g.part = part; g.part_ld = M; g.part_stride = M * N;
+  return gemm_ws_op(g, opA, opB, st);
+}
+
 // Split-K for the skinny engine GEMMs (M = trailing rows, N = b, K = 2 x block columns): enough units for
 // ~3 waves of the persistent grid, >= 256 of K per split, <= 16 splits.  Partials: splits * M * N doubles.
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {

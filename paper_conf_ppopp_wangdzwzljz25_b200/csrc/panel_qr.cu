@@ -9,7 +9,9 @@
 // vector w_j = v^T P(:,j) = P(t,j) + scale * sum x_r P(r,j) (j > t) and the T-factor inner products
 // v_t^T v_q (q < t), then applies the rank-1 update to its own rows.  Totals are summed in a fixed
 // CTA order, so every CTA (and every run) sees bitwise-identical values.
+#include "backtrans.cuh"
 #include "common.cuh"
+#include "gemm.cuh"
 #include "panel.cuh"
 #include "prof.cuh"
 
@@ -197,15 +199,70 @@ static int panel_grid(int64_t m) {
   return (int)G;
 }
 
-size_t panel_red_bytes(int w) {
+constexpr int PB_IB = 64;   // inner block of the nb-blocked panel (the register kernel's widest panel)
+static size_t panel_base_bytes(int w) {
   return sizeof(double) * (2 * (size_t)kNumSMsB200 * 2 * (size_t)w + 2 * 2 * (size_t)w) + sizeof(long long) * 2 * 256 * 8;
+}
+// blocked-path scratch (w > 64): T_k (ib x ib), X and X2 (ib x w), the Gram G (w x w), split-K partials (16 w^2)
+static size_t panel_blocked_elems(int w) {
+  return (size_t)PB_IB * PB_IB + 2 * (size_t)PB_IB * w + (size_t)w * w + 16 * (size_t)w * w;
+}
+size_t panel_red_bytes(int w) {
+  size_t base = (panel_base_bytes(w) + 255) / 256 * 256;
+  if (w > PB_IB) base += sizeof(double) * panel_blocked_elems(w);
+  return base;
+}
+
+// nb-blocked panel QR for w > 64 (north_star: "Householder panel QR on nb-wide panels"): the panel is
+// factored in sub-panels of ib = 64 columns by the register kernel; after each, its compact-WY block (I - Y_k T_k
+// Y_k^T) is applied from the left (transposed) to the remaining columns with three DMMA contractions
+// (X = Y_k^T C, X2 = T_k^T X, C -= Y_k X2); finally T of the whole panel from the Gram Y^T Y (dlarft).  The
+// reflectors are those of the unblocked column-by-column QR (blocked Householder QR), up to rounding.
+static cudaError_t panel_qr_blocked(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, double* Y,
+                                    int64_t ldy, double* red, unsigned* bar, cudaStream_t st) {
+  const int ib = PB_IB;
+  const int kk = (int)(m < w ? m : w);
+  double* scr = (double*)((char*)red + (panel_base_bytes(w) + 255) / 256 * 256);
+  double* Tk = scr;
+  double* X = Tk + (size_t)ib * ib;
+  double* X2 = X + (size_t)ib * w;
+  double* G = X2 + (size_t)ib * w;
+  double* part = G + (size_t)w * w;
+  const int64_t part_elems = 16 * (int64_t)w * w;
+  cudaError_t e = cudaMemset2DAsync(Y, sizeof(double) * ldy, 0, sizeof(double) * m, kk, st);
+  if (e != cudaSuccess) return e;
+  for (int k = 0; k < kk; k += ib) {
+    const int bk = (kk - k) < ib ? (kk - k) : ib;
+    const int64_t mk = m - k;
+    if ((e = panel_qr_reg(mk, bk, P + k + (int64_t)k * ldp, ldp, tau + k, Tk, ib, Y + k + (int64_t)k * ldy, ldy, red,
+                          bar, st)) != cudaSuccess)
+      return e;
+    const int nc = w - k - bk;
+    if (nc <= 0) continue;
+    double* C = P + k + (int64_t)(k + bk) * ldp;
+    const double* Yk = Y + k + (int64_t)k * ldy;
+    if ((e = gemm_ws_mm(OP_T, OP_N, bk, nc, mk, 1.0, Yk, ldy, C, ldp, 0.0, X, ib, part, part_elems, st)) != cudaSuccess)
+      return e;
+    if ((e = gemm_ws_mm(OP_T, OP_N, bk, nc, bk, 1.0, Tk, ib, X, ib, 0.0, X2, ib, part, part_elems, st)) != cudaSuccess)
+      return e;
+    if ((e = gemm_ws_mm(OP_N, OP_N, mk, nc, bk, -1.0, Yk, ldy, X2, ib, 1.0, C, ldp, part, part_elems, st)) !=
+        cudaSuccess)
+      return e;
+  }
+  // T of the whole panel: G = Y^T Y, then the dlarft recurrence (one CTA)
+  if ((e = gemm_ws_mm(OP_T, OP_N, kk, kk, m, 1.0, Y, ldy, Y, ldy, 0.0, G, w, part, part_elems, st)) != cudaSuccess)
+    return e;
+  if ((e = cudaMemsetAsync(T, 0, sizeof(double) * (size_t)w * w, st)) != cudaSuccess) return e;
+  return tfactor_from_gram(w, kk, G, tau, T, st);
 }
 
 cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double* T, int64_t ldt, double* Y,
                      int64_t ldy, double* red, unsigned* bar, cudaStream_t st) {
   if (m <= 0 || w <= 0) return cudaSuccess;
-  if (panel_reg_supported(m, w) && !getenv("TRID_PANEL_SMEM"))
-    return panel_qr_reg(m, w, P, ldp, tau, T, ldt, Y, ldy, red, bar, st);
+  static const bool force_general = getenv("TRID_PANEL_SMEM") != nullptr;   // A/B: the general kernel for every w
+  if (panel_reg_supported(m, w) && !force_general) return panel_qr_reg(m, w, P, ldp, tau, T, ldt, Y, ldy, red, bar, st);
+  if (w > PB_IB && ldt == w && panel_reg_supported(m, PB_IB) && !force_general)
+    return panel_qr_blocked(m, w, P, ldp, tau, T, Y, ldy, red, bar, st);
   const int G = panel_grid(m);
   PanelArgs a;
   a.m = m; a.w = w; a.kk = (int)(m < w ? m : w);

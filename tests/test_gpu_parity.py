@@ -94,7 +94,8 @@ def test_zy_parity(m, w, dev):
 
 # ------------------------------------------------------------------------------------------ DBBR
 @pytest.mark.parametrize("n,b,k", [(256, 32, 32), (256, 32, 64), (256, 32, 128), (256, 32, 256), (300, 32, 96),
-                                   (513, 16, 64), (257, 64, 128), (100, 8, 24), (40, 4, 8), (1000, 64, 256)])
+                                   (513, 16, 64), (257, 64, 128), (100, 8, 24), (40, 4, 8), (1000, 64, 256),
+                                   (700, 128, 256), (900, 256, 512), (600, 96, 192)])
 def test_dbbr_parity(n, b, k, dev):
     A = trid_gen.random_symmetric_np(n, 1001)
     Ao, to = oracle.dbbr(A, b, k)
@@ -220,7 +221,7 @@ def test_bulge_chase_noop_cases(dev):
 
 # ------------------------------------------------------------------------------------------ both stages
 @pytest.mark.parametrize("n,b,k", [(256, 32, 32), (256, 32, 256), (256, 32, 1024), (300, 32, 64), (513, 64, 128),
-                                   (1000, 16, 128), (1024, 64, 1024)])
+                                   (1000, 16, 128), (1024, 64, 1024), (700, 128, 256), (800, 256, 512)])
 def test_two_stage_gates(n, b, k, dev):
     A = trid_gen.random_symmetric_np(n, 1001 + n)
     d_o, e_o, Ao, t1o, V_o, t2o = oracle.tridiagonalize(A, b, k)
