@@ -232,14 +232,16 @@ static cudaError_t panel_qr_blocked(int64_t m, int w, double* P, int64_t ldp, do
   cudaError_t e = cudaMemset2DAsync(Y, sizeof(double) * ldy, 0, sizeof(double) * m, kk, st);
   if (e != cudaSuccess) return e;
   for (int k = 0; k < kk; k += ib) {
-    const int bk = (kk - k) < ib ? (kk - k) : ib;
+    // sub-panel columns [k, k + bw) (bw in {16, 32, 64}: w % 16 == 0), min(m - k, bw) reflectors
+    const int bw = (w - k) < ib ? (w - k) : ib;
     const int64_t mk = m - k;
-    if ((e = panel_qr_reg(mk, bk, P + k + (int64_t)k * ldp, ldp, tau + k, Tk, ib, Y + k + (int64_t)k * ldy, ldy, red,
+    const int bk = (int)(mk < bw ? mk : bw);
+    if ((e = panel_qr_reg(mk, bw, P + k + (int64_t)k * ldp, ldp, tau + k, Tk, ib, Y + k + (int64_t)k * ldy, ldy, red,
                           bar, st)) != cudaSuccess)
       return e;
-    const int nc = w - k - bk;
+    const int nc = w - k - bw;
     if (nc <= 0) continue;
-    double* C = P + k + (int64_t)(k + bk) * ldp;
+    double* C = P + k + (int64_t)(k + bw) * ldp;
     const double* Yk = Y + k + (int64_t)k * ldy;
     if ((e = gemm_ws_mm(OP_T, OP_N, bk, nc, mk, 1.0, Yk, ldy, C, ldp, 0.0, X, ib, part, part_elems, st)) != cudaSuccess)
       return e;
@@ -261,7 +263,7 @@ cudaError_t panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, doub
   if (m <= 0 || w <= 0) return cudaSuccess;
   static const bool force_general = getenv("TRID_PANEL_SMEM") != nullptr;   // A/B: the general kernel for every w
   if (panel_reg_supported(m, w) && !force_general) return panel_qr_reg(m, w, P, ldp, tau, T, ldt, Y, ldy, red, bar, st);
-  if (w > PB_IB && ldt == w && panel_reg_supported(m, PB_IB) && !force_general)
+  if (w > PB_IB && w % 16 == 0 && ldt == w && panel_reg_supported(m, PB_IB) && !force_general)
     return panel_qr_blocked(m, w, P, ldp, tau, T, Y, ldy, red, bar, st);
   const int G = panel_grid(m);
   PanelArgs a;
