@@ -303,6 +303,9 @@ def main():
     ap.add_argument("--ref-n", type=int, default=1024)
     ap.add_argument("--eig-only", action="store_true", help="eigenvalues-only BC (V2 = NULL)")
     ap.add_argument("--dry-run", action="store_true", help="rank plumbing only (gloo, no GPU work)")
+    ap.add_argument("--mode", default="sharded", choices=["sharded", "replicas"],
+                    help="N > 1: sharded = one matrix, stage 1 sharded over the ranks (strong scaling); replicas = "
+                         "one independent matrix per rank (batched multi-matrix tridiagonalization, weak scaling)")
     ap.add_argument("--oracle-worker", nargs=5, metavar=("N", "B", "SEED", "KIND", "FLAGS"), help=argparse.SUPPRESS)
     args = ap.parse_args()
     if args.oracle_worker:
@@ -346,11 +349,13 @@ def main():
 
     want = not args.eig_only
     stream = torch.cuda.current_stream()
-    if ws == 1:
+    sharded = ws > 1 and args.mode == "sharded"
+    if not sharded:
+        seed = cfg["seed"] + (rank if ws > 1 else 0)   # replicas: an independent matrix per rank
         if cfg.get("kind"):
-            A0, _ = trid_gen.clustered_symmetric(n, cfg["seed"], kind=cfg["kind"], device=dev)
+            A0, _ = trid_gen.clustered_symmetric(n, seed, kind=cfg["kind"], device=dev)
         else:
-            A0 = trid_gen.random_symmetric(n, cfg["seed"], device=dev)
+            A0 = trid_gen.random_symmetric(n, seed, device=dev)
         A = torch.empty_like(A0)
         nbytes, v2len, t2len = trid.sytrd_2stage_bufsize(n, b, nb, k)
         work = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
@@ -421,7 +426,8 @@ def main():
         ms = float(t.item())
 
     flop = 4.0 * n ** 3 / 3.0
-    value = flop * args.steps / (ms * 1e-3) / 1e12   # one matrix per step for every N (strong scaling)
+    nmat = ws if (ws > 1 and not sharded) else 1   # matrices per step over all ranks
+    value = nmat * flop * args.steps / (ms * 1e-3) / 1e12   # sharded: one matrix per step (strong scaling)
     per = {c: (v[0] / args.steps, v[1] / args.steps) for c, v in stages.items()}
     t_bc = per["bulge_chase"][0]
     t_sbr = sum(per[c][0] for c in trid.SBR_CLASSES)
@@ -452,10 +458,11 @@ def main():
     line = {
         "metric": METRIC,
         "value": round(value, 4), "unit": "TFLOP/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "strong" if ws > 1 else "weak",
+        "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True, "scaling": "strong" if sharded else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": cfg["desc"], "n": n, "b": b, "nb": nb, "k": k, "seed": cfg["seed"],
-                   "parallelism": f"sbr-colblock-cyclic-x{ws}+bc-rank0" if ws > 1 else "single-gpu",
+                   "parallelism": (f"sbr-colblock-cyclic-x{ws}+bc-rank0" if sharded else
+                                   (f"replicas-x{ws}" if ws > 1 else "single-gpu")),
                    "l2": "inputs larger than L2 (n^2*8 B matrix restored from a resident copy each step)",
                    "vectors": "stored (V1 in A, tau1, V2, tau2)" if want else "eigenvalues-only"},
         "t_sbr_ms": round(t_sbr, 3), "t_bc_ms": round(t_bc, 3),
@@ -502,8 +509,8 @@ def main():
             t = torch.tensor([ems], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
-        line["e2e"] = {"value": round(flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
-                       "h2d_bytes_per_step": 8 * A0.numel() * ws, "d2h_bytes_per_step": 8 * (n + (n - 1) + n),
+        line["e2e"] = {"value": round(nmat * flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
+                       "h2d_bytes_per_step": 8 * A0.numel() * ws, "d2h_bytes_per_step": 8 * (n + (n - 1) + n) * nmat,
                        "note": "V1/V2 reflectors stay device-resident for the back transformation"}
         del Ah
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
