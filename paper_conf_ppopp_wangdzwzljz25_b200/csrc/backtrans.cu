@@ -215,8 +215,11 @@ template <int QR>
 __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int nb, const double* __restrict__ V2,
                                                         const double* __restrict__ tau2, int trans, int64_t ncols,
                                                         double* C, int64_t ldc) {
-  extern __shared__ __align__(16) double sv[];   // nb x b staged reflectors (zero padded to b), nb taus
-  double* stau = sv + (size_t)nb * b;
+  constexpr int RW = 8 * QR;        // window rows
+  constexpr int RWP = RW + 16;      // padded: row r at r + 2 (r / QR) (16-byte pad per row group: no LDS.128 conflicts)
+  // the group's reflectors in window shape: Vw[j][r] = v_j[r - j] (zero outside [0, b)), nb x RWP; then nb taus
+  extern __shared__ __align__(16) double sv[];
+  double* stau = sv + (size_t)nb * RWP;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rg = lane >> 2, cl = lane & 3;
   const int64_t col = (int64_t)blockIdx.x * BT_COLS + warp * 4 + cl;
@@ -224,7 +227,7 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   double* Cc = C + (colok ? col : 0) * ldc;
   const int64_t nsw = n - 2;   // sweeps 0 .. n-3
   const int64_t nblk = (nsw + nb - 1) / nb;
-  const int vstride = b;   // staged vector j at sv + j*b: its entry i sits at window row j + i
+  constexpr int NWB = BT_NT / 32;
   for (int64_t bi = 0; bi < nblk; ++bi) {
     const int64_t blk = trans ? bi : nblk - 1 - bi;
     const int64_t s0 = blk * nb;
@@ -233,16 +236,18 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
     for (int64_t gi = 0; gi < M; ++gi) {
       const int64_t m = trans ? M - 1 - gi : gi;
       const int64_t w0 = s0 + 1 + m * b;   // first row of the group window
-      // stage the group's reflectors: vector of sweep s0+j (if step m exists) and its tau
+      // stage the group's reflectors, one warp per vector (its V2 offset computed once): vector of sweep s0+j
       __syncthreads();
-      for (int idx = threadIdx.x; idx < nbb * vstride; idx += BT_NT) {
-        const int j = idx / vstride, i = idx - j * vstride;
+      for (int j = warp; j < nbb; j += NWB) {
         const int64_t s = s0 + j;
-        sv[idx] = m < bt_steps(n, b, s) ? V2[(bt_offset(n, b, s) + m) * b + i] : 0.0;
-      }
-      for (int j = threadIdx.x; j < nbb; j += BT_NT) {
-        const int64_t s = s0 + j;
-        stau[j] = m < bt_steps(n, b, s) ? tau2[bt_offset(n, b, s) + m] : 0.0;
+        const bool ex = m < bt_steps(n, b, s);
+        const double* vsrc = V2 + (ex ? (bt_offset(n, b, s) + m) * b : 0);
+        double* vd = sv + (size_t)j * RWP;
+        for (int r = lane; r < RW; r += 32) {
+          const int i = r - j;
+          vd[r + 2 * (r / QR)] = (ex && i >= 0 && i < b) ? vsrc[i] : 0.0;
+        }
+        if (lane == 0) stau[j] = ex ? tau2[bt_offset(n, b, s) + m] : 0.0;
       }
       __syncthreads();
       // the window rows of this thread: w0 + rg*QR + q
@@ -257,16 +262,13 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         const int j = trans ? jj : nbb - 1 - jj;
         const double tau = stau[j];
         if (tau == 0.0) continue;
-        // v entry for window row rg*QR + q is vector index (rg*QR + q) - j (zero outside [0, b)); the shared load
-        // index is clamped so it never leaves the staged vector
-        const double* vj = sv + (size_t)j * vstride;
-        const int base = rg * QR - j;
+        const double2* vj = reinterpret_cast<const double2*>(sv + (size_t)j * RWP + rg * (QR + 2));
         double vv[QR];
 #pragma unroll
-        for (int q = 0; q < QR; ++q) {
-          const int wr = base + q;
-          const int wc = wr < 0 ? 0 : (wr >= b ? b - 1 : wr);
-          vv[q] = (wr >= 0 && wr < b) ? vj[wc] : 0.0;
+        for (int q = 0; q < QR; q += 2) {
+          const double2 t = vj[q / 2];
+          vv[q] = t.x;
+          vv[q + 1] = t.y;
         }
         double d = 0.0;
 #pragma unroll
@@ -287,12 +289,14 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   }
 }
 
+static int bc_bt_rw(int b) { return b <= 64 ? 128 : (b <= 128 ? 256 : 512); }
+
 int bc_bt_nb(int b) {
-  // window 8*QR rows >= b + nb - 1 with QR = 16 (b <= 64) or 32 (b <= 128) or 64 (b <= 256); the nb staged vectors
-  // (nb * b doubles) fit in 200 KB of shared memory
-  const int rw = b <= 64 ? 128 : (b <= 128 ? 256 : 512);
+  // window RW = 8*QR rows >= b + nb - 1 (QR = 16 for b <= 64, 32 for b <= 128, 64 for b <= 256); the nb staged
+  // window-shaped vectors (nb x (RW + 16) doubles) fit in 200 KB of shared memory
+  const int rw = bc_bt_rw(b);
   int nb = rw - b + 1;
-  const int cap = (int)(200 * 1024 / (8 * (size_t)b)) - 1;
+  const int cap = (int)(200 * 1024 / (8 * (size_t)(rw + 16))) - 1;
   if (nb > cap) nb = cap;
   return nb < 1 ? 1 : nb;
 }
@@ -301,7 +305,7 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
                              double* C, int64_t ldc, cudaStream_t st) {
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
-  const size_t smem = sizeof(double) * ((size_t)nb * b + nb);
+  const size_t smem = sizeof(double) * ((size_t)nb * (bc_bt_rw(b) + 16) + nb);
   const int64_t grid = (ncols + BT_COLS - 1) / BT_COLS;
   const void* fn = b <= 64 ? (const void*)bc_bt_kernel<16> : (b <= 128 ? (const void*)bc_bt_kernel<32>
                                                                        : (const void*)bc_bt_kernel<64>);
