@@ -21,10 +21,10 @@
 // so this order keeps every overlapping pair in sweep-major order and only commutes disjoint ones.  Group G_m
 // touches rows [s0+1+mb, s0+nb-1+(m+1)b] (R = b+nb-1 rows).  Q2 C = B_0 (B_1 (... (B_last C))), B = G_M..G_0.
 // Kernel: one CTA per 32-column slab of C; per sweep block (last to first) it slides down the rows group by group
-// (G_0 first): the group's rows are loaded from the slab (HBM) into registers (8 row groups x 4 columns per warp,
-// QR rows per thread), its nb reflectors (from V2, staged in shared memory) are applied one at a time --
-// partial dot over the thread's rows, 3 warp shuffles, rank-1 update in registers -- and the rows that no later
-// group of the block touches go back to HBM.  One pass over the slab per sweep block: C traffic n^2 ncols 16 / nb
+// (G_0 first): the group's window rows are loaded from the slab into registers (a warp holds 4 columns; its 8 row
+// lanes per column hold interleaved row pairs, so every access is 16 consecutive rows), its nb reflectors (from V2,
+// staged once per group in shared memory in window shape, zero-padded) are applied one at a time -- partial dot over
+// the thread's rows (two chains), 3 warp shuffles, rank-1 update in registers -- and stored back.  One pass over the slab per sweep block: C traffic n^2 ncols 16 / nb
 // bytes, 4 n^2 ncols / 2 useful flops on the FP64 pipe (DFMA; B200's DFMA and DMMA peaks are equal).
 #include "common.cuh"
 #include "gemm.cuh"
@@ -215,11 +215,12 @@ template <int QR>
 __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int nb, const double* __restrict__ V2,
                                                         const double* __restrict__ tau2, int trans, int64_t ncols,
                                                         double* C, int64_t ldc) {
-  constexpr int RW = 8 * QR;        // window rows
-  constexpr int RWP = RW + 16;      // padded: row r at r + 2 (r / QR) (16-byte pad per row group: no LDS.128 conflicts)
-  // the group's reflectors in window shape: Vw[j][r] = v_j[r - j] (zero outside [0, b)), nb x RWP; then nb taus
+  constexpr int RW = 8 * QR;   // window rows
+  constexpr int NP = QR / 2;   // row pairs per thread: thread (rg, cl) holds rows 16 p + 2 rg + {0, 1}, p < NP, of
+                               // column cl -- the 8 row-group lanes of a column cover 16 consecutive rows (coalesced)
+  // the group's reflectors in window shape: Vw[j][r] = v_j[r - j] (zero outside [0, b)), nb x RW; then nb taus
   extern __shared__ __align__(16) double sv[];
-  double* stau = sv + (size_t)nb * RWP;
+  double* stau = sv + (size_t)nb * RW;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rg = lane >> 2, cl = lane & 3;
   const int64_t col = (int64_t)blockIdx.x * BT_COLS + warp * 4 + cl;
@@ -242,37 +243,43 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         const int64_t s = s0 + j;
         const bool ex = m < bt_steps(n, b, s);
         const double* vsrc = V2 + (ex ? (bt_offset(n, b, s) + m) * b : 0);
-        double* vd = sv + (size_t)j * RWP;
+        double* vd = sv + (size_t)j * RW;
         for (int r = lane; r < RW; r += 32) {
           const int i = r - j;
-          vd[r + 2 * (r / QR)] = (ex && i >= 0 && i < b) ? vsrc[i] : 0.0;
+          vd[r] = (ex && i >= 0 && i < b) ? vsrc[i] : 0.0;
         }
         if (lane == 0) stau[j] = ex ? tau2[bt_offset(n, b, s) + m] : 0.0;
       }
       __syncthreads();
-      // the window rows of this thread: w0 + rg*QR + q
+      // the window rows of this thread: w0 + 16 p + 2 rg + h
       double x[QR];
 #pragma unroll
-      for (int q = 0; q < QR; ++q) {
-        const int64_t r = w0 + rg * QR + q;
-        x[q] = (colok && r < n) ? Cc[r] : 0.0;
-      }
+      for (int p = 0; p < NP; ++p)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int64_t r = w0 + 16 * p + 2 * rg + h;
+          x[2 * p + h] = (colok && r < n) ? Cc[r] : 0.0;
+        }
       // G_m C applies H_{s0+nbb-1,m} first;  G_m^T C applies H_{s0,m} first
       for (int jj = 0; jj < nbb; ++jj) {
         const int j = trans ? jj : nbb - 1 - jj;
         const double tau = stau[j];
         if (tau == 0.0) continue;
-        const double2* vj = reinterpret_cast<const double2*>(sv + (size_t)j * RWP + rg * (QR + 2));
+        const double2* vj = reinterpret_cast<const double2*>(sv + (size_t)j * RW + 2 * rg);
         double vv[QR];
 #pragma unroll
-        for (int q = 0; q < QR; q += 2) {
-          const double2 t = vj[q / 2];
-          vv[q] = t.x;
-          vv[q + 1] = t.y;
+        for (int p = 0; p < NP; ++p) {
+          const double2 t = vj[8 * p];   // rows 16 p + 2 rg, +1
+          vv[2 * p] = t.x;
+          vv[2 * p + 1] = t.y;
         }
-        double d = 0.0;
+        double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-        for (int q = 0; q < QR; ++q) d = fma(vv[q], x[q], d);
+        for (int p = 0; p < NP; ++p) {
+          d0 = fma(vv[2 * p], x[2 * p], d0);
+          d1 = fma(vv[2 * p + 1], x[2 * p + 1], d1);
+        }
+        double d = d0 + d1;
         d += __shfl_xor_sync(0xffffffffu, d, 4);
         d += __shfl_xor_sync(0xffffffffu, d, 8);
         d += __shfl_xor_sync(0xffffffffu, d, 16);
@@ -281,10 +288,12 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         for (int q = 0; q < QR; ++q) x[q] = fma(-td, vv[q], x[q]);
       }
 #pragma unroll
-      for (int q = 0; q < QR; ++q) {
-        const int64_t r = w0 + rg * QR + q;
-        if (colok && r < n) Cc[r] = x[q];
-      }
+      for (int p = 0; p < NP; ++p)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int64_t r = w0 + 16 * p + 2 * rg + h;
+          if (colok && r < n) Cc[r] = x[2 * p + h];
+        }
     }
   }
 }
@@ -293,10 +302,10 @@ static int bc_bt_rw(int b) { return b <= 64 ? 128 : (b <= 128 ? 256 : 512); }
 
 int bc_bt_nb(int b) {
   // window RW = 8*QR rows >= b + nb - 1 (QR = 16 for b <= 64, 32 for b <= 128, 64 for b <= 256); the nb staged
-  // window-shaped vectors (nb x (RW + 16) doubles) fit in 200 KB of shared memory
+  // window-shaped vectors (nb x RW doubles) fit in 200 KB of shared memory
   const int rw = bc_bt_rw(b);
   int nb = rw - b + 1;
-  const int cap = (int)(200 * 1024 / (8 * (size_t)(rw + 16))) - 1;
+  const int cap = (int)(200 * 1024 / (8 * (size_t)rw)) - 1;
   if (nb > cap) nb = cap;
   return nb < 1 ? 1 : nb;
 }
@@ -305,7 +314,7 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
                              double* C, int64_t ldc, cudaStream_t st) {
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
-  const size_t smem = sizeof(double) * ((size_t)nb * (bc_bt_rw(b) + 16) + nb);
+  const size_t smem = sizeof(double) * ((size_t)nb * bc_bt_rw(b) + nb);
   const int64_t grid = (ncols + BT_COLS - 1) / BT_COLS;
   const void* fn = b <= 64 ? (const void*)bc_bt_kernel<16> : (b <= 128 ? (const void*)bc_bt_kernel<32>
                                                                        : (const void*)bc_bt_kernel<64>);
