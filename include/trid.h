@@ -76,7 +76,9 @@ int trid_sytrd_2stage_bufsize(int64_t n, int b, int nb, int k, size_t* dwork_byt
  *      A(c+b+1 : n-1, c) holds the SBR Householder vector of column c (unit entry at row c+b implicit),
  *      tau1[c] its scalar (tau1[c] = 0 for c >= n-b-1).  tau1 has n entries.
  * b  : band width = panel width, 1 <= b <= TRID_MAX_B.
- * nb : inner block of the panel QR (R5), 1 <= nb <= b, b % nb == 0 (performance knob only).
+ * nb : inner block of the panel QR (R5), 1 <= nb <= b, b % nb == 0 (performance knob; same result up to rounding).
+ *      Panels of width b <= 64 are factored whole by the register kernel; wider panels (b % 16 == 0) in blocked form
+ *      with 64-column inner blocks (the register kernel's widest), other b by the general kernel.
  * k  : outer block = syr2k rank, k == 0 -> trid_default_k(n, b); else k >= b, k % b == 0.
  * b >= n-1 is a legal no-op (tau1 = 0).  dwork: trid_sbr_dbbr_bufsize bytes, 256-byte aligned. */
 int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, double* tau1,
@@ -91,7 +93,9 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
  *      S(s) = sum_{s'<s} steps(s'); it acts on rows s+1+m*b .. min(s+(m+1)*b, n-1) (reading R7).
  *      V2 == NULL && tau2 == NULL selects eigenvalues-only mode.
  * Sweeps run concurrently, pipelined at lag 2 by release/acquire progress counters (R9); the result
- * is bitwise identical to the sweep-major order. */
+ * is bitwise identical to the sweep-major order of the same kernel (debug env TRID_BC_SERIAL=1 runs that order;
+ * tests/test_gpu_parity.py::test_bulge_chase_serial_equals_parallel_bitwise).  b <= 64: one CTA per sweep;
+ * 64 < b <= 256: a cluster of 2 (b <= 128) or 4 CTAs per sweep. */
 int trid_bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
                      double* tau2, void* dwork, size_t dwork_bytes, cudaStream_t stream);
 
