@@ -843,14 +843,20 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       const int H = L + L2;
       const int je = cend < L ? cend : L;   // my window columns [cbeg, je)
       const double* gw = a.band + r0 * ldab;   // window column j at gw + j*ldab (rows j.. at offsets 0..)
-      // ---- lag-2 dependency (R9): sweep s-1 has completed step m+1 (serial mode: all of its steps)
+      // ---- dependencies on sweep s-1 (R9, lag 2, refined by column ownership as in bc_v6): window columns
+      // 0 .. L-2 were last written by its step m (prog_full >= m+1), the last column is column 0 of its step m+1
+      // (published early, prog >= m+2).  Serial mode: all of its steps.  The body loads while the last column is
+      // still being produced.
+      const int need_full = (int)(a.serial ? nprev : m + 1);
+      const int need_c0 = (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev);
       if (s > 0) {
-        if (tid == 0) wait_geq(a.prog + (s - 1), (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev));
+        if (tid == 0) wait_geq(a.prog_full + (s - 1), need_full);
         __syncthreads();
       }
       if (a.opt & 64) bw_csync<CS>();   // debug (TRID_BC_OPT): extra cluster barriers
-      // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j)
-      for (int j = cbeg + warp; j < je; j += NW) {
+      // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j); the last one after
+      // its producer published it
+      auto load_col = [&](int j) {
         const int len = H - j, len2 = len >> 1;
         double* dst = win + cofs[j] + j;
         const double* src = gw + (int64_t)j * ldab;
@@ -858,7 +864,14 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(dst + 2 * i)), "l"(src + 2 * i)
                        : "memory");
         if ((len & 1) && lane == 0) dst[len - 1] = __ldcg(src + len - 1);
+      };
+      for (int j = cbeg + warp; j < je && j < L - 1; j += NW) load_col(j);
+      asm volatile("cp.async.commit_group;\n" ::: "memory");
+      if (s > 0 && need_c0 > need_full) {
+        if (tid == 0) wait_geq(a.prog + (s - 1), need_c0);
+        __syncthreads();
       }
+      if (je == L && warp == (L - 1 - cbeg) % NW && L - 1 >= cbeg) load_col(L - 1);
       asm volatile("cp.async.commit_group;\n" ::: "memory");
       // ---- step 0: the reflector annihilating column s below its first subdiagonal (every CTA, same bits)
       if (m == 0) {
@@ -966,6 +979,15 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           }
           __syncthreads();
           for (int i = tid; i < L2; i += BW_NT) c0[L + i] = i == 0 ? scal[4] : 0.0;
+          // window column 0 is final (D(:, 0) after the two-sided update, O(:, 0) = beta e1): store and publish it
+          // now (prog), the next sweep's step m-1 waits only for this column of our step
+          __syncthreads();
+          {
+            double* dst = a.band + r0 * ldab;
+            for (int i = tid; i < H; i += BW_NT) __stcg(dst + i, c0[i]);
+          }
+          __syncthreads();
+          if (tid == 0) st_release_s32(a.prog + s, (int)(m + 1));
         }
         bw_csync<CS>();   // (2) vn and its scalars everywhere
         taun = scal[5];
@@ -986,6 +1008,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       if (a.opt & 256) bw_csync<CS>();
       // ---- store my columns back (one warp per column), the reflector of this step, publish
       for (int j = cbeg + warp; j < je; j += NW) {
+        if (j == 0 && L2 > 0) continue;   // column 0 went out early (step 4)
         const int len = H - j, len2 = len >> 1;
         const double* srcp = win + cofs[j] + j;
         double* dst = a.band + (r0 + j) * ldab;
@@ -1002,7 +1025,8 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       if (q == 0 && tid == 0) {
         // e_s (the rest of column s is dead): written only now, when every CTA of the cluster has read column s
         if (m == 0) __stcg(a.band + s * ldab + 1, scal[1]);
-        st_release_s32(a.prog + s, (int)(m + 1));
+        if (L2 == 0) st_release_s32(a.prog + s, (int)(m + 1));   // no early column-0 publication this step
+        st_release_s32(a.prog_full + s, (int)(m + 1));
       }
       tau = taun;
     }
