@@ -942,27 +942,24 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         const double hp = 0.5 * tau * scal[0];
         for (int i = tid; i < L; i += BW_NT) wv[i] = fma(-hp, v[i], pf[i]);
         __syncthreads();
-        // ---- 3. D -= v w^T + w v^T (lower, my columns), O -= tau y v^T (my columns); one warp per column
-        for (int j = cbeg + warp; j < je; j += NW) {
-          double* col = win + cofs[j];
-          const double vj = v[j], wj = wv[j], tvj = tau * vj;
-          int i = j + lane;
-          for (; i < L; i += 32) col[i] = fma(-wv[i], vj, fma(-v[i], wj, col[i]));
-          for (; i < H; i += 32) col[i] = fma(-pf[i], tvj, col[i]);
-        }
       }
-      // ---- 4. the next reflector from O(:, 0) (window column 0: rank 0), broadcast
+      // ---- 3. the next reflector from x = O(:, 0) - tau y v_0 (O(:, 0) after the right update; window column 0
+      //      belongs to rank 0), broadcast through DSMEM, before any column is updated
       double taun = 0.0;
       if (L2 > 0) {
-        __syncthreads();
         if (q == 0) {
-          double* c0 = win + cofs[0];
+          const double* c0 = win + cofs[0] + L;
+          const double tv0 = tau * v[0];
+          auto xo = [&](int i) { return tau != 0.0 ? fma(-pf[L + i], tv0, c0[i]) : c0[i]; };
           if (warp == 0) {
             double sg = 0.0;
-            for (int i = 1 + lane; i < L2; i += 32) sg = fma(c0[L + i], c0[L + i], sg);
+            for (int i = 1 + lane; i < L2; i += 32) {
+              const double x = xo(i);
+              sg = fma(x, x, sg);
+            }
             sg = warp_sum(sg);
             if (lane == 0) {
-              const House h = make_house(c0[L], sg);
+              const House h = make_house(xo(0), sg);
               for (unsigned r = 0; r < CS; ++r) {
                 bw_st<CS>(scal + 4, r, h.beta);
                 bw_st<CS>(scal + 5, r, h.tau);
@@ -973,34 +970,57 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           __syncthreads();
           const double hs = scal[6];
           for (int i = tid; i < b; i += BW_NT) {
-            const double x = i < L2 ? (i == 0 ? 1.0 : hs * c0[L + i]) : 0.0;
+            const double x = i < L2 ? (i == 0 ? 1.0 : hs * xo(i)) : 0.0;
 #pragma unroll
             for (unsigned r = 0; r < CS; ++r) bw_st<CS>(vn + i, r, x);
           }
-          __syncthreads();
-          for (int i = tid; i < L2; i += BW_NT) c0[L + i] = i == 0 ? scal[4] : 0.0;
-          // window column 0 is final (D(:, 0) after the two-sided update, O(:, 0) = beta e1): store and publish it
-          // now (prog), the next sweep's step m-1 waits only for this column of our step
-          __syncthreads();
-          {
-            double* dst = a.band + r0 * ldab;
-            for (int i = tid; i < H; i += BW_NT) __stcg(dst + i, c0[i]);
-          }
-          __syncthreads();
-          if (tid == 0) st_release_s32(a.prog + s, (int)(m + 1));
         }
         bw_csync<CS>();   // (2) vn and its scalars everywhere
         taun = scal[5];
-        // ---- 5. O(:, j) -= taun vn (vn^T O(:, j)) for my columns j >= 1
-        if (taun != 0.0) {
-          const int j1 = cbeg > 1 ? cbeg : 1;
-          for (int c = j1 + warp; c < je; c += NW) {
-            double* col = win + cofs[c] + L;
-            double acc = 0.0;
-            for (int i = lane; i < L2; i += 32) acc = fma(vn[i], col[i], acc);
-            acc = warp_sum(acc);
-            const double tz = taun * acc;
-            for (int i = lane; i < L2; i += 32) col[i] = fma(-tz, vn[i], col[i]);
+      }
+      // ---- 4. one fused pass per column (one warp per column): D -= v w^T + w v^T (lower); O -= tau y v^T, then
+      //      O(:, j) -= taun vn (vn^T O(:, j)) for j >= 1, O(:, 0) = beta e1.  Window column 0 (rank 0, warp 0,
+      //      first) is final right after its pass: stored and published at once (prog)
+      for (int j = cbeg + warp; j < je; j += NW) {
+        double* col = win + cofs[j];
+        if (tau != 0.0) {
+          const double vj = v[j], wj = wv[j];
+          for (int i = j + lane; i < L; i += 32) col[i] = fma(-wv[i], vj, fma(-v[i], wj, col[i]));
+        }
+        if (L2 > 0) {
+          double* oc = col + L;
+          const double tvj = tau * v[j];
+          constexpr int KO = 8;   // L2 <= b <= 256 rows of O per column: <= 8 per lane
+          double o[KO];
+          double z = 0.0;
+#pragma unroll
+          for (int k = 0; k < KO; ++k) {
+            const int i = lane + 32 * k;
+            o[k] = 0.0;
+            if (i < L2) {
+              o[k] = tau != 0.0 ? fma(-pf[L + i], tvj, oc[i]) : oc[i];
+              z = fma(vn[i], o[k], z);
+            }
+          }
+          if (j == 0) {
+#pragma unroll
+            for (int k = 0; k < KO; ++k) {
+              const int i = lane + 32 * k;
+              if (i < L2) oc[i] = i == 0 ? scal[4] : 0.0;
+            }
+            __syncwarp();
+            double* dst = a.band + r0 * ldab;
+            for (int i = lane; i < H; i += 32) __stcg(dst + i, col[i]);
+            __syncwarp();   // the warp's stores of column 0 are ordered before lane 0's release
+            if (lane == 0) st_release_s32(a.prog + s, (int)(m + 1));
+          } else {
+            z = warp_sum(z);
+            const double tz = taun * z;
+#pragma unroll
+            for (int k = 0; k < KO; ++k) {
+              const int i = lane + 32 * k;
+              if (i < L2) oc[i] = taun != 0.0 ? fma(-tz, vn[i], o[k]) : o[k];
+            }
           }
         }
       }
