@@ -867,12 +867,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       };
       for (int j = cbeg + warp; j < je && j < L - 1; j += NW) load_col(j);
       asm volatile("cp.async.commit_group;\n" ::: "memory");
-      if (s > 0 && need_c0 > need_full) {
-        if (tid == 0) wait_geq(a.prog + (s - 1), need_c0);
-        __syncthreads();
-      }
-      if (je == L && warp == (L - 1 - cbeg) % NW && L - 1 >= cbeg) load_col(L - 1);
-      asm volatile("cp.async.commit_group;\n" ::: "memory");
+      const bool own_last = je == L && L - 1 >= cbeg;   // this CTA holds the window's last column
       // ---- step 0: the reflector annihilating column s below its first subdiagonal (every CTA, same bits)
       if (m == 0) {
         for (int i = tid; i < L; i += BW_NT) colv[i] = __ldcg(a.band + s * ldab + 1 + i);
@@ -892,10 +887,11 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         for (int i = tid; i < b; i += BW_NT) v[i] = i == 0 ? 1.0 : (i < L ? scal[3] * colv[i] : 0.0);
         tau = scal[2];
       }
-      asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+      asm volatile("cp.async.wait_group 0;\n" ::: "memory");   // the body columns
       __syncthreads();
       if (a.opt & 128) bw_csync<CS>();
-      // ---- 1. partial matvec [D; O] v over my columns, all H rows
+      // ---- 1. partial matvec [D; O] v over my BODY columns (all but the window's last, which sweep s-1 may still
+      //      be producing), all H rows; the last column's terms are added once it arrives
       if (tau != 0.0) {
         {
           const int i = tid % H2, h = tid / H2;   // row i, half h (tpr == 2) of my columns
@@ -905,6 +901,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
               const int jlo = tpr == 2 ? (h ? jmid : cbeg) : cbeg;
               int jhi = tpr == 2 ? (h ? je : (jmid < je ? jmid : je)) : je;
               if (jhi > i + 1) jhi = i + 1;   // lower part of D (and all of O): columns j <= i
+              if (jhi > L - 1) jhi = L - 1;   // body only
               for (int j = jlo; j < jhi; ++j) acc = fma(win[cofs[j] + i], v[j], acc);
             }
             prt[h * H2 + i] = acc;
@@ -921,6 +918,22 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           for (int j = c + 1 + lane; j < L; j += 32) acc = fma(col[j], v[j], acc);
           acc = warp_sum(acc);
           if (lane == 0) prt[c] += acc;
+        }
+      }
+      // ---- the last column = column 0 of sweep s-1's step m+1: wait for its early publication, load, add its terms
+      //      D(L-1, L-1) v_{L-1} and O(:, L-1) v_{L-1} (fixed order: after the body and the mirror)
+      if (s > 0 && need_c0 > need_full) {
+        if (tid == 0) wait_geq(a.prog + (s - 1), need_c0);
+        __syncthreads();
+      }
+      if (own_last && warp == (L - 1 - cbeg) % NW) load_col(L - 1);
+      asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+      __syncthreads();
+      if (tau != 0.0) {
+        if (own_last) {
+          const double vl = v[L - 1];
+          const double* cl = win + cofs[L - 1];
+          for (int i = L - 1 + tid; i < H; i += BW_NT) prt[i] = fma(cl[i], vl, prt[i]);
         }
         bw_csync<CS>();   // (1) partials of every CTA complete
         // ---- 2. p = tau D v, y = O v: the CS partials summed in rank order
