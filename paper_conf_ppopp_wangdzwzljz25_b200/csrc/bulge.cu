@@ -751,9 +751,9 @@ __global__ void __launch_bounds__(NTH + 96, 1) bc_v6_kernel(BcArgs a) {
 // 197 KB even when only its stored part is kept, at b = 256 it is 788 KB.  Here a step's window lives in shared
 // memory as a TRAPEZOID: window column j holds only its rows j .. 2b-1 (the lower triangle of D and the whole
 // bulge block O), 2b - j doubles rounded up to even, packed one after the other (16-byte aligned columns, loaded and
-// stored with 16-byte cp.async / st.global.cg by all threads).  The window is split by columns over a cluster of
-// CS CTAs (CS = 2 for b <= 128, 4 beyond; balanced by stored size, <= 197 KB each) that cooperate on one sweep
-// through DSMEM:
+// stored with 16-byte cp.async / st.global.cg by all threads).  For b <= 128 one CTA holds the whole trapezoid
+// (197 KB at b = 128); beyond, the window is split by columns over a cluster of CS = 4 CTAs (balanced by stored size,
+// <= 197 KB each) that cooperate on one sweep through DSMEM:
 //   1. every CTA forms the partial matvec [D; O] v over its columns for all 2b rows (the lower part of D row-wise,
 //      the mirrored upper part as a column dot, both from its own columns), writes it to shared memory;
 //   2. cluster barrier; every CTA sums the CS partials in rank order (DSMEM loads): identical p = tau D v, y = O v;
@@ -1183,9 +1183,10 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
       }
     } else {
       // 64 < b <= 256: bc_wide_kernel, a cluster of CS CTAs per sweep
-      // cluster split: 2 CTAs per sweep for b <= 128 (measured at n = 32768, b = 128: 1588 / 1224 / 1497 ms for
-      // CS = 1 / 2 / 4 -- the chase is chain-bound there, so a shorter step beats more concurrent sweeps), 4 beyond
-      int CS = beff <= 128 ? 2 : 4;
+      // cluster split: one CTA per sweep for b <= 128 (the whole trapezoid fits), 4 beyond.  Measured at n = 32768,
+      // b = 128 with the early column-0 hand-off: CS = 1 994 ms, CS = 2 1092-1165 ms (the cluster barriers of a
+      // step cost more than the halved step work saves), profiles/r02_bc_wide_cluster_split_ab.jsonl
+      int CS = beff <= 128 ? 1 : 4;
       {
         const char* ce = getenv("TRID_BC_WCS");   // debug/A-B: force the cluster split (1, 2 or 4)
         if (ce && (atoi(ce) == 1 || atoi(ce) == 2 || atoi(ce) == 4)) CS = atoi(ce);
