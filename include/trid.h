@@ -95,7 +95,7 @@ int trid_sbr_dbbr(int64_t n, double* A, int64_t lda, int b, int nb, int k, doubl
  * Sweeps run concurrently, pipelined at lag 2 by release/acquire progress counters (R9); the result
  * is bitwise identical to the sweep-major order of the same kernel (debug env TRID_BC_SERIAL=1 runs that order;
  * tests/test_gpu_parity.py::test_bulge_chase_serial_equals_parallel_bitwise).  b <= 64: one CTA per sweep;
- * 64 < b <= 256: a cluster of 2 (b <= 128) or 4 CTAs per sweep. */
+ * 64 < b <= 128: one CTA per sweep (trapezoid window in shared memory), 128 < b <= 256: a cluster of 4. */
 int trid_bulge_chase(int64_t n, int b, const double* A, int64_t lda, double* d, double* e, double* V2,
                      double* tau2, void* dwork, size_t dwork_bytes, cudaStream_t stream);
 
