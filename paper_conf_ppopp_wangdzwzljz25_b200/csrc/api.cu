@@ -160,7 +160,18 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
     g.C = U; g.ldc = ldu; g.alpha = 1.0; g.beta = 0.0;
     g.splits = pick_splits(2 * nprev, kk, m, TILE_64x64, part_elems);
     g.part = part; g.part_ld = 2 * nprev; g.part_stride = 2 * nprev * kk;
-    if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
+    static const bool u_ws = !(getenv("TRID_ZY_WS") && getenv("TRID_ZY_WS")[0] == '0');
+    if (u_ws) {
+      // the two stacked TN products on the warp-specialized engine (op(A) = A^T), one launch per operand
+      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, 1.0, Zprev, ldyz, Wp, ldw, 0.0, U1, ldu, part, part_elems, st)) !=
+          cudaSuccess)
+        return e;
+      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, 1.0, Yprev, ldyz, Wp, ldw, 0.0, U2, ldu, part, part_elems, st)) !=
+          cudaSuccess)
+        return e;
+    } else if ((e = gemm(g, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) {
+      return e;
+    }
     // X -= Y_< U1 + Z_< U2
     GemmArgs h;
     h.M = m; h.N = kk; h.nseg = 2;
@@ -184,7 +195,13 @@ cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const doub
   s.splits = pick_splits(kk, kk, m, TILE_64x64, part_elems);
   s.part = part; s.part_ld = kk; s.part_stride = (int64_t)kk * kk;
   (void)sem;   // in-kernel last-split reduction measured slower here (serial tail per tile); kept off
-  if ((e = gemm(s, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) return e;
+  static const bool s_ws = getenv("TRID_ZY_WS") && getenv("TRID_ZY_WS")[0] == '2';
+  if (s_ws) {
+    if ((e = gemm_ws_mm(OP_T, OP_N, kk, kk, m, 1.0, Wp, ldw, X, ldx, 0.0, S, lds, part, part_elems, st)) != cudaSuccess)
+      return e;
+  } else if ((e = gemm(s, OP_T, OP_N, TILE_64x64, st)) != cudaSuccess) {
+    return e;
+  }
   // Z_p = X - 1/2 Y_p S
   GemmArgs z;
   z.M = m; z.N = kk; z.K[0] = kk; z.A[0] = Yp; z.lda[0] = ldyz; z.B[0] = S; z.ldb[0] = lds;
