@@ -221,19 +221,34 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
     double tw[CPW];   // -tau * w_j for this warp's columns (w_j = v^T P(:, j))
 #pragma unroll
     for (int c = 0; c < CPW; ++c) tw[c] = -h.tau * fma(h.scale, tot[j0 + c], tot[W + j0 + c]);
+    if (j0 > t) {
+      // every column of this warp lies right of t (the common case): a predicate-free rank-1 update of the rows >= t
 #pragma unroll
-    for (int q = 0; q < PR_RL; ++q) {
-      const int i = lane + 32 * q;
-      const int64_t r = rlo + i;
-      if (i >= nr || r < t) continue;
-      const double vr = r > t ? h.scale * xs[i] : 1.0;
+      for (int q = 0; q < PR_RL; ++q) {
+        const int i = lane + 32 * q;
+        const int64_t r = rlo + i;
+        if (i < nr && r >= t) {
+          const double vr = r > t ? h.scale * xs[i] : 1.0;
 #pragma unroll
-      for (int c = 0; c < CPW; ++c) {
-        const int j = j0 + c;
-        if (j > t) {
-          P[q][c] = fma(tw[c], vr, P[q][c]);
-        } else if (j == t) {
-          P[q][c] = r > t ? vr : h.beta;
+          for (int c = 0; c < CPW; ++c) P[q][c] = fma(tw[c], vr, P[q][c]);
+        }
+      }
+    } else if (j0 + CPW > t) {
+      // the warp holding column t: v (or beta) into column t, the update right of it, nothing left of it
+#pragma unroll
+      for (int q = 0; q < PR_RL; ++q) {
+        const int i = lane + 32 * q;
+        const int64_t r = rlo + i;
+        if (i >= nr || r < t) continue;
+        const double vr = r > t ? h.scale * xs[i] : 1.0;
+#pragma unroll
+        for (int c = 0; c < CPW; ++c) {
+          const int j = j0 + c;
+          if (j > t) {
+            P[q][c] = fma(tw[c], vr, P[q][c]);
+          } else if (j == t) {
+            P[q][c] = r > t ? vr : h.beta;
+          }
         }
       }
     }
