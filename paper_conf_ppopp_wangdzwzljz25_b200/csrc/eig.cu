@@ -9,18 +9,21 @@
 // limit of bisection on [gl, gu] (Gershgorin bounds widened by 2 eps |.| + 2 pivmin) keeping count(lo) <= k <
 // count(hi), stopped when hi - lo <= 2 eps max(|lo|, |hi|) + pivmin.
 //
-// B200 design: the count is a sequential recurrence with one IEEE division per element, so the kernel is
-// latency-bound per eigenvalue and throughput-bound over all of them: ONE thread per eigenvalue, every thread
-// of a CTA walks the same d_i / e_i^2 in lockstep out of a shared-memory tile (one global read per element per
-// CTA instead of per thread), 128 threads per CTA so n = 32768 fills 256 CTAs (1.7 per SM).  The bounds come
-// from one small reduction kernel (min/max are exact, so the order does not matter).  Every operation is the
-// plain expression above in the same order with IEEE division (no FMA can contract it): the results equal a
-// serial implementation of the same definition bit for bit.
+// B200 design: the count is a sequential recurrence with one IEEE division per element, so one bisection step is
+// a long latency-bound chain.  A group of G = 2^P lanes per eigenvalue (G chosen so n G fills ~2048 threads per SM,
+// at most a warp) runs an EXACT multisection: in one pass it counts at the 2^P - 1 nodes of the depth-P bisection
+// subtree below the current interval (each node value built by the same halvings the serial loop performs), then
+// walks P levels with the serial loop's tests -- the serial bisection, P steps per dependent recurrence.  Every
+// thread of a CTA walks the same d_i / e_i^2 in lockstep out of a shared-memory tile.  The bounds come from one
+// small reduction kernel (min/max are exact, so the order does not matter).  Every operation is the plain
+// expression above in the same order with IEEE division (no FMA can contract it): the results equal a serial
+// implementation of the same definition bit for bit (TRID_STEBZ_P=0 runs the one-thread-per-eigenvalue loop).
 #include "common.cuh"
 #include "eig.cuh"
 #include "prof.cuh"
 
 #include <float.h>
+#include <stdlib.h>
 
 namespace trid {
 
@@ -136,6 +139,104 @@ __global__ void __launch_bounds__(EIG_NT) sturm_bisect_kernel(int64_t n, const d
   if (k < n) w[k] = 0.5 * (lo + hi);
 }
 
+// Exact multisection: a group of G = 2^P lanes per eigenvalue evaluates, in one pass, the Sturm counts at all
+// 2^P - 1 midpoints of the depth-P bisection subtree below the current interval (lane l >= 1 = heap node l; each node
+// value is obtained by the same halvings 0.5 (lo + hi) the serial bisection performs along that path), then every
+// lane walks the P levels with the serial loop's termination tests, taking each level's count from the node's lane.
+// The walk visits exactly the serial bisection's midpoints, so the result is the serial result bit for bit, in
+// ceil(steps / P) dependent recurrences instead of `steps` (the count is a latency-bound chain of divisions).
+template <int P>
+__global__ void __launch_bounds__(EIG_NT) sturm_msect_kernel(int64_t n, const double* __restrict__ d,
+                                                            const double* __restrict__ e2,
+                                                            const double* __restrict__ bounds, double* w) {
+  constexpr int G = 1 << P;
+  __shared__ double sd[EIG_TILE], se[EIG_TILE];
+  __shared__ int s_active;
+  const int lane = threadIdx.x & 31, gl = threadIdx.x & (G - 1);
+  const int gbase = lane & ~(G - 1);
+  const int64_t k = ((int64_t)blockIdx.x * EIG_NT + threadIdx.x) / G;
+  const double pivmin = bounds[2];
+  double lo = bounds[0], hi = bounds[1];
+  bool active = k < n;
+  int it = 0;   // serial bisection steps taken (the serial loop stops after 256)
+  for (;;) {
+    if (threadIdx.x == 0) s_active = 0;
+    __syncthreads();
+    if (active) s_active = 1;
+    __syncthreads();
+    if (!s_active) break;
+    // this lane's node of the subtree
+    double mid = 0.0;
+    const bool node = active && gl >= 1;
+    if (node) {
+      double nl = lo, nh = hi;
+      const int depth = 31 - __clz(gl);
+      for (int dd = depth - 1; dd >= 0; --dd) {
+        const double m2 = 0.5 * (nl + nh);
+        if ((gl >> dd) & 1) nl = m2;
+        else nh = m2;
+      }
+      mid = 0.5 * (nl + nh);
+    }
+    // Sturm count of T - mid I
+    int64_t cnt = 0;
+    double q = 1.0;
+    for (int64_t t0 = 0; t0 < n; t0 += EIG_TILE) {
+      const int len = (int)((n - t0) < EIG_TILE ? (n - t0) : EIG_TILE);
+      __syncthreads();
+      for (int i = threadIdx.x; i < len; i += EIG_NT) {
+        sd[i] = d[t0 + i];
+        se[i] = (t0 + i > 0) ? e2[t0 + i - 1] : 0.0;
+      }
+      __syncthreads();
+      if (node) {
+        int i = 0;
+        if (t0 == 0) {
+          q = sd[0] - mid;
+          if (fabs(q) < pivmin) q = -pivmin;
+          if (q < 0) ++cnt;
+          i = 1;
+        }
+        for (; i < len; ++i) {
+          q = sd[i] - mid - se[i] / q;
+          if (fabs(q) < pivmin) q = -pivmin;
+          if (q < 0) ++cnt;
+        }
+      }
+    }
+    // walk the P levels exactly as the serial loop (every lane of the warp takes part in the shuffles)
+    int nd = 1;
+    for (int dd = 0; dd < P; ++dd) {
+      bool go = active && it < 256;
+      double m = 0.0;
+      if (go) {
+        const double tol = 2.0 * DBL_EPSILON * (fabs(lo) > fabs(hi) ? fabs(lo) : fabs(hi)) + pivmin;
+        if (hi - lo <= tol) {
+          go = false;
+        } else {
+          m = 0.5 * (lo + hi);
+          if (m <= lo || m >= hi) go = false;
+        }
+      }
+      const long long c = __shfl_sync(0xffffffffu, (long long)cnt, gbase + (nd < G ? nd : 0));
+      if (go) {
+        ++it;
+        if (c > k) {
+          hi = m;
+          nd = 2 * nd;
+        } else {
+          lo = m;
+          nd = 2 * nd + 1;
+        }
+      } else {
+        active = false;
+      }
+    }
+    if (it >= 256) active = false;
+  }
+  if (gl == 0 && k < n) w[k] = 0.5 * (lo + hi);
+}
+
 size_t stebz_work_bytes(int64_t n) {
   return ((sizeof(double) * (size_t)(n > 1 ? n - 1 : 1) + 255) / 256) * 256 + 256;
 }
@@ -152,8 +253,25 @@ cudaError_t stebz(int64_t n, const double* d, const double* e, double* w, void* 
   }
   sturm_bounds_kernel<<<1, 1024, 0, st>>>(n, d, e, bounds);
   count_launches(1);
-  const int64_t grid = (n + EIG_NT - 1) / EIG_NT;
-  sturm_bisect_kernel<<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w);
+  // lanes per eigenvalue: fill ~2 x 1024 threads per SM (latency-bound chains), at most a warp
+  int64_t g = (int64_t)num_sms() * 2048 / (n > 0 ? n : 1);
+  int P = 0;
+  while (P < 5 && ((int64_t)1 << (P + 1)) <= g) ++P;
+  static const char* me = getenv("TRID_STEBZ_P");   // A/B: force the multisection depth (0 = plain bisection)
+  if (me) P = atoi(me) < 0 ? 0 : (atoi(me) > 5 ? 5 : atoi(me));
+  if (P == 0) {
+    const int64_t grid = (n + EIG_NT - 1) / EIG_NT;
+    sturm_bisect_kernel<<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w);
+  } else {
+    const int64_t grid = ((n << P) + EIG_NT - 1) / EIG_NT;
+    switch (P) {
+      case 1: sturm_msect_kernel<1><<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w); break;
+      case 2: sturm_msect_kernel<2><<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w); break;
+      case 3: sturm_msect_kernel<3><<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w); break;
+      case 4: sturm_msect_kernel<4><<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w); break;
+      default: sturm_msect_kernel<5><<<(unsigned)grid, EIG_NT, 0, st>>>(n, d, e2, bounds, w); break;
+    }
+  }
   count_launches(1);
   return cudaGetLastError();
 }
