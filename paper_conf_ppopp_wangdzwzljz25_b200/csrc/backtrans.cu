@@ -207,25 +207,30 @@ __host__ __device__ inline int64_t bt_offset(int64_t n, int b, int64_t s) {   //
   return bt_F(n - 3, b) - bt_F(n - 3 - s, b);
 }
 
-constexpr int BT_COLS = 32;   // columns of C per CTA (8 warps x 4)
 constexpr int BT_NT = 256;
 
 // QR rows per thread; the group window holds 8*QR >= b + nb - 1 rows.
-template <int QR>
+template <int QR, int CC>
 __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int nb, const double* __restrict__ V2,
                                                         const double* __restrict__ tau2, int trans, int64_t ncols,
                                                         double* C, int64_t ldc) {
   constexpr int RW = 8 * QR;   // window rows
   constexpr int NP = QR / 2;   // row pairs per thread: thread (rg, cl) holds rows 16 p + 2 rg + {0, 1}, p < NP, of
-                               // column cl -- the 8 row-group lanes of a column cover 16 consecutive rows (coalesced)
+                               // its CC columns -- the 8 row-group lanes of a column cover 16 consecutive rows
+  constexpr int COLS = 32 * CC;   // columns per CTA: 8 warps x 4 column lanes x CC columns per thread
   // the group's reflectors in window shape: Vw[j][r] = v_j[r - j] (zero outside [0, b)), nb x RW; then nb taus
   extern __shared__ __align__(16) double sv[];
   double* stau = sv + (size_t)nb * RW;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rg = lane >> 2, cl = lane & 3;
-  const int64_t col = (int64_t)blockIdx.x * BT_COLS + warp * 4 + cl;
-  const bool colok = col < ncols;
-  double* Cc = C + (colok ? col : 0) * ldc;
+  double* Cc[CC];
+  bool colok[CC];
+#pragma unroll
+  for (int u = 0; u < CC; ++u) {
+    const int64_t col = (int64_t)blockIdx.x * COLS + (warp * 4 + cl) * CC + u;
+    colok[u] = col < ncols;
+    Cc[u] = C + (colok[u] ? col : 0) * ldc;
+  }
   const int64_t nsw = n - 2;   // sweeps 0 .. n-3
   const int64_t nblk = (nsw + nb - 1) / nb;
   constexpr int NWB = BT_NT / 32;
@@ -251,15 +256,17 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         if (lane == 0) stau[j] = ex ? tau2[bt_offset(n, b, s) + m] : 0.0;
       }
       __syncthreads();
-      // the window rows of this thread: w0 + 16 p + 2 rg + h
-      double x[QR];
+      // the window rows of this thread: w0 + 16 p + 2 rg + h, for each of its CC columns
+      double x[CC][QR];
 #pragma unroll
-      for (int p = 0; p < NP; ++p)
+      for (int u = 0; u < CC; ++u)
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int64_t r = w0 + 16 * p + 2 * rg + h;
-          x[2 * p + h] = (colok && r < n) ? Cc[r] : 0.0;
-        }
+        for (int p = 0; p < NP; ++p)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int64_t r = w0 + 16 * p + 2 * rg + h;
+            x[u][2 * p + h] = (colok[u] && r < n) ? Cc[u][r] : 0.0;
+          }
       // G_m C applies H_{s0+nbb-1,m} first;  G_m^T C applies H_{s0,m} first
       for (int jj = 0; jj < nbb; ++jj) {
         const int j = trans ? jj : nbb - 1 - jj;
@@ -273,27 +280,39 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
           vv[2 * p] = t.x;
           vv[2 * p + 1] = t.y;
         }
-        double d0 = 0.0, d1 = 0.0;
+        double d[CC];
 #pragma unroll
-        for (int p = 0; p < NP; ++p) {
-          d0 = fma(vv[2 * p], x[2 * p], d0);
-          d1 = fma(vv[2 * p + 1], x[2 * p + 1], d1);
+        for (int u = 0; u < CC; ++u) {
+          double d0 = 0.0, d1 = 0.0;
+#pragma unroll
+          for (int p = 0; p < NP; ++p) {
+            d0 = fma(vv[2 * p], x[u][2 * p], d0);
+            d1 = fma(vv[2 * p + 1], x[u][2 * p + 1], d1);
+          }
+          d[u] = d0 + d1;
         }
-        double d = d0 + d1;
-        d += __shfl_xor_sync(0xffffffffu, d, 4);
-        d += __shfl_xor_sync(0xffffffffu, d, 8);
-        d += __shfl_xor_sync(0xffffffffu, d, 16);
-        const double td = tau * d;
 #pragma unroll
-        for (int q = 0; q < QR; ++q) x[q] = fma(-td, vv[q], x[q]);
+        for (int u = 0; u < CC; ++u) d[u] += __shfl_xor_sync(0xffffffffu, d[u], 4);
+#pragma unroll
+        for (int u = 0; u < CC; ++u) d[u] += __shfl_xor_sync(0xffffffffu, d[u], 8);
+#pragma unroll
+        for (int u = 0; u < CC; ++u) d[u] += __shfl_xor_sync(0xffffffffu, d[u], 16);
+#pragma unroll
+        for (int u = 0; u < CC; ++u) {
+          const double td = tau * d[u];
+#pragma unroll
+          for (int q = 0; q < QR; ++q) x[u][q] = fma(-td, vv[q], x[u][q]);
+        }
       }
 #pragma unroll
-      for (int p = 0; p < NP; ++p)
+      for (int u = 0; u < CC; ++u)
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int64_t r = w0 + 16 * p + 2 * rg + h;
-          if (colok && r < n) Cc[r] = x[2 * p + h];
-        }
+        for (int p = 0; p < NP; ++p)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int64_t r = w0 + 16 * p + 2 * rg + h;
+            if (colok[u] && r < n) Cc[u][r] = x[u][2 * p + h];
+          }
     }
   }
 }
@@ -315,18 +334,28 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
   const size_t smem = sizeof(double) * ((size_t)nb * bc_bt_rw(b) + nb);
-  const int64_t grid = (ncols + BT_COLS - 1) / BT_COLS;
-  const void* fn = b <= 64 ? (const void*)bc_bt_kernel<16> : (b <= 128 ? (const void*)bc_bt_kernel<32>
-                                                                       : (const void*)bc_bt_kernel<64>);
-  static DeviceOnce attr16, attr32, attr64;
-  DeviceOnce& at = b <= 64 ? attr16 : (b <= 128 ? attr32 : attr64);
+  // two columns per thread (two independent reflector chains per warp) when that still gives every SM a CTA;
+  // b > 64 keeps one (register budget of the 32/64-row windows)
+  static const char* ce = getenv("TRID_BT_CC");   // A/B
+  int cc = (b <= 64 && (ncols + 63) / 64 >= num_sms()) ? 2 : 1;
+  if (ce) cc = atoi(ce) == 2 && b <= 64 ? 2 : 1;
+  const int64_t grid = (ncols + 32 * cc - 1) / (32 * cc);
+  const void* fn = b <= 64 ? (cc == 2 ? (const void*)bc_bt_kernel<16, 2> : (const void*)bc_bt_kernel<16, 1>)
+                           : (b <= 128 ? (const void*)bc_bt_kernel<32, 1> : (const void*)bc_bt_kernel<64, 1>);
+  static DeviceOnce attr16, attr16b, attr32, attr64;
+  DeviceOnce& at = b <= 64 ? (cc == 2 ? attr16b : attr16) : (b <= 128 ? attr32 : attr64);
   cudaError_t e = at([&] {
     return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   });
   if (e != cudaSuccess) return e;
-  if (b <= 64) bc_bt_kernel<16><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
-  else if (b <= 128) bc_bt_kernel<32><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
-  else bc_bt_kernel<64><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  if (b <= 64 && cc == 2)
+    bc_bt_kernel<16, 2><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (b <= 64)
+    bc_bt_kernel<16, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (b <= 128)
+    bc_bt_kernel<32, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else
+    bc_bt_kernel<64, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
   count_launches(1);
   return cudaGetLastError();
 }
