@@ -334,11 +334,10 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
   const size_t smem = sizeof(double) * ((size_t)nb * bc_bt_rw(b) + nb);
-  // two columns per thread (two independent reflector chains per warp) when that still gives every SM a CTA;
-  // b > 64 keeps one (register budget of the 32/64-row windows)
-  static const char* ce = getenv("TRID_BT_CC");   // A/B
-  int cc = (b <= 64 && (ncols + 63) / 64 >= num_sms()) ? 2 : 1;
-  if (ce) cc = atoi(ce) == 2 && b <= 64 ? 2 : 1;
+  // one column per thread; TRID_BT_CC=2 (A/B, b <= 64) gives each thread two columns -- two independent reflector
+  // chains per warp -- measured slower at n = 8192 (345 vs 317 ms: half the CTAs, same per-reflector latency)
+  static const char* ce = getenv("TRID_BT_CC");
+  const int cc = (ce && atoi(ce) == 2 && b <= 64) ? 2 : 1;
   const int64_t grid = (ncols + 32 * cc - 1) / (32 * cc);
   const void* fn = b <= 64 ? (cc == 2 ? (const void*)bc_bt_kernel<16, 2> : (const void*)bc_bt_kernel<16, 1>)
                            : (b <= 128 ? (const void*)bc_bt_kernel<32, 1> : (const void*)bc_bt_kernel<64, 1>);
