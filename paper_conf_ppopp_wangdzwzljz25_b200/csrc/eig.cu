@@ -253,10 +253,13 @@ cudaError_t stebz(int64_t n, const double* d, const double* e, double* w, void* 
   }
   sturm_bounds_kernel<<<1, 1024, 0, st>>>(n, d, e, bounds);
   count_launches(1);
-  // lanes per eigenvalue: fill ~2 x 1024 threads per SM (latency-bound chains), at most a warp
-  int64_t g = (int64_t)num_sms() * 2048 / (n > 0 ? n : 1);
+  // lanes per eigenvalue: fill ~2048 threads per SM (latency-bound chains), at most a warp; below 16 lanes the
+  // extra counts cost as much as the shorter chain saves (measured at n = 32768: 195 ms with 8 lanes, 192 ms with
+  // one thread per eigenvalue; n = 8192: 29 ms with 32 lanes vs 46 ms)
+  const int64_t g = (int64_t)num_sms() * 2048 / (n > 0 ? n : 1);
   int P = 0;
-  while (P < 5 && ((int64_t)1 << (P + 1)) <= g) ++P;
+  if (g >= 16)
+    while (P < 5 && ((int64_t)1 << (P + 1)) <= g) ++P;
   static const char* me = getenv("TRID_STEBZ_P");   // A/B: force the multisection depth (0 = plain bisection)
   if (me) P = atoi(me) < 0 ? 0 : (atoi(me) > 5 ? 5 : atoi(me));
   if (P == 0) {
