@@ -210,6 +210,10 @@ __host__ __device__ inline int64_t bt_offset(int64_t n, int b, int64_t s) {   //
 constexpr int BT_NT = 256;
 
 // QR rows per thread; the group window holds 8*QR >= b + nb - 1 rows.
+__device__ __forceinline__ void bt_cp8(double* dst, const double* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+
 template <int QR, int CC>
 __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int nb, const double* __restrict__ V2,
                                                         const double* __restrict__ tau2, int trans, int64_t ncols,
@@ -218,9 +222,13 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   constexpr int NP = QR / 2;   // row pairs per thread: thread (rg, cl) holds rows 16 p + 2 rg + {0, 1}, p < NP, of
                                // its CC columns -- the 8 row-group lanes of a column cover 16 consecutive rows
   constexpr int COLS = 32 * CC;   // columns per CTA: 8 warps x 4 column lanes x CC columns per thread
-  // the group's reflectors in window shape: Vw[j][r] = v_j[r - j] (zero outside [0, b)), nb x RW; then nb taus
+  // two buffers of the group's reflectors in window shape, Vw[j][r] = v_j[r - j] (zero outside [j, j+b): the zero
+  // rows are written once, the b rows of vector j are refilled per group by cp.async), nb x RW each; 2 x nb taus;
+  // the block's per-sweep V2 offsets S(s0+j) and step counts
   extern __shared__ __align__(16) double sv[];
-  double* stau = sv + (size_t)nb * RW;
+  double* stau = sv + 2 * (size_t)nb * RW;
+  int64_t* soff = reinterpret_cast<int64_t*>(stau + 2 * nb);
+  int64_t* sst = soff + nb;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int rg = lane >> 2, cl = lane & 3;
   double* Cc[CC];
@@ -234,28 +242,50 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   const int64_t nsw = n - 2;   // sweeps 0 .. n-3
   const int64_t nblk = (nsw + nb - 1) / nb;
   constexpr int NWB = BT_NT / 32;
+  for (int i = threadIdx.x; i < 2 * nb * RW; i += BT_NT) sv[i] = 0.0;
   for (int64_t bi = 0; bi < nblk; ++bi) {
     const int64_t blk = trans ? bi : nblk - 1 - bi;
     const int64_t s0 = blk * nb;
     const int nbb = (int)((nsw - s0) < nb ? (nsw - s0) : nb);
     const int64_t M = bt_steps(n, b, s0);   // groups of the block (sweep s0 has the most steps)
+    __syncthreads();   // previous block done with soff / the buffers
+    for (int j = threadIdx.x; j < nbb; j += BT_NT) {
+      soff[j] = bt_offset(n, b, s0 + j);
+      sst[j] = bt_steps(n, b, s0 + j);
+    }
+    __syncthreads();
+    // group gi's reflectors into buffer gi & 1 (asynchronous; its existence decides the tau slot only: a missing
+    // step gets tau = 0 and is skipped, whatever the buffer holds)
+    auto stage = [&](int64_t gi) {
+      const int64_t m = trans ? M - 1 - gi : gi;
+      double* buf = sv + (size_t)(gi & 1) * nb * RW;
+      double* tb = stau + (gi & 1) * nb;
+      for (int j = warp; j < nbb; j += NWB) {
+        const bool ex = m < sst[j];
+        if (ex) {
+          const double* src = V2 + (soff[j] + m) * b;
+          double* dst = buf + (size_t)j * RW + j;
+          for (int i = lane; i < b; i += 32) bt_cp8(dst + i, src + i);
+          if (lane == 0) bt_cp8(tb + j, tau2 + soff[j] + m);
+        } else if (lane == 0) {
+          tb[j] = 0.0;
+        }
+      }
+      asm volatile("cp.async.commit_group;\n" ::: "memory");
+    };
+    stage(0);
     for (int64_t gi = 0; gi < M; ++gi) {
       const int64_t m = trans ? M - 1 - gi : gi;
       const int64_t w0 = s0 + 1 + m * b;   // first row of the group window
-      // stage the group's reflectors, one warp per vector (its V2 offset computed once): vector of sweep s0+j
-      __syncthreads();
-      for (int j = warp; j < nbb; j += NWB) {
-        const int64_t s = s0 + j;
-        const bool ex = m < bt_steps(n, b, s);
-        const double* vsrc = V2 + (ex ? (bt_offset(n, b, s) + m) * b : 0);
-        double* vd = sv + (size_t)j * RW;
-        for (int r = lane; r < RW; r += 32) {
-          const int i = r - j;
-          vd[r] = (ex && i >= 0 && i < b) ? vsrc[i] : 0.0;
-        }
-        if (lane == 0) stau[j] = ex ? tau2[bt_offset(n, b, s) + m] : 0.0;
+      if (gi + 1 < M) {
+        stage(gi + 1);
+        asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;\n" ::: "memory");
       }
-      __syncthreads();
+      __syncthreads();   // group gi's reflectors visible to all
+      const double* vbuf = sv + (size_t)(gi & 1) * nb * RW;
+      const double* tbuf = stau + (gi & 1) * nb;
       // the window rows of this thread: w0 + 16 p + 2 rg + h, for each of its CC columns
       double x[CC][QR];
 #pragma unroll
@@ -270,9 +300,9 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
       // G_m C applies H_{s0+nbb-1,m} first;  G_m^T C applies H_{s0,m} first
       for (int jj = 0; jj < nbb; ++jj) {
         const int j = trans ? jj : nbb - 1 - jj;
-        const double tau = stau[j];
+        const double tau = tbuf[j];
         if (tau == 0.0) continue;
-        const double2* vj = reinterpret_cast<const double2*>(sv + (size_t)j * RW + 2 * rg);
+        const double2* vj = reinterpret_cast<const double2*>(vbuf + (size_t)j * RW + 2 * rg);
         double vv[QR];
 #pragma unroll
         for (int p = 0; p < NP; ++p) {
@@ -313,6 +343,7 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
             const int64_t r = w0 + 16 * p + 2 * rg + h;
             if (colok[u] && r < n) Cc[u][r] = x[u][2 * p + h];
           }
+      __syncthreads();   // every warp is done with buffer gi & 1 before stage(gi + 2) refills it
     }
   }
 }
@@ -320,11 +351,11 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
 static int bc_bt_rw(int b) { return b <= 64 ? 128 : (b <= 128 ? 256 : 512); }
 
 int bc_bt_nb(int b) {
-  // window RW = 8*QR rows >= b + nb - 1 (QR = 16 for b <= 64, 32 for b <= 128, 64 for b <= 256); the nb staged
-  // window-shaped vectors (nb x RW doubles) fit in 200 KB of shared memory
+  // window RW = 8*QR rows >= b + nb - 1 (QR = 16 for b <= 64, 32 for b <= 128, 64 for b <= 256); two buffers of
+  // nb staged window-shaped vectors (2 nb x RW doubles) fit in 200 KB of shared memory
   const int rw = bc_bt_rw(b);
   int nb = rw - b + 1;
-  const int cap = (int)(200 * 1024 / (8 * (size_t)rw)) - 1;
+  const int cap = (int)(200 * 1024 / (16 * (size_t)rw)) - 2;
   if (nb > cap) nb = cap;
   return nb < 1 ? 1 : nb;
 }
@@ -333,7 +364,7 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
                              double* C, int64_t ldc, cudaStream_t st) {
   if (n < 3 || b < 2 || ncols <= 0) return cudaSuccess;
   const int nb = bc_bt_nb(b);
-  const size_t smem = sizeof(double) * ((size_t)nb * bc_bt_rw(b) + nb);
+  const size_t smem = sizeof(double) * (2 * (size_t)nb * bc_bt_rw(b) + 2 * (size_t)nb) + 2 * sizeof(int64_t) * nb;
   // one column per thread; TRID_BT_CC=2 (A/B, b <= 64) gives each thread two columns -- two independent reflector
   // chains per warp -- measured slower at n = 8192 (345 vs 317 ms: half the CTAs, same per-reflector latency)
   static const char* ce = getenv("TRID_BT_CC");

@@ -168,7 +168,7 @@ def trid_bufsize_sbr(n, b, k, ncols):
 def trid_bc_bt_nb(b):
     rw = 128 if b <= 64 else (256 if b <= 128 else 512)
     nb = rw - b + 1
-    cap = 200 * 1024 // (8 * rw) - 1
+    cap = 200 * 1024 // (16 * rw) - 2
     return max(1, min(nb, cap))
 
 
