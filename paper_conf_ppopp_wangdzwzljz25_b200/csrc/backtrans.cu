@@ -313,18 +313,13 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
         double d[CC];
 #pragma unroll
         for (int u = 0; u < CC; ++u) {
-          // four independent chains (rows 16 p + 2 rg + h, p even / odd), summed in a fixed order
-          double d0 = 0.0, d1 = 0.0, d2 = 0.0, d3 = 0.0;
+          double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-          for (int p = 0; p < NP; p += 2) {
+          for (int p = 0; p < NP; ++p) {
             d0 = fma(vv[2 * p], x[u][2 * p], d0);
             d1 = fma(vv[2 * p + 1], x[u][2 * p + 1], d1);
-            if (p + 1 < NP) {
-              d2 = fma(vv[2 * p + 2], x[u][2 * p + 2], d2);
-              d3 = fma(vv[2 * p + 3], x[u][2 * p + 3], d3);
-            }
           }
-          d[u] = (d0 + d1) + (d2 + d3);
+          d[u] = d0 + d1;
         }
 #pragma unroll
         for (int u = 0; u < CC; ++u) d[u] += __shfl_xor_sync(0xffffffffu, d[u], 4);
