@@ -255,7 +255,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
     recv_ctr = 0;
     for (int i = 0; i < 2; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&lastb[i], 1);
+      mbar_init(&lastb[i], (!CL && (a.opt & 32)) ? 2 * B : 1);
       mbar_init(&empty[i], 1);
       mbar_init(&col0b[i], 2 * B);
       mbar_init(&colsb[i], (a.opt & 8) ? NW : 1);
@@ -302,7 +302,8 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
         const bool fwd = has_prod && bc_step_full(n, b, B, s, m);
         info_f[bi] = fwd;
         mbar_arrive_expect_tx(&full[bi], (unsigned)((L - 1 + (m == 0 ? 1 : 0)) * ldab * 8));
-        mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
+        const bool c0fetch = !CL && (a.opt & 32);   // the column-0 path threads fetch the last column themselves
+        if (!c0fetch) mbar_arrive_expect_tx(&lastb[bi], (unsigned)(ldab * 8));
         if (fwd) {   // the producer CTA copies body (+ column s at m = 0) and the last column into this buffer
           cl_st_release(cl_mapa(&armed_ctr, crank - 1), (int)(it + 1));
           BCW_TRACE(s, m, 8);
@@ -318,6 +319,7 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
         fence_proxy_async_global();
         if (m == 0) bulk_g2s(colb + bi * ldab, a.band + s * ldab, (unsigned)(ldab * 8), &full[bi]);
         if (L > 1) bulk_g2s(win, a.band + r0 * ldab, (unsigned)((L - 1) * ldab * 8), &full[bi]);
+        if (c0fetch) continue;
         if (s > 0) wait_geq_opt(a.prog + (s - 1) * a.fs, (int)((m + 2 < nprev) ? m + 2 : nprev), a.opt & 4);
         BCW_TRACE(s, m, 9);
         fence_proxy_async_global();
@@ -524,10 +526,27 @@ __device__ __forceinline__ void bc_v6_body(const BcArgs& a) {
       double acc = 0.0;
 #pragma unroll
       for (int q = 0; q < TPR; ++q) acc += part[q * 2 * B + r];
-      mbar_wait(&lastb[bi], ph);
+      double lastv = 0.0;   // element (r, L-1): the last window column, the predecessor's fresh column 0
+      if (!CL && (a.opt & 32)) {
+        // TRID_BC_OPT bit 32: these 2B threads (idle until the last column lands) poll the predecessor's counter and
+        // load the column straight from L2 -- no LOAD-warp detection, bulk copy or mbarrier on the chain; they fill
+        // the shared window column for the rest of the step and release it on lastb (2B arrivals)
+        if (s > 0 && tid == 0) {
+          const int64_t nprev = bc_steps(n, b, s - 1);
+          wait_geq_opt(a.prog + (s - 1) * a.fs, (int)((m + 2 < nprev) ? m + 2 : nprev), a.opt & 4);
+        }
+        c0bar();
+        const double* gl = a.band + (r0 + Lx - 1) * ldab;
+        if (r < ldab) win[(Lx - 1) * ldab + r] = __ldcg(gl + r);
+        if (r >= Lx - 1 && r - (Lx - 1) < ldab) lastv = __ldcg(gl + (r - (Lx - 1)));
+        mbar_arrive(&lastb[bi]);
+      } else {
+        mbar_wait(&lastb[bi], ph);
+        if (active && r >= L - 1) lastv = win[(L - 1) * lda1 + r];
+      }
       if (tid == 0) BCW_TRACE(s, m, 11);
       if (CL && tid == 0 && info_f[bi]) cl_st_release(cl_mapa(&recv_ctr, crank - 1), (int)(it + 1));
-      if (active && r >= L - 1) acc = fma(win[(L - 1) * lda1 + r], v[L - 1], acc);
+      if (active && r >= L - 1) acc = fma(lastv, v[L - 1], acc);
       const double py = (r >= L) ? acc : tau * acc;   // p_r = tau (D v)_r  |  y_r = (O v)_r
       pyv[r] = py;
       const double vr = r < L ? v[r] : 0.0;
