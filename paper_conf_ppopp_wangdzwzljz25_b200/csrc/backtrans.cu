@@ -348,11 +348,15 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   }
 }
 
-static int bc_bt_rw(int b) { return b <= 64 ? 128 : (b <= 128 ? 256 : 512); }
+// window rows RW = 8 QR: about b + 32, so a block holds ~33 sweeps and a reflector (b rows) covers most of the
+// window (round 2 first used 2b rows: half of every dot and update multiplied zeros, ncu: FP64 pipe 28 % busy for
+// 10 % useful flops)
+static int bc_bt_qr(int b) { return b <= 32 ? 8 : (b <= 64 ? 12 : (b <= 128 ? 20 : 36)); }
+static int bc_bt_rw(int b) { return 8 * bc_bt_qr(b); }
 
 int bc_bt_nb(int b) {
-  // window RW = 8*QR rows >= b + nb - 1 (QR = 16 for b <= 64, 32 for b <= 128, 64 for b <= 256); two buffers of
-  // nb staged window-shaped vectors (2 nb x RW doubles) fit in 200 KB of shared memory
+  // window RW = 8*QR rows >= b + nb - 1; two buffers of nb staged window-shaped vectors (2 nb x RW doubles) fit in
+  // 200 KB of shared memory
   const int rw = bc_bt_rw(b);
   int nb = rw - b + 1;
   const int cap = (int)(200 * 1024 / (16 * (size_t)rw)) - 2;
@@ -372,22 +376,28 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
   static const char* ce = getenv("TRID_BT_CC");
   const int cc = (ce && atoi(ce) == 2 && b <= 64) ? 2 : 1;
   const int64_t grid = (ncols + 32 * cc - 1) / (32 * cc);
-  const void* fn = b <= 64 ? (cc == 2 ? (const void*)bc_bt_kernel<16, 2> : (const void*)bc_bt_kernel<16, 1>)
-                           : (b <= 128 ? (const void*)bc_bt_kernel<32, 1> : (const void*)bc_bt_kernel<64, 1>);
-  static DeviceOnce attr16, attr16b, attr32, attr64;
-  DeviceOnce& at = b <= 64 ? (cc == 2 ? attr16b : attr16) : (b <= 128 ? attr32 : attr64);
-  cudaError_t e = at([&] {
+  const int qr = bc_bt_qr(b);
+  const void* fn = qr == 8 ? (cc == 2 ? (const void*)bc_bt_kernel<8, 2> : (const void*)bc_bt_kernel<8, 1>)
+                 : qr == 12 ? (cc == 2 ? (const void*)bc_bt_kernel<12, 2> : (const void*)bc_bt_kernel<12, 1>)
+                 : qr == 20 ? (const void*)bc_bt_kernel<20, 1> : (const void*)bc_bt_kernel<36, 1>;
+  static DeviceOnce attrs[6];
+  const int ai = qr == 8 ? (cc == 2 ? 0 : 1) : qr == 12 ? (cc == 2 ? 2 : 3) : qr == 20 ? 4 : 5;
+  cudaError_t e = attrs[ai]([&] {
     return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   });
   if (e != cudaSuccess) return e;
-  if (b <= 64 && cc == 2)
-    bc_bt_kernel<16, 2><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
-  else if (b <= 64)
-    bc_bt_kernel<16, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
-  else if (b <= 128)
-    bc_bt_kernel<32, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  if (qr == 8 && cc == 2)
+    bc_bt_kernel<8, 2><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (qr == 8)
+    bc_bt_kernel<8, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (qr == 12 && cc == 2)
+    bc_bt_kernel<12, 2><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (qr == 12)
+    bc_bt_kernel<12, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+  else if (qr == 20)
+    bc_bt_kernel<20, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
   else
-    bc_bt_kernel<64, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
+    bc_bt_kernel<36, 1><<<(unsigned)grid, BT_NT, smem, st>>>(n, b, nb, V2, tau2, trans, ncols, C, ldc);
   count_launches(1);
   return cudaGetLastError();
 }

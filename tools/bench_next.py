@@ -166,7 +166,7 @@ def trid_bufsize_sbr(n, b, k, ncols):
 
 
 def trid_bc_bt_nb(b):
-    rw = 128 if b <= 64 else (256 if b <= 128 else 512)
+    rw = 8 * (8 if b <= 32 else (12 if b <= 64 else (20 if b <= 128 else 36)))
     nb = rw - b + 1
     cap = 200 * 1024 // (16 * rw) - 2
     return max(1, min(nb, cap))
