@@ -20,7 +20,7 @@
 // rows overlap always satisfy m' <= m for s < s' (rows s+1+mb.. and s'+1+m'b.. overlap iff |s'-s+(m'-m)b| < b),
 // so this order keeps every overlapping pair in sweep-major order and only commutes disjoint ones.  Group G_m
 // touches rows [s0+1+mb, s0+nb-1+(m+1)b] (R = b+nb-1 rows).  Q2 C = B_0 (B_1 (... (B_last C))), B = G_M..G_0.
-// Kernel: one CTA per 32-column slab of C; per sweep block (last to first) it slides down the rows group by group
+// Kernel: one CTA per 16-column slab of C; per sweep block (last to first) it slides down the rows group by group
 // (G_0 first): the group's window rows are loaded from the slab into registers (a warp holds 4 columns; its 8 row
 // lanes per column hold interleaved row pairs, so every access is 16 consecutive rows), its nb reflectors (from V2,
 // staged once per group in shared memory in window shape, zero-padded) are applied one at a time -- partial dot over
@@ -207,7 +207,7 @@ __host__ __device__ inline int64_t bt_offset(int64_t n, int b, int64_t s) {   //
   return bt_F(n - 3, b) - bt_F(n - 3 - s, b);
 }
 
-constexpr int BT_NT = 256;
+constexpr int BT_NT = 128;   // 4 warps x 4 column lanes: 16 columns per CTA (n / 16 CTAs: balanced over the SMs)
 
 // QR rows per thread; the group window holds 8*QR >= b + nb - 1 rows.
 __device__ __forceinline__ void bt_cp8(double* dst, const double* src) {
@@ -221,7 +221,7 @@ __global__ void __launch_bounds__(BT_NT, 1) bc_bt_kernel(int64_t n, int b, int n
   constexpr int RW = 8 * QR;   // window rows
   constexpr int NP = QR / 2;   // row pairs per thread: thread (rg, cl) holds rows 16 p + 2 rg + {0, 1}, p < NP, of
                                // its CC columns -- the 8 row-group lanes of a column cover 16 consecutive rows
-  constexpr int COLS = 32 * CC;   // columns per CTA: 8 warps x 4 column lanes x CC columns per thread
+  constexpr int COLS = (BT_NT / 8) * CC;   // columns per CTA: (BT_NT / 32) warps x 4 column lanes x CC per thread
   // two buffers of the group's reflectors in window shape, Vw[j][r] = v_j[r - j] (zero outside [j, j+b): the zero
   // rows are written once, the b rows of vector j are refilled per group by cp.async), nb x RW each; 2 x nb taus;
   // the block's per-sweep V2 offsets S(s0+j) and step counts
@@ -375,7 +375,8 @@ cudaError_t bc_backtransform(int64_t n, int b, const double* V2, const double* t
   // chains per warp -- measured slower at n = 8192 (345 vs 317 ms: half the CTAs, same per-reflector latency)
   static const char* ce = getenv("TRID_BT_CC");
   const int cc = (ce && atoi(ce) == 2 && b <= 64) ? 2 : 1;
-  const int64_t grid = (ncols + 32 * cc - 1) / (32 * cc);
+  const int cols = (BT_NT / 8) * cc;
+  const int64_t grid = (ncols + cols - 1) / cols;
   const int qr = bc_bt_qr(b);
   const void* fn = qr == 8 ? (cc == 2 ? (const void*)bc_bt_kernel<8, 2> : (const void*)bc_bt_kernel<8, 1>)
                  : qr == 12 ? (cc == 2 ? (const void*)bc_bt_kernel<12, 2> : (const void*)bc_bt_kernel<12, 1>)
