@@ -20,7 +20,7 @@
 // rows overlap always satisfy m' <= m for s < s' (rows s+1+mb.. and s'+1+m'b.. overlap iff |s'-s+(m'-m)b| < b),
 // so this order keeps every overlapping pair in sweep-major order and only commutes disjoint ones.  Group G_m
 // touches rows [s0+1+mb, s0+nb-1+(m+1)b] (R = b+nb-1 rows).  Q2 C = B_0 (B_1 (... (B_last C))), B = G_M..G_0.
-// Kernel: one CTA per 16-column slab of C; per sweep block (last to first) it slides down the rows group by group
+// Kernel: one CTA per 32-column slab of C; per sweep block (last to first) it slides down the rows group by group
 // (G_0 first): the group's window rows are loaded from the slab into registers (a warp holds 4 columns; its 8 row
 // lanes per column hold interleaved row pairs, so every access is 16 consecutive rows), its nb reflectors (from V2,
 // staged once per group in shared memory in window shape, zero-padded) are applied one at a time -- partial dot over
@@ -207,7 +207,7 @@ __host__ __device__ inline int64_t bt_offset(int64_t n, int b, int64_t s) {   //
   return bt_F(n - 3, b) - bt_F(n - 3 - s, b);
 }
 
-constexpr int BT_NT = 128;   // 4 warps x 4 column lanes: 16 columns per CTA (n / 16 CTAs: balanced over the SMs)
+constexpr int BT_NT = 256;   // 8 warps x 4 column lanes: 32 columns per CTA (16-column CTAs measured slower)
 
 // QR rows per thread; the group window holds 8*QR >= b + nb - 1 rows.
 __device__ __forceinline__ void bt_cp8(double* dst, const double* src) {
