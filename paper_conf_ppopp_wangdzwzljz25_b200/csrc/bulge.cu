@@ -837,6 +837,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
   __syncthreads();
   // threads per window row in the matvec (b <= 128: two, each over half of my columns)
   const int tpr = BW_NT / H2 >= 2 ? 2 : 1;
+  const int jmid = cbeg + (cend - cbeg + 1) / 2;
   for (;;) {
     if (q == 0 && tid == 0) {
       const double s0 = (double)atomicAdd(a.ticket, 1u);   // exact (< 2^53)
@@ -916,12 +917,11 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           if (h < tpr) {
             double acc = 0.0;
             if (i < H) {
-              // the two threads of a row take alternate columns (equal work for every row)
-              int jhi = je;
+              const int jlo = tpr == 2 ? (h ? jmid : cbeg) : cbeg;
+              int jhi = tpr == 2 ? (h ? je : (jmid < je ? jmid : je)) : je;
               if (jhi > i + 1) jhi = i + 1;   // lower part of D (and all of O): columns j <= i
               if (jhi > L - 1) jhi = L - 1;   // body only
-              const int jst = tpr == 2 ? 2 : 1;
-              for (int j = cbeg + (tpr == 2 ? h : 0); j < jhi; j += jst) acc = fma(win[cofs[j] + i], v[j], acc);
+              for (int j = jlo; j < jhi; ++j) acc = fma(win[cofs[j] + i], v[j], acc);
             }
             prt[h * H2 + i] = acc;
           }
@@ -1055,20 +1055,19 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
             }
           }
         }
-        if (j > 0 || L2 == 0) {
-          // the column is final: this warp stores it now (overlapping the other warps' passes)
-          __syncwarp();
-          const int len = H - j, len2 = len >> 1;
-          const double* srcp = col + j;
-          double* dst = a.band + (r0 + j) * ldab;
-          for (int i = lane; i < len2; i += 32)
-            __stcg(reinterpret_cast<double2*>(dst) + i, reinterpret_cast<const double2*>(srcp)[i]);
-          if ((len & 1) && lane == 0) __stcg(dst + len - 1, srcp[len - 1]);
-        }
       }
       __syncthreads();
       if (a.opt & 256) bw_csync<CS>();
-      // ---- (every column was stored by its warp right after its pass) the reflector of this step, publish
+      // ---- store my columns back (one warp per column), the reflector of this step, publish
+      for (int j = cbeg + warp; j < je; j += NW) {
+        if (j == 0 && L2 > 0) continue;   // column 0 went out early (step 4)
+        const int len = H - j, len2 = len >> 1;
+        const double* srcp = win + cofs[j] + j;
+        double* dst = a.band + (r0 + j) * ldab;
+        for (int i = lane; i < len2; i += 32)
+          __stcg(reinterpret_cast<double2*>(dst) + i, reinterpret_cast<const double2*>(srcp)[i]);
+        if ((len & 1) && lane == 0) __stcg(dst + len - 1, srcp[len - 1]);
+      }
       if (q == 0 && a.V2) {
         double* vd = a.V2 + (off + m) * a.vs;
         for (int i = tid; i < a.vs; i += BW_NT) vd[i] = i < L ? v[i] : 0.0;
