@@ -74,6 +74,9 @@ struct WsArgs {
   // mg_g <= 1: identity.  Used by the lower epilogue mask (C's columns are local) and the SYMM modes 2/3.
   int mg_g, mg_q, mg_cb;
   int64_t mg_lofs, mg_gofs;
+  // TMA-staged operands (GEMM segments with A op N and B op T, 128 x 128 tiles, vec16, even M and N: the
+  // deferred syr2k): the producer stages every k-row of a tile with one bulk copy (cp.async.bulk) per operand
+  int tma;
 };
 
 template <bool MG>
@@ -355,7 +358,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], NPW * 32);   // one cp.async.mbarrier.arrive.noinc per producer thread
+      mbar_init(&full[s], a.tma ? 32 : NPW * 32);   // one arrive per producer thread (TMA: warp 0 only)
       mbar_init(&empty[s], NCW);  // one arrive per consumer warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -366,6 +369,57 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
     // ======================= producer warpgroup =======================
     if (NCW == 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;\n" ::: "memory");
     const int pt = threadIdx.x - NCW * 32;
+    if constexpr (!MG && OPB == OP_T && BM == 128 && BN == 128) {
+      if (a.tma) {
+        // TMA staging: producer warp 0 alone; per stage, lane 0 issues one bulk copy per k-row of A and of B (the
+        // tile's rows of one column: contiguous, 16-byte multiple since M and N are even) straight into the padded
+        // stage rows the consumers' DMMA fragment loads expect (no bank conflicts; 32 copies of <= 1 KB per stage
+        // instead of 128 threads x 16 cp.async).  Rows past M / N and k past the segment end are zeroed by the
+        // warp with generic stores (fenced to the async proxy: the next use of the slot may be a bulk copy).
+        // full[slot] expects 32 arrivals: lane 0's expect_tx + 31 plain arrives (each releases its own stores).
+        if (pt >= 32) return;
+        uint32_t kt = 0;
+        for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+          int64_t m0, n0;
+          int z;
+          unit_geom<BM, BN>(a, u, m0, n0, z);
+          if (a.lower && m0 + BM - 1 + a.diag_off < n0) continue;
+          Seg s0, s1;
+          const int ns = unit_segs<BM, BN, MG>(a, m0, z, s0, s1);
+          const int rm = (int)(a.M - m0 < BM ? a.M - m0 : BM), rn = (int)(a.N - n0 < BN ? a.N - n0 : BN);
+          auto run = [&](const Seg& sgm) {
+            for (int64_t k0 = sgm.kb; k0 < sgm.ke; k0 += BK, ++kt) {
+              const int slot = kt % STAGES;
+              const uint32_t use = kt / STAGES;
+              if (use > 0) mbar_wait(&empty[slot], (use - 1) & 1u);
+              double* As = smem + (size_t)slot * C::STAGE;
+              double* Bs = As + C::A_ELEMS;
+              const int kc = (int)((sgm.ke - k0) < BK ? (sgm.ke - k0) : BK);
+              if (kc < BK || rm < BM || rn < BN) {
+                for (int kk = 0; kk < BK; ++kk) {
+                  const int ra = kk < kc ? rm : 0, rb = kk < kc ? rn : 0;
+                  for (int r = ra + pt; r < BM; r += 32) As[kk * C::A_LD_N + r] = 0.0;
+                  for (int r = rb + pt; r < BN; r += 32) Bs[kk * C::B_LD_T + r] = 0.0;
+                }
+                asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+              }
+              if (pt == 0) {
+                mbar_arrive_expect_tx(&full[slot], (unsigned)(kc * (rm + rn) * 8));
+                for (int kk = 0; kk < kc; ++kk) {
+                  bulk_g2s(As + kk * C::A_LD_N, sgm.A + m0 + (k0 + kk) * sgm.lda, rm * 8, &full[slot]);
+                  bulk_g2s(Bs + kk * C::B_LD_T, sgm.B + n0 + (k0 + kk) * sgm.ldb, rn * 8, &full[slot]);
+                }
+              } else {
+                mbar_arrive(&full[slot]);
+              }
+            }
+          };
+          if (ns > 0) run(s0);
+          if (ns > 1) run(s1);
+        }
+        return;
+      }
+    }
     uint32_t kt = 0;   // global K-tile counter (ring position)
     for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
       int64_t m0, n0;
@@ -530,6 +584,10 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   if (g.N <= 64) {
     return opB == OP_T ? ws::launch<128, 64, 4, 2, OP_T>(a, st) : ws::launch<128, 64, 4, 2, OP_N>(a, st);
   }
+  // bulk-copy (TMA) staging for A op N / B op T on 128 x 128 tiles (the syr2k and the other NT contractions);
+  // env TRID_WS_TMA=0 restores the cp.async producer warpgroup
+  const char* tenv = getenv("TRID_WS_TMA");   // read per call (tests toggle it)
+  a.tma = (!tenv || atoi(tenv) != 0) && opA == OP_N && opB == OP_T && v16 && !(g.M & 1) && !(g.N & 1);
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 

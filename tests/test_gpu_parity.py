@@ -47,6 +47,41 @@ def test_syr2k_lower_parity(m, kk, dev):
     assert np.array_equal(got[iu], C[iu])      # strict upper untouched, bitwise
 
 
+@pytest.mark.parametrize("m,kk", [(1000, 100), (512, 64), (258, 37), (2048, 256)])
+def test_syr2k_tma_staging_bitwise(m, kk, dev, monkeypatch):
+    """The bulk-copy (TMA) producer of the NT engine path stages the same tile values into the same padded
+    layout as the cp.async producer, so the consumers' DMMA order and the result are identical bit for bit
+    (ragged row tails m % 128 != 0 and ragged K tails kk % 16 != 0 included); both match the oracle."""
+    rng = np.random.default_rng(m + 7 * kk)
+    C = rng.uniform(-1, 1, (m, m))
+    Y = rng.uniform(-1, 1, (m, kk))
+    Z = rng.uniform(-1, 1, (m, kk))
+    outs = []
+    for env in ("1", "0"):
+        monkeypatch.setenv("TRID_WS_TMA", env)
+        Cd = to_dev(C)
+        trid.syr2k_lower(Cd, to_dev(Y), to_dev(Z))
+        outs.append(from_dev(Cd))
+    assert np.array_equal(outs[0], outs[1])
+    ref = oracle.syr2k_lower(C, Y, Z)
+    il = np.tril_indices(m)
+    bound = 2 * 4 * (2 * kk + 1) * U * (np.abs(Y) @ np.abs(Z).T + np.abs(Z) @ np.abs(Y).T + np.abs(C))
+    assert np.all(np.abs(outs[0] - ref)[il] <= bound[il])
+
+
+@pytest.mark.parametrize("n,b", [(1024, 64), (1030, 32)])
+def test_dbbr_tma_staging_bitwise(n, b, dev, monkeypatch):
+    """DBBR with the bulk-copy producer equals DBBR with the cp.async producer bit for bit."""
+    A = trid_gen.random_symmetric_np(n, 4242 + n)
+    outs = []
+    for env in ("1", "0"):
+        monkeypatch.setenv("TRID_WS_TMA", env)
+        Ad = to_dev(A)
+        tau = trid.sbr_dbbr(Ad, b, nb=min(16, b), k=4 * b)
+        outs.append((from_dev(Ad), tau.cpu().numpy()))
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
 # ------------------------------------------------------------------------------------------ panel QR
 @pytest.mark.parametrize("m,w", [(224, 32), (1000, 64), (5000, 64), (64, 64), (40, 64), (33, 8), (7000, 128),
                                  (3000, 256), (2, 4)])
