@@ -679,7 +679,11 @@ int trid_zy(int64_t m, int w, const double* A, int64_t lda, const double* W, int
   if (pe < (int64_t)32 * w * w) pe = (int64_t)32 * w * w;
   double* part = c.take<double>((size_t)pe);
   // Eq. (1) with no earlier panels: Y and Z of this call are separate buffers (ldy, ldz)
-  cudaError_t e = symm_ws(m, w, A, lda, W, ldw, X, m, part, pe, stream);
+  cudaError_t e;
+  {
+    ProfScope ps(PROF_SYMM, stream);
+    e = symm_ws(m, w, A, lda, W, ldw, X, m, part, pe, stream);
+  }
   if (e != cudaSuccess) return TRID_ERR_CUDA;
   GemmArgs s;
   s.M = w; s.N = w; s.K[0] = m; s.A[0] = W; s.lda[0] = ldw; s.B[0] = X; s.ldb[0] = m;
