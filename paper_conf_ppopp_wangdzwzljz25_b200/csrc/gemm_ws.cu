@@ -22,6 +22,9 @@
 
 #include <stdlib.h>
 
+#include <mutex>
+#include <unordered_map>
+
 namespace trid {
 
 namespace ws {
@@ -672,17 +675,67 @@ int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {
   return sp < 1 ? 1 : (int)sp;
 }
 
-// Strip splits of the SYMM: the persistent grid runs >= ~8 waves of units (tail imbalance <~ 6%);
-// env TRID_SYMM_WAVES overrides (tuning).
+// Strip splits of the SYMM, chosen by a makespan model of the persistent grid (148 CTAs walking units
+// u = z * tiles + t with stride 148, unit z covering the K chunk [z cz, (z + 1) cz) of the strip, cz a multiple of
+// 16): unit cost = (its K + the diagonal-block overlap) / 16 stages x 1.19 us (one 128 x 64 x 16 DMMA stage at
+// ~0.88 of 37 TF/s over 148 SMs) + 2 us (unit epilogue / refill); + the split-K reduction over HBM (read s + 1,
+// write 1 partial, 5 TB/s).  Pure function of (m, w) and fixed constants (the workspace sizing and the
+// deterministic sums use it), memoized.  The former rule (>= 8 waves, K >= 512 per split) left up to 9% of the
+// last wave idle at some m (e.g. m = 28608: 1344 units = 9.08 waves).  env TRID_SYMM_WAVES=W restores it.
+static int64_t symm_splits_model(int64_t m, int64_t w) {
+  const int64_t tm = (m + 127) / 128, rows = tm * ((w + 63) / 64);
+  int64_t maxs = (m + 255) / 256 < 32 ? (m + 255) / 256 : 32;
+  const int64_t maxw = (24 * kNumSMsB200 + rows - 1) / rows;   // <= ~24 waves (bounds the search)
+  if (maxs > maxw) maxs = maxw;
+  double best = 1e300;
+  int64_t bs = 1;
+  double load[kNumSMsB200];
+  for (int64_t sp = 1; sp <= maxs; ++sp) {
+    const int64_t chunk = (m + sp - 1) / sp, cz = (chunk + 15) / 16 * 16;
+    for (int c = 0; c < kNumSMsB200; ++c) load[c] = 0.0;
+    const int64_t units = rows * sp;
+    for (int64_t u = 0; u < units; ++u) {
+      const int64_t z = u / rows, t = (u % rows) % tm;
+      const int64_t k0 = z * cz, k1 = k0 + cz < m ? k0 + cz : m;
+      double kk = k1 > k0 ? (double)(k1 - k0) : 0.0;
+      const int64_t d0 = t * 128, d1 = d0 + 128 < m ? d0 + 128 : m;   // diagonal block, counted by both strips
+      const int64_t o0 = k0 > d0 ? k0 : d0, o1 = k1 < d1 ? k1 : d1;
+      if (o1 > o0) kk += (double)(o1 - o0);
+      load[u % kNumSMsB200] += kk / 16.0 * 1.19 + 2.0;
+    }
+    double mk = 0.0;
+    for (int c = 0; c < kNumSMsB200; ++c) mk = load[c] > mk ? load[c] : mk;
+    if (sp > 1) mk += (double)(sp + 2) * (double)m * (double)w * 8.0 / 5.0e6;
+    if (mk < best * 0.999) {
+      best = mk;
+      bs = sp;
+    }
+  }
+  return bs;
+}
+
 int64_t symm_ws_splits(int64_t m, int64_t w) {
-  const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
   static const char* wv = getenv("TRID_SYMM_WAVES");
-  const int64_t waves = wv ? atoll(wv) : 8;
-  int64_t sp = (waves * kNumSMsB200 + rows - 1) / rows;
-  const int64_t maxs = (m + 511) / 512;
-  if (sp > maxs) sp = maxs;
-  if (sp > 32) sp = 32;
-  if (sp < 1) sp = 1;
+  if (wv) {
+    const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
+    int64_t sp = (atoll(wv) * kNumSMsB200 + rows - 1) / rows;
+    const int64_t maxs = (m + 511) / 512;
+    if (sp > maxs) sp = maxs;
+    if (sp > 32) sp = 32;
+    return sp < 1 ? 1 : sp;
+  }
+  if (m <= 0 || w <= 0) return 1;
+  static std::mutex mu;
+  static std::unordered_map<int64_t, int64_t> memo;
+  const int64_t key = m * 4096 + w;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = memo.find(key);
+    if (it != memo.end()) return it->second;
+  }
+  const int64_t sp = symm_splits_model(m, w);
+  std::lock_guard<std::mutex> lk(mu);
+  memo[key] = sp;
   return sp;
 }
 int64_t symm_ws_part_elems(int64_t m, int64_t w) {
