@@ -107,6 +107,44 @@ def test_panel_qr_parity(m, w, dev):
     assert np.max(np.abs(Vu @ Tl - W_o)) <= 64 * m * U * np.max(np.abs(W_o))
 
 
+@pytest.mark.parametrize("m,w,kind", [(5000, 64, "parallel"), (5000, 64, "near"), (1000, 32, "parallel"),
+                                      (32704, 64, "near"), (700, 16, "zero")])
+def test_panel_qr_dependent_columns(m, w, kind, dev):
+    """Columns (nearly) parallel to their left neighbour make the pair kernel's look-ahead norm a cancelling
+    difference; it must fall back to one reflector per reduction there.  Checked by backward error: the Householder
+    product Q (from V, tau) is orthogonal and Q R reproduces the panel, both to O(m u) (the reflectors themselves
+    are ill-conditioned here, so no element parity)."""
+    rng = np.random.default_rng(m + w)
+    P = rng.uniform(-1, 1, (m, w))
+    if kind == "parallel":
+        P[:, 1] = 2.0 * P[:, 0]
+        P[:, 9] = -P[:, 8]
+        P[:, w - 1] = 0.5 * P[:, w - 2]
+    elif kind == "near":
+        P[:, 1] = P[:, 0] * (1 + 1e-9) + 1e-12 * rng.uniform(-1, 1, m)
+        P[:, 6] = P[:, 5] + 1e-7 * rng.uniform(-1, 1, m)
+    else:
+        P[:, 3] = 0.0
+        P[:, 4] = 0.0
+    Pd = to_dev(P)
+    tau, T, Y = trid.panel_qr(Pd)
+    got = from_dev(Pd)
+    kk = min(m, w)
+    tau = tau.cpu().numpy()
+    V = np.tril(got, -1)[:, :kk] + np.eye(m, kk)
+    R = np.triu(got)[:kk, :]
+    E = np.eye(m, kk)
+    Q = E.copy()
+    for j in range(kk - 1, -1, -1):      # Q = H_0 ... H_{kk-1} applied to the first kk unit vectors
+        v = V[:, j]
+        Q -= tau[j] * np.outer(v, v @ Q)
+    assert np.linalg.norm(Q.T @ Q - np.eye(kk)) <= 64 * m * U
+    assert np.linalg.norm(Q @ R - P) <= 64 * m * U * np.linalg.norm(P)
+    Tl = from_dev(T)[:kk, :kk]
+    Qt = E - V @ (Tl @ (V.T @ E))
+    assert np.linalg.norm(Qt - Q) <= 64 * m * U
+
+
 # ------------------------------------------------------------------------------------------ Z builder
 @pytest.mark.parametrize("m,w", [(200, 32), (1000, 64), (3000, 64), (700, 16), (513, 128)])
 def test_zy_parity(m, w, dev):
