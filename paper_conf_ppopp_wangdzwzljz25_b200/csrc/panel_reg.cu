@@ -302,12 +302,398 @@ __global__ void __launch_bounds__(PR_NT, 1) panel_reg_kernel(const __grid_consta
   cl.sync();   // no CTA leaves while a cluster peer may still read its shared memory
 }
 
-size_t panel_reg_gpart_bytes(int w) { return sizeof(double) * 2 * PR_MAXNC * 2 * (size_t)w; }
+// Transposed butterfly: NVv per-lane partial sums -> lane holds the warp total of value index qb in f (lanes with
+// (lane & (32 / NVv - 1)) == 0 own a distinct index; NVv a power of two <= 32).
+template <int NVv>
+__device__ __forceinline__ double warp_butterfly(double (&acc)[NVv], int lane, int& qb) {
+  qb = 0;
+#pragma unroll
+  for (int o = 16, K = NVv; K > 1; o >>= 1, K >>= 1) {
+    const bool up = (lane & o) != 0;
+#pragma unroll
+    for (int i = 0; i < K / 2; ++i) {
+      const double send = up ? acc[i] : acc[i + K / 2];
+      const double keep = up ? acc[i + K / 2] : acc[i];
+      acc[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+    }
+    if (up) qb += K / 2;
+  }
+  constexpr int LV = NVv >= 32 ? 5 : (NVv == 16 ? 4 : (NVv == 8 ? 3 : (NVv == 4 ? 2 : (NVv == 2 ? 1 : 0))));
+  double f = acc[0];
+#pragma unroll
+  for (int o = 16 >> LV; o >= 1; o >>= 1) f += __shfl_xor_sync(0xffffffffu, f, o);
+  return f;
+}
 
+// ---- two reflectors per grid barrier (look-ahead by one column) ----------------------------------------------
+// One reduction serves the column pair (p, q = p + 1): besides the Gram row of column p (G1[j] = sum_{r>p} a_p a_j)
+// and row p (Rp[j] = a_j(p)) it carries the Gram row of column q over rows > q (G2[j] = sum_{r>q} a_q a_j) and row q
+// (Rq[j]); sums of a_p a_j over rows > q are G1[j] - Rq[p] Rq[j].  Reflector p is formed as in panel_reg_kernel: w_j = Rp[j] + s G1[j], a'_j = a_j - tau v_p w_j, i.e.
+// a'_j(r) = a_j(r) - c_j a_p(r) below row p with c_j = tau s w_j.  Column q after it, and every product reflector q
+// needs, follow from the same sums (exact algebra, sums over r > q):
+//   sigma' = sum a'_q^2          = G2[q] - 2 c_q G2[p] + c_q^2 (G1[p] - Rq[p]^2),   alpha' = Rq[q] - c_q Rq[p],
+//   sum a'_q a'_j                = G2[j] - c_j G2[p] - c_q (G1[j] - Rq[p] Rq[j]) + c_q c_j (G1[p] - Rq[p]^2),
+//   w'_j = a'_j(q) + s' sum a'_q a'_j,  a'_j(q) = Rq[j] - c_j Rq[p],
+// and v_q^T v_s (the T factor) likewise.  sigma' is a difference: when it falls below 1/16 of the magnitude of its
+// terms, G1[p] and Rq[p]^2 counted separately (column q nearly parallel to column p, or a_p(q) dominating column p
+// below row p: cancellation could cost more than 4 bits of the norm, and with it the orthogonality of H_q) the step
+// takes reflector p alone and the next reduction restarts at q.  Every CTA sums
+// the same partials in the same order, so all CTAs take the same branch.  Halves the grid barriers of the panel.
+template <int CPW>
+__global__ void __launch_bounds__(PR_NT, 1) panel_reg2_kernel(const __grid_constant__ PanelRegArgs a) {
+  constexpr int W = 8 * CPW;
+  constexpr int RS = 4 * W;   // [G1 | G2 | Rp | Rq]
+  constexpr int NV = 2 * CPW;
+  static_assert(RS % (8 * PR_CL) == 0, "the DSMEM reduction loop must be warp-uniform");
+  constexpr int XS = 32 * PR_RL;
+  extern __shared__ __align__(16) double sm[];
+  double* xsb = sm;                     // [parity][column p, column q][rows of this CTA]
+  double* mypart = xsb + 4 * XS;        // 2 x RS (by parity)
+  double* tot = mypart + 2 * RS;        // RS
+  double* Ts = tot + RS;                // W x W    (CTA 0)
+  double* Dm = Ts + W * W;              // W x W    (CTA 0): v_t^T v_p, p < t
+  double* taus = Dm + W * W;            // W        (CTA 0)
+  cg::cluster_group cl = cg::this_cluster();
+  const int g = blockIdx.x, G = gridDim.x, NC = G / PR_CL;
+  const int crank = (int)cl.block_rank(), cid = g / PR_CL;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t rlo = (int64_t)g * a.rows;
+  const int nr = (int)((rlo + a.rows <= a.m) ? a.rows : (a.m > rlo ? a.m - rlo : 0));
+  const int j0 = warp * CPW;
+
+  double P[PR_RL][CPW];
+#pragma unroll
+  for (int q = 0; q < PR_RL; ++q) {
+    const int i = lane + 32 * q;
+#pragma unroll
+    for (int c = 0; c < CPW; ++c)
+      P[q][c] = (i < nr && j0 + c < a.w) ? a.P[(rlo + i) + (int64_t)(j0 + c) * a.ldp] : 0.0;
+  }
+  // columns 0 and 1 -> parity-0 buffers
+#pragma unroll
+  for (int cc = 0; cc < 2; ++cc)
+    if (cc < a.w && warp == cc / CPW) {
+#pragma unroll
+      for (int q = 0; q < PR_RL; ++q) {
+        double v = 0.0;
+#pragma unroll
+        for (int c = 0; c < CPW; ++c)
+          if (c == cc % CPW) v = P[q][c];
+        xsb[cc * XS + lane + 32 * q] = v;
+      }
+    }
+  unsigned epoch = 0;
+  int par = 0;
+  int tp0 = -1, tp1 = -1;   // reflectors of the previous step whose T columns are still to be built (CTA 0)
+  __syncthreads();
+
+  for (int t = 0; t < a.kk;) {
+    const bool pair = t + 1 < a.kk;
+    const double* x1 = xsb + (2 * par) * XS;
+    const double* x2 = x1 + XS;
+    // ---- 1. Gram slots of this warp's columns: G1 over rows > t, G2 over rows > t + 1; rows t and t + 1
+    double acc[NV];
+#pragma unroll
+    for (int c = 0; c < NV; ++c) acc[c] = 0.0;
+    int qt = -1, qt2 = -1;
+#pragma unroll
+    for (int q = 0; q < PR_RL; ++q) {
+      const int i = lane + 32 * q;
+      const int64_t r = rlo + i;
+      const bool ok = i < nr;
+      const double x = (ok && r > t) ? x1[i] : 0.0;
+      const double y = (ok && pair && r > t + 1) ? x2[i] : 0.0;
+      if (ok && r == t) qt = q;
+      if (ok && r == t + 1) qt2 = q;
+#pragma unroll
+      for (int c = 0; c < CPW; ++c) {
+        acc[c] = fma(x, P[q][c], acc[c]);
+        acc[CPW + c] = fma(y, P[q][c], acc[CPW + c]);
+      }
+    }
+    double* mp = mypart + par * RS;
+    {
+      int qb;
+      const double f = warp_butterfly<NV>(acc, lane, qb);
+      constexpr int LV = NV >= 16 ? 4 : (NV == 8 ? 3 : (NV == 4 ? 2 : 1));
+      if ((lane & ((32 >> LV) - 1)) == 0) mp[qb < CPW ? j0 + qb : W + j0 + qb - CPW] = f;
+    }
+    // rows t and t + 1 of this warp's columns (owner lane) or zero
+#pragma unroll
+    for (int rr = 0; rr < 2; ++rr) {
+      const int qo = rr ? qt2 : qt;
+      const unsigned own = __ballot_sync(0xffffffffu, qo >= 0);
+      double* dst = mp + (2 + rr) * W + j0;
+      if (own) {
+        const int src = __ffs(own) - 1;
+#pragma unroll
+        for (int c = 0; c < CPW; ++c) {
+          double vv = 0.0;
+#pragma unroll
+          for (int q = 0; q < PR_RL; ++q)
+            if (q == qo) vv = P[q][c];
+          vv = __shfl_sync(0xffffffffu, vv, src);
+          if (lane == 0) dst[c] = vv;
+        }
+      } else if (lane < CPW) {
+        dst[lane] = 0.0;
+      }
+    }
+    // ---- 2. cluster reduction through DSMEM (fixed order over the cluster's CTAs)
+    cl.sync();
+    for (int k = tid / PR_CL; PR_CL * k < RS; k += PR_NT / PR_CL) {
+      const int c = tid % PR_CL;
+      const int sl = crank + PR_CL * k;
+      double v = 0.0;
+      if (sl < RS) {
+        const double* rp = cl.map_shared_rank(mypart + par * RS, c);
+        v = rp[sl];
+      }
+#pragma unroll
+      for (int o = 1; o < PR_CL; o <<= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+      if (c == 0 && sl < RS) __stcg(a.gpart + ((size_t)par * NC + cid) * RS + sl, v);
+    }
+    // ---- 3. one grid barrier; CTA 0 builds the previous step's T columns meanwhile (warps 2-3, named barrier)
+    __syncthreads();
+    epoch += 1;
+    if (tid == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;\n" ::"l"(a.bar + 32 * (g % PR_NBAR)) : "memory");
+    if (g == 0 && tid >= 64 && tid < 128 && tp0 >= 0) {
+      const int u = tid - 64;
+      for (int pass = 0; pass < 2; ++pass) {
+        const int c = pass ? tp1 : tp0;
+        if (c < 0) break;
+        for (int q2 = u; q2 < W; q2 += 64) {
+          double v = 0.0;
+          if (q2 < c) {
+            double sacc = 0.0;
+            for (int p = q2; p < c; ++p) sacc += Ts[q2 + p * W] * Dm[c * W + p];
+            v = -taus[c] * sacc;
+          } else if (q2 == c) {
+            v = taus[c];
+          }
+          Ts[q2 + c * W] = v;
+        }
+        asm volatile("bar.sync 1, 64;\n" ::: "memory");
+      }
+    }
+    if (tid < PR_NBAR) {
+      const unsigned target = epoch * (unsigned)((G - tid + PR_NBAR - 1) / PR_NBAR);
+      const unsigned* cnt = a.bar + 32 * tid;
+      while (ld_relaxed_u32(cnt) < target) {
+      }
+      (void)ld_acquire_u32(cnt);
+    }
+    __syncthreads();
+    // ---- 4. totals over the NC cluster partials, fixed order
+    for (int sl = tid; sl < RS; sl += PR_NT) {
+      double vals[PR_MAXNC];
+#pragma unroll
+      for (int q = 0; q < PR_MAXNC; ++q) vals[q] = q < NC ? __ldcg(a.gpart + ((size_t)par * NC + q) * RS + sl) : 0.0;
+      double v = vals[0];
+#pragma unroll
+      for (int q = 1; q < PR_MAXNC; ++q)
+        if (q < NC) v += vals[q];
+      tot[sl] = v;
+    }
+    __syncthreads();
+    // ---- 5. reflector p (and q), update, T inputs
+    const double* G1 = tot;
+    const double* G2 = tot + W;
+    const double* Rp = tot + 2 * W;
+    const double* Rq = tot + 3 * W;
+    const House h = make_house(Rp[t], G1[t]);
+    bool two = false;
+    House h2{0.0, 0.0, 0.0};
+    double cq = 0.0, rqp = 0.0, g1pq = 0.0;
+    if (pair) {
+      const double wq = Rp[t + 1] + h.scale * G1[t + 1];
+      cq = h.tau * h.scale * wq;
+      rqp = Rq[t];
+      g1pq = G1[t] - rqp * rqp;
+      const double t1 = G2[t + 1], t2 = 2.0 * cq * G2[t], t3 = cq * cq * g1pq;
+      const double sig2 = t1 - t2 + t3;
+      two = sig2 >= 0.0625 * (fabs(t1) + fabs(t2) + cq * cq * (G1[t] + rqp * rqp));
+      if (two) h2 = make_house(Rq[t + 1] - cq * rqp, sig2);
+    }
+    double cj[CPW], tw[CPW], dj[CPW], tw2[CPW];
+#pragma unroll
+    for (int c = 0; c < CPW; ++c) {
+      const int j = j0 + c;
+      const double wj = Rp[j] + h.scale * G1[j];
+      cj[c] = h.tau * h.scale * wj;
+      tw[c] = -h.tau * wj;
+      dj[c] = 0.0;
+      tw2[c] = 0.0;
+      if (two) {
+        const double ajq = Rq[j] - cj[c] * rqp;
+        const double sj = G2[j] - cj[c] * G2[t] - cq * (G1[j] - rqp * Rq[j]) + cq * cj[c] * g1pq;
+        const double w2 = ajq + h2.scale * sj;
+        dj[c] = h2.tau * h2.scale * w2;
+        tw2[c] = -h2.tau * w2;
+      }
+    }
+    if (!two) {
+      // reflector t alone (as panel_reg_kernel)
+      if (j0 > t) {
+#pragma unroll
+        for (int q = 0; q < PR_RL; ++q) {
+          const int i = lane + 32 * q;
+          const int64_t r = rlo + i;
+          if (i < nr && r >= t) {
+            const double vr = r > t ? h.scale * x1[i] : 1.0;
+#pragma unroll
+            for (int c = 0; c < CPW; ++c) P[q][c] = fma(tw[c], vr, P[q][c]);
+          }
+        }
+      } else if (j0 + CPW > t) {
+#pragma unroll
+        for (int q = 0; q < PR_RL; ++q) {
+          const int i = lane + 32 * q;
+          const int64_t r = rlo + i;
+          if (i >= nr || r < t) continue;
+          const double vr = r > t ? h.scale * x1[i] : 1.0;
+#pragma unroll
+          for (int c = 0; c < CPW; ++c) {
+            const int j = j0 + c;
+            if (j > t) P[q][c] = fma(tw[c], vr, P[q][c]);
+            else if (j == t) P[q][c] = r > t ? vr : h.beta;
+          }
+        }
+      }
+    } else {
+      const int q1 = t + 1;
+      if (j0 > q1) {
+        // every column right of q: a'' = a - c_j a_p - d_j a'_q below q; row q: a - c_j a_p(q) - tau' w'_j;
+        // row p: a - tau w_j
+#pragma unroll
+        for (int q = 0; q < PR_RL; ++q) {
+          const int i = lane + 32 * q;
+          const int64_t r = rlo + i;
+          if (i < nr && r >= t) {
+            const double xp = x1[i];
+            const double aq = x2[i] - cq * xp;
+            if (r > q1) {
+#pragma unroll
+              for (int c = 0; c < CPW; ++c) P[q][c] = fma(-dj[c], aq, fma(-cj[c], xp, P[q][c]));
+            } else if (r == q1) {
+#pragma unroll
+              for (int c = 0; c < CPW; ++c) P[q][c] = fma(-cj[c], xp, P[q][c]) + tw2[c];
+            } else {
+#pragma unroll
+              for (int c = 0; c < CPW; ++c) P[q][c] += tw[c];
+            }
+          }
+        }
+      } else if (j0 + CPW > t) {
+#pragma unroll
+        for (int q = 0; q < PR_RL; ++q) {
+          const int i = lane + 32 * q;
+          const int64_t r = rlo + i;
+          if (i >= nr || r < t) continue;
+          const double xp = x1[i];
+          const double aq = x2[i] - cq * xp;
+#pragma unroll
+          for (int c = 0; c < CPW; ++c) {
+            const int j = j0 + c;
+            if (j > q1) {
+              if (r > q1) P[q][c] = fma(-dj[c], aq, fma(-cj[c], xp, P[q][c]));
+              else if (r == q1) P[q][c] = fma(-cj[c], xp, P[q][c]) + tw2[c];
+              else P[q][c] += tw[c];
+            } else if (j == q1) {
+              if (r > q1) P[q][c] = h2.scale * aq;
+              else if (r == q1) P[q][c] = h2.beta;
+              else P[q][c] += tw[c];
+            } else if (j == t) {
+              P[q][c] = r > t ? h.scale * xp : h.beta;
+            }
+          }
+        }
+      }
+    }
+    if (g == 0) {
+      // v_t^T v_s (s < t) as panel_reg_kernel; v_q^T v_s (s < q) from the pair's sums
+      for (int sp = tid; sp < t; sp += PR_NT) {
+        Dm[t * W + sp] = Rp[sp] + h.scale * G1[sp];
+        if (two) Dm[(t + 1) * W + sp] = Rq[sp] + h2.scale * (G2[sp] - cq * (G1[sp] - rqp * Rq[sp]));
+      }
+      if (tid == 0) {
+        taus[t] = h.tau;
+        a.tau[t] = h.tau;
+        if (two) {
+          Dm[(t + 1) * W + t] = h.scale * rqp + h2.scale * h.scale * (G2[t] - cq * g1pq);
+          taus[t + 1] = h2.tau;
+          a.tau[t + 1] = h2.tau;
+        }
+      }
+    }
+    tp0 = t;
+    tp1 = two ? t + 1 : -1;
+    const int tn = t + (two ? 2 : 1);
+    // next pair of columns -> the other parity's buffers (their previous readers finished before this barrier)
+#pragma unroll
+    for (int cc = 0; cc < 2; ++cc) {
+      const int col = tn + cc;
+      if (col < a.w && warp == col / CPW) {
+        double* xn = xsb + (2 * (par ^ 1) + cc) * XS;
+        const int cn = col % CPW;
+#pragma unroll
+        for (int q = 0; q < PR_RL; ++q) {
+          double v = 0.0;
+#pragma unroll
+          for (int c = 0; c < CPW; ++c)
+            if (c == cn) v = P[q][c];
+          xn[lane + 32 * q] = v;
+        }
+      }
+    }
+    t = tn;
+    par ^= 1;
+    __syncthreads();
+  }
+  if (g == 0) {
+    // T columns of the last step
+    for (int pass = 0; pass < 2; ++pass) {
+      const int c = pass ? tp1 : tp0;
+      if (c >= 0) t_column(Ts, Dm, taus, c, W, tid);
+      __syncthreads();
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < PR_RL; ++q) {
+    const int i = lane + 32 * q;
+    if (i >= nr) continue;
+    const int64_t r = rlo + i;
+#pragma unroll
+    for (int c = 0; c < CPW; ++c) {
+      const int j = j0 + c;
+      if (j < a.w) a.P[r + (int64_t)j * a.ldp] = P[q][c];
+      if (j < a.kk) a.Y[r + (int64_t)j * a.ldy] = r > j ? P[q][c] : (r == j ? 1.0 : 0.0);
+    }
+  }
+  if (g == 0) {
+    for (int idx = tid; idx < W * W; idx += PR_NT) {
+      const int q2 = idx % W, c = idx / W;
+      a.T[q2 + (int64_t)c * a.ldt] = (c < a.kk) ? Ts[q2 + c * W] : 0.0;
+    }
+  }
+  cl.sync();
+}
+
+size_t panel_reg_gpart_bytes(int w) { return sizeof(double) * 2 * PR_MAXNC * 4 * (size_t)w; }
+
+// TRID_PANEL_PAIR=0 selects the one-reflector-per-barrier kernel (A/B); default: two per barrier
+static bool panel_pair() {
+  static const bool on = !(getenv("TRID_PANEL_PAIR") && getenv("TRID_PANEL_PAIR")[0] == '0');
+  return on;
+}
 static size_t panel_reg_smem(int w) {
+  if (panel_pair()) return sizeof(double) * (size_t)(4 * 32 * PR_RL + 3 * 4 * w + 2 * w * w + w);
   return sizeof(double) * (size_t)(2 * 32 * PR_RL + 2 * 2 * w + 2 * w + 2 * w * w + w + 2 * w);
 }
 static const void* panel_reg_fn(int w) {
+  if (panel_pair())
+    return w == 16 ? (const void*)panel_reg2_kernel<2>
+                   : (w == 32 ? (const void*)panel_reg2_kernel<4> : (const void*)panel_reg2_kernel<8>);
   return w == 16 ? (const void*)panel_reg_kernel<2>
                  : (w == 32 ? (const void*)panel_reg_kernel<4> : (const void*)panel_reg_kernel<8>);
 }
@@ -394,6 +780,13 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   cfg.numAttrs = profiler_attached() ? 1 : 2;
   count_launches(1);
   auto launch = [&]() -> cudaError_t {
+    if (panel_pair()) {
+      switch (w) {
+        case 16: return cudaLaunchKernelEx(&cfg, panel_reg2_kernel<2>, a);
+        case 32: return cudaLaunchKernelEx(&cfg, panel_reg2_kernel<4>, a);
+        default: return cudaLaunchKernelEx(&cfg, panel_reg2_kernel<8>, a);
+      }
+    }
     switch (w) {
       case 16: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<2>, a);
       case 32: return cudaLaunchKernelEx(&cfg, panel_reg_kernel<4>, a);

@@ -1,7 +1,7 @@
 #!/bin/bash
-O=gpurun_out/r02p2; mkdir -p $O
+O=gpurun_out/r02p4; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -k "panel or dbbr or two_stage" > $O/pytest.log 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py -q --timeout 300 -k "panel or dbbr or two_stage" > $O/pytest.log 2>&1
 echo "pytest rc=$?" >> $O/pytest.log
 timeout 900 python -m pytest tests/test_gpu_parity_large.py tests/test_gpu_fullsize.py -q > $O/pytest_large.log 2>&1
 echo "pytest rc=$?" >> $O/pytest_large.log
