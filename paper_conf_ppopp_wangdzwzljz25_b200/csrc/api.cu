@@ -75,12 +75,14 @@ int default_k(int64_t n, int b) {
 }
 
 // largest SYMM split-K partial footprint over all panels of the reduction
-int64_t max_symm_part(int64_t n, int b) {
+int64_t max_symm_part(int64_t n, int b, int k) {
   int64_t best = 0;
   for (int64_t j = 0; j + b + 1 < n; j += b) {
     const int64_t m = n - j - b;
     const int64_t kk = m < b ? m : b;
-    const int64_t e = symm_ws_part_elems(m, kk);
+    int64_t e = symm_ws_part_elems(m, kk);
+    const int64_t ef = symm_ws_part_elems(m, kk, j % k);   // with the block's corrections folded in
+    if (ef > e) e = ef;
     if (e > best) best = e;
   }
   return best;
@@ -114,7 +116,7 @@ DbbrWork carve_dbbr(void* base, int64_t n, int b, int k) {
   w.T = c.take<double>((size_t)b * b);
   w.U = c.take<double>((size_t)2 * k * b);   // [Z_<^T W; Y_<^T W], ld 2k
   w.S = c.take<double>((size_t)b * b);
-  int64_t pe = max_symm_part(n, b);
+  int64_t pe = max_symm_part(n, b, k);
   const int64_t tn = (int64_t)64 * k * b;  // split-K partials of the tall reductions (2k x b stacked)
   if (pe < tn) pe = tn;
   const int64_t sk = max_skinny_part(n, b, k);   // next-panel update / corrections split-K
@@ -144,13 +146,14 @@ cudaError_t gemm_skinny_k(GemmArgs g, cudaStream_t st) {
 
 // ---- the Z builder after the SYMM (a3): corrections for the block's earlier panels (R4e), S = W^T X,
 // Z_p = X - 1/2 Y_p S (Eq. (1)).  X (m x kk, ld ldx) holds A_blk W_p on entry and is updated.
+// folded: the corrections were already applied inside the SYMM launch (zy_panel), only S and Z remain.
 cudaError_t zy_tail(int64_t m, int kk, const double* Wp, int64_t ldw, const double* Yp, const double* Yprev,
                     const double* Zprev, int64_t ldyz, int64_t nprev, double* Zp, double* X, int64_t ldx, double* U,
                     int64_t ldu, double* S, int64_t lds, double* part, int64_t part_elems, unsigned* sem,
-                    cudaStream_t st) {
+                    cudaStream_t st, bool folded) {
   cudaError_t e;
   ProfScope ps(PROF_ZY, st);
-  if (nprev > 0) {
+  if (nprev > 0 && !folded) {
     // [U1; U2] = [Z_<^T W; Y_<^T W]   (TN, K = m, deterministic split-K; one launch, stacked rows)
     double* U1 = U;
     double* U2 = U + nprev;
@@ -217,12 +220,33 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
                      double* Zp, double* X, int64_t ldx, double* U, int64_t ldu, double* S, int64_t lds,
                      double* part, int64_t part_elems, unsigned* sem, cudaStream_t st) {
   cudaError_t e;
-  {
+  // Default: the corrections X -= Y_< U1 + Z_< U2 ride in the SYMM launch as two extra K segments (U computed
+  // first, negated); TRID_ZY_FOLD=0 keeps them as a separate split-K launch after the SYMM (zy_tail).
+  static const bool fold = !(getenv("TRID_ZY_FOLD") && getenv("TRID_ZY_FOLD")[0] == '0') &&
+                           !(getenv("TRID_ZY_WS") && getenv("TRID_ZY_WS")[0] == '0');
+  const bool folded = fold && nprev > 0;
+  if (folded) {
+    double* U1 = U;
+    double* U2 = U + nprev;
+    {
+      ProfScope ps(PROF_ZY, st);
+      // [U1; U2] = -[Z_<^T W; Y_<^T W]   (TN, K = m, deterministic split-K)
+      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Zprev, ldyz, Wp, ldw, 0.0, U1, ldu, part, part_elems,
+                          st)) != cudaSuccess)
+        return e;
+      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Yprev, ldyz, Wp, ldw, 0.0, U2, ldu, part, part_elems,
+                          st)) != cudaSuccess)
+        return e;
+    }
+    ProfScope ps(PROF_SYMM, st);
+    e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st, nprev, Yprev, U1, Zprev, U2, ldyz, ldu);
+  } else {
     ProfScope ps(PROF_SYMM, st);
     e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st);
   }
   if (e != cudaSuccess) return e;
-  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U, ldu, S, lds, part, part_elems, sem, st);
+  return zy_tail(m, kk, Wp, ldw, Yp, Yprev, Zprev, ldyz, nprev, Zp, X, ldx, U, ldu, S, lds, part, part_elems, sem, st,
+                 folded);
 }
 
 int check_common(int64_t n, const void* A, int64_t lda, int b) {

@@ -68,11 +68,14 @@ cudaError_t gemm_ws_op(GemmArgs a, int opA, int opB, cudaStream_t st);
 cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
                        const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
                        int64_t part_elems, cudaStream_t st);
-int64_t symm_ws_splits(int64_t m, int64_t w);
+// nc: columns of each of the two correction segments folded into the SYMM's K axis (0: none)
+int64_t symm_ws_splits(int64_t m, int64_t w, int64_t nc = 0);
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K);
-int64_t symm_ws_part_elems(int64_t m, int64_t w);
+int64_t symm_ws_part_elems(int64_t m, int64_t w, int64_t nc = 0);
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
-                    int64_t ldx, double* part, int64_t part_elems, cudaStream_t st);
+                    int64_t ldx, double* part, int64_t part_elems, cudaStream_t st, int64_t nc = 0,
+                    const double* CA0 = nullptr, const double* CB0 = nullptr, const double* CA1 = nullptr,
+                    const double* CB1 = nullptr, int64_t ldca = 0, int64_t ldcb = 0);
 
 // Multi-GPU SYMM partials over a rank's local trailing columns (nqt of them, A_loc rows = global rows).
 int64_t symm_mg_part_elems(int64_t m, int64_t w, int64_t nqt);

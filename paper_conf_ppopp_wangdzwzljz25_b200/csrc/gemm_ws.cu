@@ -63,6 +63,11 @@ struct WsArgs {
   const double* B[2];
   int64_t lda[2], ldb[2], K[2];
   int symm;                 // 1: SYMM X = Asym W (A lower referenced), segments derived per tile
+  // symm == 1 only: ncorr > 0 appends two GEMM K-segments CA[i] (M x ncorr, op N, ld ldca) x CB[i] (ncorr x N,
+  // op N, ld ldcb) to every row block's K axis (the Z builder's corrections, R4e), chunked across the splits
+  int64_t ncorr, ldca, ldcb;
+  const double* CA[2];
+  const double* CB[2];
   double alpha, beta;
   const double* Cin;
   int64_t ldcin;
@@ -178,10 +183,12 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
     return 1;
   }
   if (a.symm) {
-    // K chunk z of the strip: [k0, k1); row strip (k <= row) then column strip (k > row)
-    const int64_t chunk = (a.K[0] + a.splits - 1) / a.splits;
+    // K chunk z of the strip (+ correction segments): [k0, k1); row strip (k <= row) then column strip (k > row)
+    const int64_t ktot = a.K[0] + 2 * a.ncorr;
+    const int64_t chunk = (ktot + a.splits - 1) / a.splits;
     const int64_t cz = (chunk + BK - 1) / BK * BK;
     const int64_t k0 = (int64_t)z * cz, k1 = (k0 + cz < a.K[0]) ? k0 + cz : a.K[0];
+    if (k0 >= a.K[0]) return 0;
     const int64_t e1 = (k1 < m0 + BM) ? k1 : m0 + BM;
     const int64_t s2 = (k0 > m0) ? k0 : m0;
     const Seg row{a.A[0], a.B[0], a.lda[0], a.ldb[0], k0, e1, OP_N, 1, 0, 0};
@@ -218,6 +225,20 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
   }
   s0 = g1;
   return ke1 > kb1 ? 1 : 0;
+}
+
+// Correction segment i (0, 1) of unit chunk z (symm == 1, ncorr > 0): the part of [m + i ncorr, m + (i+1) ncorr)
+// inside the chunk, in the segment's own k coordinates.
+__device__ __forceinline__ bool corr_seg(const WsArgs& a, int z, int i, Seg& sg) {
+  const int64_t ktot = a.K[0] + 2 * a.ncorr;
+  const int64_t chunk = (ktot + a.splits - 1) / a.splits;
+  const int64_t cz = (chunk + BK - 1) / BK * BK;
+  const int64_t k0 = (int64_t)z * cz, k1 = (k0 + cz < ktot) ? k0 + cz : ktot;
+  const int64_t s0 = a.K[0] + i * a.ncorr, s1 = s0 + a.ncorr;
+  const int64_t b0 = k0 > s0 ? k0 : s0, e0 = k1 < s1 ? k1 : s1;
+  if (e0 <= b0) return false;
+  sg = Seg{a.CA[i], a.CB[i], a.ldca, a.ldcb, b0 - s0, e0 - s0, OP_N, 0, 0, 0};
+  return true;
 }
 
 __device__ __forceinline__ void cp16(double* dst, const double* src, int bytes) {
@@ -469,6 +490,13 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
       };
       if (ns > 0) run(s0);
       if (ns > 1) run(s1);
+      if constexpr (BN == 64 && OPB == OP_N && !MG) {   // the SYMM instantiation only
+        if (a.ncorr) {
+          Seg c;
+          if (corr_seg(a, z, 0, c)) run(c);
+          if (corr_seg(a, z, 1, c)) run(c);
+        }
+      }
     }
     return;
   }
@@ -504,6 +532,13 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
     };
     if (ns > 0) run(s0);
     if (ns > 1) run(s1);
+    if constexpr (BN == 64 && OPB == OP_N && !MG) {   // the SYMM instantiation only
+      if (a.ncorr) {
+        Seg c;
+        if (corr_seg(a, z, 0, c)) run(c);
+        if (corr_seg(a, z, 1, c)) run(c);
+      }
+    }
     // ---- epilogue.  Cin may alias C, so a load issued after a store of the same thread could not be hoisted
     // above it by the compiler (one dependent global round trip per element); the Cin values of EN
     // fragments are loaded first, then combined and stored (MT * NT / EN round trips per tile instead of 64;
@@ -682,7 +717,7 @@ int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {
 // write 1 partial, 5 TB/s).  Pure function of (m, w) and fixed constants (the workspace sizing and the
 // deterministic sums use it), memoized.  The former rule (>= 8 waves, K >= 512 per split) left up to 9% of the
 // last wave idle at some m (e.g. m = 28608: 1344 units = 9.08 waves).  env TRID_SYMM_WAVES=W restores it.
-static int64_t symm_splits_model(int64_t m, int64_t w) {
+static int64_t symm_splits_model(int64_t m, int64_t w, int64_t nc) {
   const int64_t tm = (m + 127) / 128, rows = tm * ((w + 63) / 64);
   int64_t maxs = (m + 255) / 256 < 32 ? (m + 255) / 256 : 32;
   const int64_t maxw = (24 * kNumSMsB200 + rows - 1) / rows;   // <= ~24 waves (bounds the search)
@@ -691,12 +726,13 @@ static int64_t symm_splits_model(int64_t m, int64_t w) {
   int64_t bs = 1;
   double load[kNumSMsB200];
   for (int64_t sp = 1; sp <= maxs; ++sp) {
-    const int64_t chunk = (m + sp - 1) / sp, cz = (chunk + 15) / 16 * 16;
+    const int64_t kt = m + 2 * nc;   // strip + correction segments
+    const int64_t chunk = (kt + sp - 1) / sp, cz = (chunk + 15) / 16 * 16;
     for (int c = 0; c < kNumSMsB200; ++c) load[c] = 0.0;
     const int64_t units = rows * sp;
     for (int64_t u = 0; u < units; ++u) {
       const int64_t z = u / rows, t = (u % rows) % tm;
-      const int64_t k0 = z * cz, k1 = k0 + cz < m ? k0 + cz : m;
+      const int64_t k0 = z * cz, k1 = k0 + cz < kt ? k0 + cz : kt;
       double kk = k1 > k0 ? (double)(k1 - k0) : 0.0;
       const int64_t d0 = t * 128, d1 = d0 + 128 < m ? d0 + 128 : m;   // diagonal block, counted by both strips
       const int64_t o0 = k0 > d0 ? k0 : d0, o1 = k1 < d1 ? k1 : d1;
@@ -714,7 +750,7 @@ static int64_t symm_splits_model(int64_t m, int64_t w) {
   return bs;
 }
 
-int64_t symm_ws_splits(int64_t m, int64_t w) {
+int64_t symm_ws_splits(int64_t m, int64_t w, int64_t nc) {
   static const char* wv = getenv("TRID_SYMM_WAVES");
   if (wv) {
     const int64_t rows = (m + 127) / 128 * ((w + 63) / 64);
@@ -727,32 +763,39 @@ int64_t symm_ws_splits(int64_t m, int64_t w) {
   if (m <= 0 || w <= 0) return 1;
   static std::mutex mu;
   static std::unordered_map<int64_t, int64_t> memo;
-  const int64_t key = m * 4096 + w;
+  const int64_t key = (m * 4096 + w) * 8192 + nc;
   {
     std::lock_guard<std::mutex> lk(mu);
     auto it = memo.find(key);
     if (it != memo.end()) return it->second;
   }
-  const int64_t sp = symm_splits_model(m, w);
+  const int64_t sp = symm_splits_model(m, w, nc);
   std::lock_guard<std::mutex> lk(mu);
   memo[key] = sp;
   return sp;
 }
-int64_t symm_ws_part_elems(int64_t m, int64_t w) {
-  const int64_t sp = symm_ws_splits(m, w);
+int64_t symm_ws_part_elems(int64_t m, int64_t w, int64_t nc) {
+  const int64_t sp = symm_ws_splits(m, w, nc);
   return sp > 1 ? sp * m * w : 0;
 }
 
-// X = Asym W on the warp-specialized engine (row strip + transposed column strip per row block).
+// X = Asym W (+ CA0 CB0 + CA1 CB1 when nc > 0) on the warp-specialized engine (row strip + transposed column strip
+// per row block, then the two correction segments, all in one K axis chunked across the splits).
 cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const double* W, int64_t ldw, double* X,
-                    int64_t ldx, double* part, int64_t part_elems, cudaStream_t st) {
+                    int64_t ldx, double* part, int64_t part_elems, cudaStream_t st, int64_t nc, const double* CA0,
+                    const double* CB0, const double* CA1, const double* CB1, int64_t ldca, int64_t ldcb) {
   if (m <= 0 || w <= 0) return cudaSuccess;
   ws::WsArgs a{};
   a.M = m; a.N = w; a.opb = OP_N; a.nseg = 1; a.symm = 1;
   a.A[0] = A; a.B[0] = W; a.lda[0] = lda; a.ldb[0] = ldw; a.K[0] = m;
   a.vec16 = ws::al16(A) && ws::al16(W) && !(lda & 1) && !(ldw & 1);
+  if (nc > 0) {
+    a.ncorr = nc; a.CA[0] = CA0; a.CB[0] = CB0; a.CA[1] = CA1; a.CB[1] = CB1; a.ldca = ldca; a.ldcb = ldcb;
+    a.vec16 = a.vec16 && ws::al16(CA0) && ws::al16(CA1) && ws::al16(CB0) && ws::al16(CB1) && !(ldca & 1) &&
+              !(ldcb & 1);
+  }
   a.alpha = 1.0; a.beta = 0.0; a.C = X; a.ldc = ldx;
-  int64_t sp = symm_ws_splits(m, w);
+  int64_t sp = symm_ws_splits(m, w, nc > 0 ? nc : 0);
   if (sp * m * w > part_elems) sp = part_elems / (m * w);
   if (sp < 1) sp = 1;
   a.splits = (int)sp;
