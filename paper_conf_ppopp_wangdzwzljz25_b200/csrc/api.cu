@@ -88,15 +88,11 @@ int64_t max_symm_part(int64_t n, int b, int k) {
   return best;
 }
 
-// largest split-K partial footprint of the skinny engine GEMMs (M = m, N = b, K <= 2k)
+// split-K partial footprint bound of the skinny engine GEMMs (M = m <= n - b, N = b, <= 16 splits)
 int64_t max_skinny_part(int64_t n, int b, int k) {
-  int64_t best = 0;
-  for (int64_t j = 0; j + b + 1 < n; j += b) {
-    const int64_t m = n - j - b;
-    const int64_t e = (int64_t)ws_skinny_splits(m, b, 2 * (int64_t)k) * m * b;
-    if (e > best) best = e;
-  }
-  return best;
+  (void)k;
+  const int64_t m = n - b > 0 ? n - b : 0;
+  return (int64_t)16 * m * b;
 }
 
 struct DbbrWork {

@@ -22,7 +22,11 @@
 
 #include <stdlib.h>
 
+#include <stdint.h>
+#include <stdio.h>
+
 #include <mutex>
+#include <string>
 #include <unordered_map>
 
 namespace trid {
@@ -678,19 +682,79 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 
-// C (M x N) = alpha op(A) op(B) + beta Cin with a fixed split-K count (deterministic sums) when the output grid is
-// small: ~3 waves of units, >= 256 of K per split, <= 64 splits, within part_elems partials.
+// Split-K count of a GEMM on the persistent engine from a makespan model (as for the SYMM below): units
+// u = z * tiles + t walked by 148 CTAs with stride 148, unit z covering K-tiles [z per, (z + 1) per) of the
+// ceil(K / 16) K-tiles; unit cost = K-tiles x 1.19 us (128 x 64 tile; 2.38 us for 128 x 128) + 2 us; + the split-K
+// reduction (read s + 1, write 1 partial at 5 TB/s, + 3 us launch).  Pure function of the shape and the caps
+// (deterministic sums; the workspace sizing uses it), memoized.  env TRID_SPLIT_MODEL=0 restores the former
+// rule (~3 waves of units, >= 256 of K per split).
+static int gemm_splits_model(int64_t M, int64_t N, int64_t K, int cap, int64_t part_cap) {
+  const int64_t bn = N <= 64 ? 64 : 128;
+  const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
+  const double ts = bn == 64 ? 1.19 : 2.38;
+  const int64_t kt = (K + 15) / 16;
+  double best = 1e300;
+  int bs = 1;
+  double load[kNumSMsB200];
+  for (int64_t sp = 1; sp <= cap && sp <= kt; ++sp) {
+    if (sp > 1 && sp * M * N > part_cap) break;
+    const int64_t per = (kt + sp - 1) / sp;
+    for (int c = 0; c < kNumSMsB200; ++c) load[c] = 0.0;
+    for (int64_t u = 0; u < tiles * sp; ++u) {
+      const int64_t z = u / tiles;
+      int64_t k = kt - z * per;
+      k = k < per ? k : per;
+      load[u % kNumSMsB200] += (k > 0 ? (double)k : 0.0) * ts + 2.0;
+    }
+    double mk = 0.0;
+    for (int c = 0; c < kNumSMsB200; ++c) mk = load[c] > mk ? load[c] : mk;
+    if (sp > 1) mk += (double)(sp + 2) * (double)M * (double)N * 8.0 / 5.0e6 + 3.0;
+    if (mk < best * 0.999) {
+      best = mk;
+      bs = (int)sp;
+    }
+  }
+  return bs;
+}
+static bool split_model_on() {
+  static const bool on = !(getenv("TRID_SPLIT_MODEL") && getenv("TRID_SPLIT_MODEL")[0] == '0');
+  return on;
+}
+static int gemm_splits(int64_t M, int64_t N, int64_t K, int cap, int64_t part_cap) {
+  static std::mutex mu;
+  static std::unordered_map<std::string, int> memo;
+  char key[96];
+  snprintf(key, sizeof key, "%lld/%lld/%lld/%d/%lld", (long long)M, (long long)N, (long long)K, cap,
+           (long long)part_cap);
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = memo.find(key);
+    if (it != memo.end()) return it->second;
+  }
+  const int sp = gemm_splits_model(M, N, K, cap, part_cap);
+  std::lock_guard<std::mutex> lk(mu);
+  memo[key] = sp;
+  return sp;
+}
+
+// C (M x N) = alpha op(A) op(B) + beta Cin with a split-K count (deterministic sums) from the makespan model,
+// within part_elems partials and <= 64 splits.
 cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
                        const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
                        int64_t part_elems, cudaStream_t st) {
   if (M <= 0 || N <= 0) return cudaSuccess;
-  const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
-  int64_t s = (3 * kNumSMsB200 + tiles - 1) / tiles;
-  const int64_t maxk = K / 256;
-  if (s > maxk) s = maxk;
-  if (s > 64) s = 64;
-  if (s > 1 && s * M * N > part_elems) s = part_elems / (M * N);
-  if (s < 1) s = 1;
+  int64_t s;
+  if (split_model_on()) {
+    s = gemm_splits(M, N, K, 64, part_elems);
+  } else {
+    const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
+    s = (3 * kNumSMsB200 + tiles - 1) / tiles;
+    const int64_t maxk = K / 256;
+    if (s > maxk) s = maxk;
+    if (s > 64) s = 64;
+    if (s > 1 && s * M * N > part_elems) s = part_elems / (M * N);
+    if (s < 1) s = 1;
+  }
   GemmArgs g;
   g.M = M; g.N = N; g.K[0] = K; g.A[0] = A; g.lda[0] = lda; g.B[0] = B; g.ldb[0] = ldb;
   g.alpha = alpha; g.beta = beta; g.Cin = C; g.ldcin = ldc; g.C = C; g.ldc = ldc;
@@ -699,9 +763,10 @@ cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double
   return gemm_ws_op(g, opA, opB, st);
 }
 
-// Split-K for the skinny engine GEMMs (M = trailing rows, N = b, K = 2 x block columns): enough units for
-// ~3 waves of the persistent grid, >= 256 of K per split, <= 16 splits.  Partials: splits * M * N doubles.
+// Split-K for the skinny engine GEMMs (M = trailing rows, N = b, K = 2 x block columns): the makespan model with
+// <= 16 splits (the former rule: ~3 waves of units, >= 256 of K per split).  Partials: splits * M * N doubles.
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K) {
+  if (split_model_on()) return gemm_splits(M, N, K, 16, INT64_MAX);
   const int64_t tiles = ((M + 127) / 128) * ((N + (N <= 64 ? 63 : 127)) / (N <= 64 ? 64 : 128));
   int64_t sp = (3 * kNumSMsB200 + tiles - 1) / tiles;   // fixed (not the device's): sizes workspaces, fixes sums
   const int64_t maxs = K / 256;

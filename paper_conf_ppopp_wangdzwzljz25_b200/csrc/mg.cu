@@ -290,9 +290,8 @@ struct MgWork {
 MgWork carve_mg(void* base, int64_t n, int b, int k, int g, int q) {
   const int64_t nq = local_cols(n, b, g, q);
   int64_t pe = (int64_t)32 * k * b;
-  for (int64_t j = 0; j + b + 1 < n; j += b) {
-    const int64_t m = n - j - b;
-    const int64_t e = (int64_t)ws_skinny_splits(m, b, 2 * (int64_t)k) * m * b;
+  {
+    const int64_t e = (int64_t)16 * (n - b) * b;   // skinny split-K bound (<= 16 splits, M <= n - b)
     if (e > pe) pe = e;
   }
   for (int64_t j = 0; j + b + 1 < n; j += b) {
