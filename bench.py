@@ -50,8 +50,10 @@ def peaks():
 
 
 # ------------------------------------------------------------------ algorithmic work (pure counting)
-def dbbr_flops(n, b, k):
-    """Per-class algorithmic flops of the DBBR loop structure (same loop bounds as Alg. 1 / R4)."""
+def dbbr_flops(n, b, k, fold=True):
+    """Per-class algorithmic flops of the DBBR loop structure (same loop bounds as Alg. 1 / R4).  fold: the Z
+    builder's corrections X -= Y_< U1 + Z_< U2 (4 m kk ncols flops, R4e) run inside the SYMM launch (the
+    single-GPU default, TRID_ZY_FOLD) and count towards its class."""
     fl = {"symm": 0.0, "syr2k": 0.0, "symm_launches": 0, "syr2k_launches": 0}
     i = 0
     while i + b + 1 < n:
@@ -59,7 +61,7 @@ def dbbr_flops(n, b, k):
         while j < i + k and j + b + 1 < n:
             m = n - j - b
             kk = min(b, m)
-            fl["symm"] += 2.0 * m * m * kk
+            fl["symm"] += 2.0 * m * m * kk + (4.0 * m * kk * ncols if fold else 0.0)
             fl["symm_launches"] += 1
             ncols += kk
             jlast = j
@@ -297,7 +299,7 @@ def main():
     ap.add_argument("--b", type=int, default=0)
     ap.add_argument("--k", type=int, default=-1)
     ap.add_argument("--nb", type=int, default=0)
-    ap.add_argument("--e2e-steps", type=int, default=1)
+    ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--ref-n", type=int, default=1024)
@@ -433,7 +435,8 @@ def main():
     t_sbr = sum(per[c][0] for c in trid.SBR_CLASSES)
 
     # roofline: the dominant DBBR contraction (largest time share) against the measured FP64 DMMA peak
-    fl = dbbr_flops(n, b, k)
+    fold = not sharded and os.environ.get("TRID_ZY_FOLD", "1")[:1] != "0"
+    fl = dbbr_flops(n, b, k, fold=fold)
     cand = {"symm": (fl["symm"], per["symm"]), "syr2k": (fl["syr2k"], per["syr2k"])}
     dom = max(cand, key=lambda c: cand[c][1][0])
     dflops, (dms, dcalls) = cand[dom]
@@ -491,28 +494,65 @@ def main():
         eh = torch.empty(max(n - 1, 1), dtype=torch.float64, pin_memory=True)
         th = torch.empty(n, dtype=torch.float64, pin_memory=True)
         torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        if ws > 1:
-            dist.barrier()
-        e0.record(stream)
-        for _ in range(args.e2e_steps):
-            A.copy_(Ah, non_blocking=True)
-            res = run(A)
+
+        def fetch(res):
             if res is not None:
                 dh.copy_(res[0], non_blocking=True)
                 eh.copy_(res[1][: max(n - 1, 1)], non_blocking=True)
                 th.copy_(res[2], non_blocking=True)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        ems = e0.elapsed_time(e1)
-        if ws > 1:
-            t = torch.tensor([ems], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
-        line["e2e"] = {"value": round(nmat * flop * args.e2e_steps / (ems * 1e-3) / 1e12, 4), "unit": "TFLOP/s",
+
+        def timed_e2e(pipelined):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            if ws > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0.record(stream)
+            if not pipelined:
+                for _ in range(args.e2e_steps):
+                    A.copy_(Ah, non_blocking=True)
+                    fetch(run(A))
+            else:
+                # serving pipeline: step i+1's H2D (copy stream, into the other device buffer) overlaps step i's
+                # compute; every step still copies its whole input from pinned host memory inside the region
+                bufs = (A, Abuf2)
+                cs = torch.cuda.Stream(device=dev)
+                ready = [torch.cuda.Event(), torch.cuda.Event()]
+                free = [torch.cuda.Event(), torch.cuda.Event()]
+                cs.wait_stream(stream)
+                with torch.cuda.stream(cs):
+                    bufs[0].copy_(Ah, non_blocking=True)
+                    ready[0].record(cs)
+                for i in range(args.e2e_steps):
+                    cur, nxt = i % 2, (i + 1) % 2
+                    if i + 1 < args.e2e_steps:
+                        with torch.cuda.stream(cs):
+                            if i >= 1:
+                                cs.wait_event(free[nxt])
+                            bufs[nxt].copy_(Ah, non_blocking=True)
+                            ready[nxt].record(cs)
+                    stream.wait_event(ready[cur])
+                    fetch(run(bufs[cur]))
+                    free[cur].record(stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ems = e0.elapsed_time(e1)
+            if ws > 1:
+                t = torch.tensor([ems], dtype=torch.float64, device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ems = float(t.item())
+            return nmat * flop * args.e2e_steps / (ems * 1e-3) / 1e12
+
+        Abuf2 = torch.empty_like(A) if not sharded else None
+        serial = timed_e2e(False)
+        piped = timed_e2e(True) if not sharded else None
+        line["e2e"] = {"value": round(piped if piped is not None else serial, 4), "unit": "TFLOP/s",
                        "h2d_bytes_per_step": 8 * A0.numel() * ws, "d2h_bytes_per_step": 8 * (n + (n - 1) + n) * nmat,
+                       "steps": args.e2e_steps,
+                       "mode": ("pipelined: step i+1's pinned H2D on a copy stream overlaps step i's compute "
+                                "(double-buffered device input)") if piped is not None else "serial",
+                       "serial_value": round(serial, 4),
                        "note": "V1/V2 reflectors stay device-resident for the back transformation"}
-        del Ah
+        del Ah, Abuf2
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(b, cfg["seed"])
     if rank == 0:
