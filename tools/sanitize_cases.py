@@ -1,6 +1,6 @@
 """Small hot-path invocations for compute-sanitizer (racecheck / synccheck / memcheck): the bulge chase (v6 at
 b = 32/64, bc_kernel at b = 128, serial and pipelined), the register and general panel kernels, and one small
-two-stage run.  Usage: compute-sanitizer --tool racecheck python tools/sanitize_cases.py"""
+two-stage run, the TMA-staged syr2k and a DBBR with the folded Z-builder corrections.  Usage: compute-sanitizer --tool racecheck python tools/sanitize_cases.py"""
 import os
 import sys
 
@@ -24,6 +24,12 @@ def main():
     for m, w in [(500, 64), (300, 32), (400, 128)]:
         P = np.random.default_rng(m).uniform(-1, 1, (m, w))
         trid.panel_qr(to_dev(P))
+    # the syr2k on the bulk-copy (TMA) producer path, and a DBBR whose Z builder folds the corrections into the SYMM
+    C = to_dev(trid_gen.random_symmetric_np(300, 5))
+    rng = np.random.default_rng(3)
+    trid.syr2k_lower(C, to_dev(rng.uniform(-1, 1, (300, 40))), to_dev(rng.uniform(-1, 1, (300, 40))))
+    A = to_dev(trid_gen.random_symmetric_np(600, 7))
+    trid.sbr_dbbr(A, 32, nb=8, k=128)
     A = to_dev(trid_gen.random_symmetric_np(256, 1001))
     trid.sytrd_2stage(A, 32, nb=8, k=64)
     torch.cuda.synchronize()
