@@ -44,28 +44,30 @@ def per_launch(rows):
 
 
 def classify(launches):
-    """Assign each launch a stage class using the per-panel launch order."""
+    """Assign each launch a stage class using the per-panel launch order (round 2, corrections folded into the
+    SYMM): panel, W = Y T, U1 = Z_<^T W (+ reduce), U2 = Y_<^T W (+ reduce), the SYMM with the correction K
+    segments (+ reduce), S = W^T X (gemm_kernel + reduce), Z, the next-panel update (ws_kernel<.., 1, 0>)."""
     cls = []
     ws_since_panel = 99
     for d in launches:
         nm = d["name"]
-        if "panel_reg_kernel" in nm or "panel_qr_kernel" in nm:
+        if "panel_" in nm:
             c = "panel_qr"
             ws_since_panel = 0
         elif "ws_kernel<128, 128" in nm:
             c = "syr2k"
         elif "ws_kernel" in nm:
             ws_since_panel += 1
-            if ws_since_panel == 1:
-                c = "wy"
-            elif ws_since_panel == 2:
-                c = "symm"
-            elif "ws_kernel<128, 64, 4, 2, 1>" in nm:
+            if "ws_kernel<128, 64, 4, 2, 1" in nm:
                 c = "next_panel"
+            elif ws_since_panel == 1:
+                c = "wy"
+            elif ws_since_panel == 4:
+                c = "symm"
             else:
                 c = "zy"
         elif "ws_reduce_kernel" in nm:
-            c = "symm" if ws_since_panel == 2 else "zy"
+            c = "symm" if ws_since_panel == 4 else "zy"
         elif "gemm_kernel" in nm or "reduce_partials" in nm:
             c = "zy"
         elif "bc_" in nm or "band_" in nm:
