@@ -20,6 +20,8 @@
 #include "gemm.cuh"
 #include "prof.cuh"
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <stdlib.h>
 
 #include <stdint.h>
@@ -56,6 +58,7 @@ struct Seg {
   int opa;          // OP_N / OP_T
   int mask;         // 0 none, 1 keep k <= row, 2 keep k > row (global row = m0 + r)
   int mapk, mapr;   // multi-GPU: compare cmap(k) / cmap(row) instead of k / row (block-cyclic local columns)
+  int seg;          // GEMM segment index (selects the segment's tensor maps)
 };
 
 struct WsArgs {
@@ -92,8 +95,12 @@ struct WsArgs {
   int mg_g, mg_q, mg_cb;
   int64_t mg_lofs, mg_gofs;
   // TMA-staged operands (GEMM segments with A op N and B op T, 128 x 128 tiles, vec16, even M and N: the
-  // deferred syr2k): the producer stages every k-row of a tile with one bulk copy (cp.async.bulk) per operand
+  // deferred syr2k): tma = 1: the producer stages every k-row of a tile with one bulk copy (cp.async.bulk) per
+  // operand; tma = 2: one tensor copy (cp.async.bulk.tensor.2d) per operand and stage, from the segment's tensor
+  // maps tmA / tmB (FP64, dims {rows, K}, box {BM + 4, BK}: the box lands as the padded [BK][BM + 4] stage layout;
+  // rows past M / N and k past K are zero-filled by the copy engine)
   int tma;
+  CUtensorMap tmA[2], tmB[2];
 };
 
 template <bool MG>
@@ -221,7 +228,7 @@ __device__ __forceinline__ int unit_segs(const WsArgs& a, int64_t m0, int z, Seg
     ke1 = (e * BK < a.K[1]) ? e * BK : a.K[1];
   }
   const Seg g0{a.A[0], a.B[0], a.lda[0], a.ldb[0], kb0, ke0, a.opa, 0, 0, 0};
-  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, a.opa, 0, 0, 0};
+  const Seg g1{a.A[1], a.B[1], a.lda[1], a.ldb[1], kb1, ke1, a.opa, 0, 0, 0, 1};
   if (ke0 > kb0) {
     s0 = g0;
     s1 = g1;
@@ -255,6 +262,14 @@ __device__ __forceinline__ void cp8(double* dst, const double* src, int bytes) {
 }
 __device__ __forceinline__ void cp_arrive_noinc(uint64_t* bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+// 2D tensor copy global -> shared (TMA), completing on an mbarrier; c0 = innermost (row) coordinate
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int c0, int c1, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
 }
 
 // ---- producer fast paths (16-byte aligned operands, no triangle mask): per-thread offsets are fixed,
@@ -406,7 +421,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
   constexpr int WTM = BM / CWM, WTN = BN / CWN;
   constexpr int MT = WTM / 16, NT = WTN / 8;
   constexpr int STAGES = C::STAGES;
-  extern __shared__ __align__(16) double smem[];
+  extern __shared__ __align__(128) double smem[];   // 128-byte aligned stages (tensor copies)
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)STAGES * C::STAGE);
   uint64_t* empty = full + STAGES;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -448,6 +463,17 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
               if (use > 0) mbar_wait(&empty[slot], (use - 1) & 1u);
               double* As = smem + (size_t)slot * C::STAGE;
               double* Bs = As + C::A_ELEMS;
+              if (a.tma == 2) {
+                // one tensor copy per operand: box {BM + 4, BK} at (row m0 / n0, k0) of the segment's maps
+                if (pt == 0) {
+                  mbar_arrive_expect_tx(&full[slot], (unsigned)(2 * BK * (BM + 4) * 8));
+                  tma_load_2d(As, &a.tmA[sgm.seg], (int)m0, (int)k0, &full[slot]);
+                  tma_load_2d(Bs, &a.tmB[sgm.seg], (int)n0, (int)k0, &full[slot]);
+                } else {
+                  mbar_arrive(&full[slot]);
+                }
+                continue;
+              }
               const int kc = (int)((sgm.ke - k0) < BK ? (sgm.ke - k0) : BK);
               if (kc < BK || rm < BM || rn < BN) {
                 for (int kk = 0; kk < BK; ++kk) {
@@ -645,6 +671,28 @@ static cudaError_t launch(WsArgs& a, cudaStream_t st) {
 
 static bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 
+// FP64 2D tensor map of a column-major operand X (rows x cols, leading dimension ld): dims {rows, cols}, box
+// {128 + 4, BK} (the engine's padded [BK][BM + 4] stage), no swizzle, out-of-bounds elements zero-filled.  The
+// driver entry point is resolved once through the runtime (no link against libcuda).
+static bool encode_rows_map(CUtensorMap* map, const double* X, int64_t rows, int64_t cols, int64_t ld) {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      p = nullptr;
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }();
+  if (!fn || rows <= 0 || cols <= 0 || rows >= (1ll << 31) || cols >= (1ll << 31)) return false;
+  const cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
+  const cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(double)};
+  const cuuint32_t box[2] = {128 + 4, BK};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(X), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 }  // namespace ws
 
 // C = alpha * sum_seg op(A_seg) op(B_seg) + beta * Cin; tile 128x128 (wide N) or 128x64 (N <= 64).  Same
@@ -677,8 +725,17 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   }
   // bulk-copy (TMA) staging for A op N / B op T on 128 x 128 tiles (the syr2k and the other NT contractions);
   // (measured: syr2k 70.7 -> 65.9 ms at n = 32768, k = 1024); env TRID_WS_TMA=0 restores the cp.async producer
+  // TRID_WS_TMA: 0 cp.async producer, 1 per-row bulk copies, 2 (default) tensor maps (cp.async.bulk.tensor)
   const char* tenv = getenv("TRID_WS_TMA");   // read per call (tests toggle it)
-  a.tma = (!tenv || atoi(tenv) != 0) && opA == OP_N && opB == OP_T && v16 && !(g.M & 1) && !(g.N & 1);
+  const int tmode = tenv ? atoi(tenv) : 2;
+  a.tma = (tmode != 0) && opA == OP_N && opB == OP_T && v16 && !(g.M & 1) && !(g.N & 1);
+  if (a.tma && tmode == 2) {
+    bool ok = true;
+    for (int i = 0; i < g.nseg && ok; ++i)
+      ok = ws::encode_rows_map(&a.tmA[i], g.A[i], g.M, g.K[i], g.lda[i]) &&
+           ws::encode_rows_map(&a.tmB[i], g.B[i], g.N, g.K[i], g.ldb[i]);
+    a.tma = ok ? 2 : 1;   // no driver entry point: the per-row bulk copies (same staged values)
+  }
   return opB == OP_T ? ws::launch<128, 128, 4, 2, OP_T>(a, st) : ws::launch<128, 128, 4, 2, OP_N>(a, st);
 }
 

@@ -47,22 +47,24 @@ def test_syr2k_lower_parity(m, kk, dev):
     assert np.array_equal(got[iu], C[iu])      # strict upper untouched, bitwise
 
 
-@pytest.mark.parametrize("m,kk", [(1000, 100), (512, 64), (258, 37), (2048, 256)])
+@pytest.mark.parametrize("m,kk", [(1000, 100), (512, 64), (258, 37), (2048, 256), (130, 3), (4100, 1024)])
 def test_syr2k_tma_staging_bitwise(m, kk, dev, monkeypatch):
-    """The bulk-copy (TMA) producer of the NT engine path stages the same tile values into the same padded
-    layout as the cp.async producer, so the consumers' DMMA order and the result are identical bit for bit
-    (ragged row tails m % 128 != 0 and ragged K tails kk % 16 != 0 included); both match the oracle."""
+    """The TMA producers of the NT engine path (2: one tensor copy per operand and stage from FP64 tensor maps,
+    out-of-bounds rows / k zero-filled by the copy engine; 1: one bulk copy per k-row) stage the same tile values
+    into the same padded layout as the cp.async producer (0), so the consumers' DMMA order and the result are
+    identical bit for bit (ragged row tails m % 128 != 0 and ragged K tails kk % 16 != 0 included); all match the
+    oracle."""
     rng = np.random.default_rng(m + 7 * kk)
     C = rng.uniform(-1, 1, (m, m))
     Y = rng.uniform(-1, 1, (m, kk))
     Z = rng.uniform(-1, 1, (m, kk))
     outs = []
-    for env in ("1", "0"):
+    for env in ("2", "1", "0"):
         monkeypatch.setenv("TRID_WS_TMA", env)
         Cd = to_dev(C)
         trid.syr2k_lower(Cd, to_dev(Y), to_dev(Z))
         outs.append(from_dev(Cd))
-    assert np.array_equal(outs[0], outs[1])
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
     ref = oracle.syr2k_lower(C, Y, Z)
     il = np.tril_indices(m)
     bound = 2 * 4 * (2 * kk + 1) * U * (np.abs(Y) @ np.abs(Z).T + np.abs(Z) @ np.abs(Y).T + np.abs(C))
@@ -71,15 +73,17 @@ def test_syr2k_tma_staging_bitwise(m, kk, dev, monkeypatch):
 
 @pytest.mark.parametrize("n,b", [(1024, 64), (1030, 32)])
 def test_dbbr_tma_staging_bitwise(n, b, dev, monkeypatch):
-    """DBBR with the bulk-copy producer equals DBBR with the cp.async producer bit for bit."""
+    """DBBR with either TMA producer (tensor maps, per-row bulk copies) equals DBBR with the cp.async producer bit
+    for bit."""
     A = trid_gen.random_symmetric_np(n, 4242 + n)
     outs = []
-    for env in ("1", "0"):
+    for env in ("2", "1", "0"):
         monkeypatch.setenv("TRID_WS_TMA", env)
         Ad = to_dev(A)
         tau = trid.sbr_dbbr(Ad, b, nb=min(16, b), k=4 * b)
         outs.append((from_dev(Ad), tau.cpu().numpy()))
-    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    for o in outs[1:]:
+        assert np.array_equal(outs[0][0], o[0]) and np.array_equal(outs[0][1], o[1])
 
 
 # ------------------------------------------------------------------------------------------ panel QR
