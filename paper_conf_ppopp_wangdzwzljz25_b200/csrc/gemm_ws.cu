@@ -520,7 +520,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
       };
       if (ns > 0) run(s0);
       if (ns > 1) run(s1);
-      if constexpr (BN == 64 && OPB == OP_N && !MG) {   // the SYMM instantiation only
+      if constexpr (BN <= 64 && OPB == OP_N && !MG) {   // the SYMM instantiations only
         if (a.ncorr) {
           Seg c;
           if (corr_seg(a, z, 0, c)) run(c);
@@ -562,7 +562,7 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
     };
     if (ns > 0) run(s0);
     if (ns > 1) run(s1);
-    if constexpr (BN == 64 && OPB == OP_N && !MG) {   // the SYMM instantiation only
+    if constexpr (BN <= 64 && OPB == OP_N && !MG) {   // the SYMM instantiations only
       if (a.ncorr) {
         Seg c;
         if (corr_seg(a, z, 0, c)) run(c);
@@ -671,10 +671,24 @@ static cudaError_t launch(WsArgs& a, cudaStream_t st) {
 
 static bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 
+// 128 x 32 tiles for N <= 32 (default on; TRID_WS_NARROW=0 falls back to 128 x 64 for A/B).  Read once: the
+// split counts (and hence the workspace sizes and the deterministic sums) depend on it.
+static bool narrow_tiles() {
+  static const bool on = !(getenv("TRID_WS_NARROW") && getenv("TRID_WS_NARROW")[0] == '0');
+  return on;
+}
+
 // FP64 2D tensor map of a column-major operand X (rows x cols, leading dimension ld): dims {rows, cols}, box
 // {128 + 4, BK} (the engine's padded [BK][BM + 4] stage), no swizzle, out-of-bounds elements zero-filled.  The
 // driver entry point is resolved once through the runtime (no link against libcuda).
+static bool encode_map(CUtensorMap* map, const double* X, int64_t rows, int64_t cols, int64_t ld, unsigned box0,
+                       unsigned box1);
 static bool encode_rows_map(CUtensorMap* map, const double* X, int64_t rows, int64_t cols, int64_t ld) {
+  return encode_map(map, X, rows, cols, ld, 128 + 4, BK);
+}
+// FP64 2D tensor map of a column-major X (rows x cols, ld), box {box0 rows, box1 columns}, no swizzle, OOB zero
+static bool encode_map(CUtensorMap* map, const double* X, int64_t rows, int64_t cols, int64_t ld, unsigned box0,
+                       unsigned box1) {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
     void* p = nullptr;
     cudaDriverEntryPointQueryResult q;
@@ -686,7 +700,7 @@ static bool encode_rows_map(CUtensorMap* map, const double* X, int64_t rows, int
   if (!fn || rows <= 0 || cols <= 0 || rows >= (1ll << 31) || cols >= (1ll << 31)) return false;
   const cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
   const cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(double)};
-  const cuuint32_t box[2] = {128 + 4, BK};
+  const cuuint32_t box[2] = {box0, box1};
   const cuuint32_t estr[2] = {1, 1};
   return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(X), dims, strides, box, estr,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -695,7 +709,8 @@ static bool encode_rows_map(CUtensorMap* map, const double* X, int64_t rows, int
 
 }  // namespace ws
 
-// C = alpha * sum_seg op(A_seg) op(B_seg) + beta * Cin; tile 128x128 (wide N) or 128x64 (N <= 64).  Same
+// C = alpha * sum_seg op(A_seg) op(B_seg) + beta * Cin; tile 128x128 (wide N), 128x64 (N <= 64) or 128x32 (N <= 32,
+// the b = 32 band: a 128x64 tile would multiply half zeros; warps 8x1 of 16x32).  Same
 // semantics as gemm().
 cudaError_t gemm_ws(GemmArgs g, int opB, cudaStream_t st) { return gemm_ws_op(g, OP_N, opB, st); }
 
@@ -719,6 +734,9 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   if (a.mg_g > 1) {   // multi-GPU column map (only the lower-masked syr2k of mg.cu uses it)
     if (opB != OP_T || opA != OP_N) return cudaErrorInvalidValue;
     return g.N <= 64 ? ws::launch<128, 64, 4, 2, OP_T, true>(a, st) : ws::launch<128, 128, 4, 2, OP_T, true>(a, st);
+  }
+  if (g.N <= 32 && ws::narrow_tiles()) {
+    return opB == OP_T ? ws::launch<128, 32, 8, 1, OP_T>(a, st) : ws::launch<128, 32, 8, 1, OP_N>(a, st);
   }
   if (g.N <= 64) {
     return opB == OP_T ? ws::launch<128, 64, 4, 2, OP_T>(a, st) : ws::launch<128, 64, 4, 2, OP_N>(a, st);
@@ -746,9 +764,9 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
 // (deterministic sums; the workspace sizing uses it), memoized.  env TRID_SPLIT_MODEL=0 restores the former
 // rule (~3 waves of units, >= 256 of K per split).
 static int gemm_splits_model(int64_t M, int64_t N, int64_t K, int cap, int64_t part_cap) {
-  const int64_t bn = N <= 64 ? 64 : 128;
+  const int64_t bn = (N <= 32 && ws::narrow_tiles()) ? 32 : (N <= 64 ? 64 : 128);
   const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
-  const double ts = bn == 64 ? 1.19 : 2.38;
+  const double ts = bn == 32 ? 0.60 : (bn == 64 ? 1.19 : 2.38);
   const int64_t kt = (K + 15) / 16;
   double best = 1e300;
   int bs = 1;
@@ -843,6 +861,7 @@ static int64_t symm_splits_model(int64_t m, int64_t w, int64_t nc) {
   const int64_t tm = (m + 127) / 128, rows = tm * ((w + 63) / 64);
   int64_t maxs = (m + 255) / 256 < 32 ? (m + 255) / 256 : 32;
   const int64_t maxw = (24 * kNumSMsB200 + rows - 1) / rows;   // <= ~24 waves (bounds the search)
+  const double ts = (w <= 32 && ws::narrow_tiles()) ? 0.60 : 1.19;   // us per 128 x BN x 16 stage
   if (maxs > maxw) maxs = maxw;
   double best = 1e300;
   int64_t bs = 1;
@@ -859,7 +878,7 @@ static int64_t symm_splits_model(int64_t m, int64_t w, int64_t nc) {
       const int64_t d0 = t * 128, d1 = d0 + 128 < m ? d0 + 128 : m;   // diagonal block, counted by both strips
       const int64_t o0 = k0 > d0 ? k0 : d0, o1 = k1 < d1 ? k1 : d1;
       if (o1 > o0) kk += (double)(o1 - o0);
-      load[u % kNumSMsB200] += kk / 16.0 * 1.19 + 2.0;
+      load[u % kNumSMsB200] += kk / 16.0 * ts + 2.0;
     }
     double mk = 0.0;
     for (int c = 0; c < kNumSMsB200; ++c) mk = load[c] > mk ? load[c] : mk;
@@ -922,6 +941,7 @@ cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const do
   if (sp < 1) sp = 1;
   a.splits = (int)sp;
   a.part = part; a.part_ld = m; a.part_stride = m * w;
+  if (w <= 32 && ws::narrow_tiles()) return ws::launch<128, 32, 8, 1, OP_N>(a, st);
   return ws::launch<128, 64, 4, 2, OP_N>(a, st);
 }
 
