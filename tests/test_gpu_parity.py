@@ -71,7 +71,7 @@ def test_syr2k_tma_staging_bitwise(m, kk, dev, monkeypatch):
     assert np.all(np.abs(outs[0] - ref)[il] <= bound[il])
 
 
-@pytest.mark.parametrize("n,b", [(1024, 64), (1030, 32)])
+@pytest.mark.parametrize("n,b", [(1024, 64), (1030, 32), (2101, 64), (1501, 16)])
 def test_dbbr_tma_staging_bitwise(n, b, dev, monkeypatch):
     """DBBR with either TMA producer (tensor maps, per-row bulk copies) equals DBBR with the cp.async producer bit
     for bit."""
