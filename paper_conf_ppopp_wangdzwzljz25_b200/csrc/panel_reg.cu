@@ -754,8 +754,14 @@ cudaError_t panel_qr_reg(int64_t m, int w, double* P, int64_t ldp, double* tau, 
   const size_t smem = panel_reg_smem(w);
   const int maxc = panel_reg_max_clusters(w);
   if (maxc < 1) return cudaErrorInvalidConfiguration;   // caller checks panel_reg_supported
-  // as few rows per CTA as possible within the co-resident clusters
-  int64_t G = (m + 63) / 64;
+  // as few rows per CTA as possible within the co-resident clusters (target 64 rows per CTA; env
+  // TRID_PANEL_ROWS=r for A/B: the grid barrier's cost grows with G, the per-column work with the rows)
+  static const int prow = [] {
+    const char* e = getenv("TRID_PANEL_ROWS");
+    const int v = e ? atoi(e) : 64;
+    return v >= 16 && v <= 32 * PR_RL ? v : 64;
+  }();
+  int64_t G = (m + prow - 1) / prow;
   G = (G + PR_CL - 1) / PR_CL * PR_CL;
   if (G > (int64_t)PR_CL * maxc) G = (int64_t)PR_CL * maxc;
   if (G < PR_CL) G = PR_CL;
