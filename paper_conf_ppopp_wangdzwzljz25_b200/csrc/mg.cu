@@ -454,6 +454,8 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
   if (dwork_bytes < w.bytes) return TRID_ERR_WORKSPACE;
   TRID_CUDA_TRY(cudaMemsetAsync(w.sem, 0, sizeof(unsigned) * 1024, st));
   const int64_t ld = n;   // Y, Z, W leading dimension
+  // row-sharded corrections (below); env TRID_MG_SHARD_CORR=0 (read per call, A/B and tests) repeats them per rank
+  const bool shard_env = !(getenv("TRID_MG_SHARD_CORR") && getenv("TRID_MG_SHARD_CORR")[0] == '0');
   int r;
   for (int64_t i = 0; i + b + 1 < n; i += k) {                       // l.1
     int64_t ncols = 0, jlast = i;
@@ -500,10 +502,41 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
         } else {
           TRID_CUDA_TRY(cudaMemsetAsync(w.X, 0, sizeof(double) * (size_t)ldx * kk, st));
         }
+      }
+      // Row-sharded corrections (R4e): every rank forms U = -[Z_<^T W; Y_<^T W] (Y, Z are replicated) and adds
+      // Y_<(its row slice) U1 + Z_<(slice) U2 to its partial X, so the all-reduce returns the corrected X and the
+      // correction GEMM (4 m b ncols flops per panel) is split over the g ranks instead of repeated on each one.
+      // env TRID_MG_SHARD_CORR=0: every rank applies the whole correction after the all-reduce (zy_tail).
+      const bool shard = shard_env && ncols > 0;
+      if (shard) {
+        ProfScope ps(PROF_ZY, st);
+        double* U1 = w.U;
+        double* U2 = w.U + ncols;
+        TRID_CUDA_TRY(gemm_ws_mm(OP_T, OP_N, ncols, kk, m, -1.0, w.Z + o, ld, w.W, ld, 0.0, U1, 2 * k, w.part,
+                                 w.part_elems, st));
+        TRID_CUDA_TRY(gemm_ws_mm(OP_T, OP_N, ncols, kk, m, -1.0, w.Y + o, ld, w.W, ld, 0.0, U2, 2 * k, w.part,
+                                 w.part_elems, st));
+        // contiguous row slices starting at even rows (16-byte aligned operands for the engine's fast producer)
+        const int64_t rlo = q == 0 ? 0 : (m * q / g) & ~(int64_t)1;
+        const int64_t rhi = q == g - 1 ? m : (m * (q + 1) / g) & ~(int64_t)1;
+        if (rhi > rlo) {
+          GemmArgs h;
+          h.M = rhi - rlo; h.N = kk; h.nseg = 2;
+          h.A[0] = w.Y + o + rlo; h.lda[0] = ld; h.B[0] = U1; h.ldb[0] = 2 * k; h.K[0] = ncols;
+          h.A[1] = w.Z + o + rlo; h.lda[1] = ld; h.B[1] = U2; h.ldb[1] = 2 * k; h.K[1] = ncols;
+          h.alpha = 1.0; h.beta = 1.0; h.Cin = w.X + rlo; h.ldcin = ldx; h.C = w.X + rlo; h.ldc = ldx;
+          h.splits = ws_skinny_splits(rhi - rlo, kk, 2 * ncols);
+          if ((int64_t)h.splits * (rhi - rlo) * kk > w.part_elems) h.splits = 1;
+          h.part = w.part; h.part_ld = rhi - rlo; h.part_stride = (rhi - rlo) * kk;
+          TRID_CUDA_TRY(gemm_ws(h, OP_N, st));
+        }
+      }
+      {
+        ProfScope ps(PROF_SYMM, st);
         if ((r = comm_sum(comm, w.X, ldx * kk, true, 0, st))) return r;   // padding rows ride along unread
       }
       TRID_CUDA_TRY(zy_tail(m, kk, w.W, ld, Yp, w.Y + o, w.Z + o, ld, ncols, Zp, w.X, ldx, w.U, 2 * k, w.S, b,
-                            w.part, w.part_elems, w.sem, st));
+                            w.part, w.part_elems, w.sem, st, shard));
       ncols += kk;                                                  // l.6
       jlast = j;
       const int64_t jn = j + b;

@@ -52,9 +52,13 @@ def run_mg(n, b, k, g, seed, nb=8):
     return full, [t.cpu().numpy() for t in taus], ABs[0]
 
 
+@pytest.mark.parametrize("shard", ["1", "0"])
 @pytest.mark.parametrize("n,b,k,g", [(256, 32, 64, 1), (256, 32, 64, 2), (300, 32, 96, 3), (300, 32, 64, 4),
                                      (513, 16, 64, 3), (1000, 64, 256, 2), (640, 64, 128, 5)])
-def test_mg_dbbr_parity(n, b, k, g, dev):
+def test_mg_dbbr_parity(n, b, k, g, shard, dev, monkeypatch):
+    """shard = 1 (default): the implicit-update corrections are split by rows over the ranks and ride in the X
+    all-reduce; 0: every rank applies them after it.  Both against the oracle's Alg. 1 (R4e)."""
+    monkeypatch.setenv("TRID_MG_SHARD_CORR", shard)
     A = trid_gen.random_symmetric_np(n, 1001)
     Ao, to = oracle.dbbr(A, b, k)
     full, taus, AB = run_mg(n, b, k, g, 1001)
