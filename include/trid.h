@@ -167,8 +167,9 @@ int trid_comm_rank(trid_comm_t comm);
 int64_t trid_mg_local_cols(int64_t n, int colblock, int nranks, int rank);
 int trid_sbr_dbbr_mg_bufsize(int64_t n, int b, int nb, int k, int nranks, int rank, size_t* dwork_bytes);
 /* Alg. 1 with the per-panel exchange of SURVEY 8(e): the panel owner's [Y_p | T | tau] is broadcast,
- * the partial X = A_blk W_p over each rank's stored entries is all-reduced (sum), the Z builder runs
- * redundantly, the next-panel update on the next panel's owner, the syr2k on every rank's own columns.
+ * the partial X = A_blk W_p over each rank's stored entries plus the rank's row slice of the implicit-update
+ * corrections (R4e) is all-reduced (sum), S and Z_p are formed redundantly, the next-panel update runs on the
+ * next panel's owner, the syr2k on every rank's own columns.
  * Out: as trid_sbr_dbbr, in the block-cyclic layout (band + SBR vectors in each owner's columns);
  * tau1[n] complete on every rank.  colblock must equal b. */
 int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A_local, int64_t lda_local, int colblock, int b, int nb,
@@ -203,7 +204,8 @@ int trid_panel_qr(int64_t m, int w, double* P, int64_t ldp, double* tau, double*
                   double* Y, int64_t ldy, void* dwork, size_t dwork_bytes, cudaStream_t stream);
 
 /* a5 / a4: C -= Y Z^T + Z Y^T on the lower triangle of the m x m matrix C (strict upper untouched);
- * Y, Z are m x kk.  The DMMA syr2k of Alg. 1 l.15 (Fig. 7). */
+ * Y, Z are m x kk.  The DMMA syr2k of Alg. 1 l.15 (Fig. 7); its tiles are staged by TMA tensor copies when the
+ * operands are 16-byte aligned with even leading dimensions and m is even (else by cp.async; same bits). */
 int trid_syr2k_lower(int64_t m, int64_t kk, double* C, int64_t ldc, const double* Y, int64_t ldy,
                      const double* Z, int64_t ldz, cudaStream_t stream);
 

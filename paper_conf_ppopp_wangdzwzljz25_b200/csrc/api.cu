@@ -226,13 +226,21 @@ cudaError_t zy_panel(int64_t m, int kk, const double* Atr, int64_t lda, const do
     double* U2 = U + nprev;
     {
       ProfScope ps(PROF_ZY, st);
-      // [U1; U2] = -[Z_<^T W; Y_<^T W]   (TN, K = m, deterministic split-K)
-      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Zprev, ldyz, Wp, ldw, 0.0, U1, ldu, part, part_elems,
-                          st)) != cudaSuccess)
-        return e;
-      if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Yprev, ldyz, Wp, ldw, 0.0, U2, ldu, part, part_elems,
-                          st)) != cudaSuccess)
-        return e;
+      // [U1; U2] = -[Z_<^T W; Y_<^T W]   (TN, K = m, deterministic split-K): ONE launch over the stacked operands
+      // (they share W; U2 = U1 + nprev in U's column); TRID_ZY_USTACK=0 runs the two products separately (A/B)
+      static const bool ustack = !(getenv("TRID_ZY_USTACK") && getenv("TRID_ZY_USTACK")[0] == '0');
+      if (ustack) {
+        if ((e = gemm_ws_mm(OP_T, OP_N, 2 * nprev, kk, m, -1.0, Zprev, ldyz, Wp, ldw, 0.0, U1, ldu, part, part_elems,
+                            st, Yprev, nprev)) != cudaSuccess)
+          return e;
+      } else {
+        if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Zprev, ldyz, Wp, ldw, 0.0, U1, ldu, part, part_elems,
+                            st)) != cudaSuccess)
+          return e;
+        if ((e = gemm_ws_mm(OP_T, OP_N, nprev, kk, m, -1.0, Yprev, ldyz, Wp, ldw, 0.0, U2, ldu, part, part_elems,
+                            st)) != cudaSuccess)
+          return e;
+      }
     }
     ProfScope ps(PROF_SYMM, st);
     e = symm_ws(m, kk, Atr, lda, Wp, ldw, X, ldx, part, part_elems, st, nprev, Yprev, U1, Zprev, U2, ldyz, ldu);

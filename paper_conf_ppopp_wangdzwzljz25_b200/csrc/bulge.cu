@@ -872,6 +872,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (tid == 0) wait_geq(a.prog_full + (s - 1), need_full);
         __syncthreads();
       }
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 0);
       if (a.opt & 64) bw_csync<CS>();   // debug (TRID_BC_OPT): extra cluster barriers
       // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j); the last one after
       // its producer published it
@@ -908,6 +909,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       }
       asm volatile("cp.async.wait_group 0;\n" ::: "memory");   // the body columns
       __syncthreads();
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 1);
       if (a.opt & 128) bw_csync<CS>();
       // ---- 1. partial matvec [D; O] v over my BODY columns (all but the window's last, which sweep s-1 may still
       //      be producing), all H rows; the last column's terms are added once it arrives
@@ -945,6 +947,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (tid == 0) wait_geq(a.prog + (s - 1), need_c0);
         __syncthreads();
       }
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 2);
       if (own_last && warp == (L - 1 - cbeg) % NW) load_col(L - 1);
       asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
       __syncthreads();
@@ -955,6 +958,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           for (int i = L - 1 + tid; i < H; i += BW_NT) prt[i] = fma(cl[i], vl, prt[i]);
         }
         bw_csync<CS>();   // (1) partials of every CTA complete
+        if (q == 0 && tid == 0) BCW_TRACE(s, m, 3);
         // ---- 2. p = tau D v, y = O v: the CS partials summed in rank order
         for (int i = tid; i < H; i += BW_NT) {
           double acc = 0.0;
@@ -1008,6 +1012,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           }
         }
         bw_csync<CS>();   // (2) vn and its scalars everywhere
+        if (q == 0 && tid == 0) BCW_TRACE(s, m, 4);
         taun = scal[5];
       }
       // ---- 4. one fused pass per column (one warp per column): D -= v w^T + w v^T (lower); O -= tau y v^T, then
@@ -1045,6 +1050,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
             for (int i = lane; i < H; i += 32) __stcg(dst + i, col[i]);
             __syncwarp();   // the warp's stores of column 0 are ordered before lane 0's release
             if (lane == 0) st_release_s32(a.prog + s, (int)(m + 1));
+            if (q == 0 && tid == 0) BCW_TRACE(s, m, 8);
           } else {
             z = warp_sum(z);
             const double tz = taun * z;
@@ -1058,6 +1064,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       }
       __syncthreads();
       if (a.opt & 256) bw_csync<CS>();
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 5);
       // ---- store my columns back (one warp per column), the reflector of this step, publish
       for (int j = cbeg + warp; j < je; j += NW) {
         if (j == 0 && L2 > 0) continue;   // column 0 went out early (step 4)
@@ -1074,11 +1081,13 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
         if (tid == 0) a.tau2[off + m] = tau;
       }
       bw_csync<CS>();   // (3) every CTA's stores of this step issued (ordered before the release below)
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 6);
       if (q == 0 && tid == 0) {
         // e_s (the rest of column s is dead): written only now, when every CTA of the cluster has read column s
         if (m == 0) __stcg(a.band + s * ldab + 1, scal[1]);
         if (L2 == 0) st_release_s32(a.prog + s, (int)(m + 1));   // no early column-0 publication this step
         st_release_s32(a.prog_full + s, (int)(m + 1));
+        BCW_TRACE(s, m, 7);
       }
       tau = taun;
     }

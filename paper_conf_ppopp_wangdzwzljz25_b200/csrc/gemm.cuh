@@ -65,9 +65,10 @@ int pick_splits(int64_t M, int64_t N, int64_t K, int tile, int64_t max_part_elem
 cudaError_t gemm_ws(GemmArgs a, int opB, cudaStream_t st);
 cudaError_t gemm_ws_op(GemmArgs a, int opA, int opB, cudaStream_t st);
 // C (M x N) = alpha op(A) op(B) + beta Cin (ld lda/ldb/ldc), deterministic split-K over part (part_elems doubles)
+// A2 != nullptr (opA == OP_T): rows >= msplit of op(A) come from A2 (the stacked [op(A); op(A2)], same ld)
 cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
                        const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
-                       int64_t part_elems, cudaStream_t st);
+                       int64_t part_elems, cudaStream_t st, const double* A2 = nullptr, int64_t msplit = 0);
 // nc: columns of each of the two correction segments folded into the SYMM's K axis (0: none)
 int64_t symm_ws_splits(int64_t m, int64_t w, int64_t nc = 0);
 int ws_skinny_splits(int64_t M, int64_t N, int64_t K);

@@ -101,6 +101,10 @@ struct WsArgs {
   // rows past M / N and k past K are zero-filled by the copy engine)
   int tma;
   CUtensorMap tmA[2], tmB[2];
+  // GEMM segment 0 with A op T only, when A2 != nullptr: rows >= msplit of op(A) are rows (row - msplit) of A2 (same
+  // ld): two stacked operands [op(A); op(A2)] sharing B in one launch (the Z builder's U = [Z_<^T W; Y_<^T W])
+  const double* A2;
+  int64_t msplit;
 };
 
 template <bool MG>
@@ -306,7 +310,8 @@ __device__ __forceinline__ void load_minner16(double* T, const double* base, int
 // k-inner tile (A op T / B op N): R rows of BK contiguous k (BK/2 = 8 pairs per row).
 template <int R, int LD, int NP>
 __device__ __forceinline__ void load_kinner16(double* T, const double* base, int64_t ld, int64_t r0, int64_t rmax,
-                                              int64_t k0, int64_t kend, int pt) {
+                                              int64_t k0, int64_t kend, int pt, const double* base2 = nullptr,
+                                              int64_t msplit = INT64_MAX) {
   constexpr int NCP = R * (BK / 2) / NP;
   constexpr int RS = NP / (BK / 2);
   const int kk = 2 * (pt % (BK / 2)), rl = pt / (BK / 2);
@@ -316,7 +321,8 @@ __device__ __forceinline__ void load_kinner16(double* T, const double* base, int
     const int rr = rl + RS * i;
     const int64_t row = r0 + rr;
     const int bytes = row < rmax ? kbytes : 0;
-    cp16(T + rr * LD + kk, bytes ? base + k0 + kk + row * ld : base, bytes);
+    const double* rp = row < msplit ? base + row * ld : base2 + (row - msplit) * ld;
+    cp16(T + rr * LD + kk, bytes ? rp + k0 + kk : base, bytes);
   }
 }
 
@@ -336,6 +342,8 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
   // ---- A
   if (v16) {
     if (s.opa == OP_N) load_minner16<BM, C::A_LD_N, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt);
+    else if (s.seg == 0 && a.A2)
+      load_kinner16<BM, C::A_LD_T, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt, a.A2, a.msplit);
     else load_kinner16<BM, C::A_LD_T, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt);
   } else if (s.opa == OP_N) {   // A(m, k) at A[m + k*lda], tile As[k][m]
     for (int e = pt; e < BM * BK; e += NP) {
@@ -353,7 +361,8 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
       bool p = row < a.M && k < kend;
       if (s.mask == 1) p = p && (km(k) <= rm(row));
       if (s.mask == 2) p = p && (km(k) > rm(row));
-      cp8(As + r * C::A_LD_T + kk, p ? s.A + k + row * s.lda : s.A, p ? 8 : 0);
+      const double* rp = (s.seg == 0 && a.A2 && row >= a.msplit) ? a.A2 + (row - a.msplit) * s.lda : s.A + row * s.lda;
+      cp8(As + r * C::A_LD_T + kk, p ? rp + k : s.A, p ? 8 : 0);
     }
   }
   // ---- B
@@ -731,6 +740,12 @@ cudaError_t gemm_ws_op(GemmArgs g, int opA, int opB, cudaStream_t st) {
   a.mg_g = g.mg_g; a.mg_q = g.mg_q; a.mg_cb = g.mg_cb; a.mg_lofs = g.mg_lofs; a.mg_gofs = g.mg_gofs;
   if (a.mg_g > 1 && (a.tri || (a.lower && a.splits > 1) || a.mg_cb < 1)) return cudaErrorInvalidValue;
   a.part = g.part; a.part_ld = g.part_ld; a.part_stride = g.part_stride;
+  a.A2 = (g.A2m && g.msplit < g.M) ? g.A2m : nullptr;
+  a.msplit = g.msplit;
+  if (a.A2) {   // stacked operands: A op T, one segment, no multi-GPU map
+    if (opA != OP_T || g.nseg != 1 || a.mg_g > 1) return cudaErrorInvalidValue;
+    a.vec16 = a.vec16 && ws::al16(g.A2m);
+  }
   if (a.mg_g > 1) {   // multi-GPU column map (only the lower-masked syr2k of mg.cu uses it)
     if (opB != OP_T || opA != OP_N) return cudaErrorInvalidValue;
     return g.N <= 64 ? ws::launch<128, 64, 4, 2, OP_T, true>(a, st) : ws::launch<128, 128, 4, 2, OP_T, true>(a, st);
@@ -816,7 +831,7 @@ static int gemm_splits(int64_t M, int64_t N, int64_t K, int cap, int64_t part_ca
 // within part_elems partials and <= 64 splits.
 cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double alpha, const double* A, int64_t lda,
                        const double* B, int64_t ldb, double beta, double* C, int64_t ldc, double* part,
-                       int64_t part_elems, cudaStream_t st) {
+                       int64_t part_elems, cudaStream_t st, const double* A2, int64_t msplit) {
   if (M <= 0 || N <= 0) return cudaSuccess;
   int64_t s;
   if (split_model_on()) {
@@ -833,6 +848,10 @@ cudaError_t gemm_ws_mm(int opA, int opB, int64_t M, int64_t N, int64_t K, double
   GemmArgs g;
   g.M = M; g.N = N; g.K[0] = K; g.A[0] = A; g.lda[0] = lda; g.B[0] = B; g.ldb[0] = ldb;
   g.alpha = alpha; g.beta = beta; g.Cin = C; g.ldcin = ldc; g.C = C; g.ldc = ldc;
+  if (A2) {
+    g.A2m = A2;
+    g.msplit = msplit;
+  }
   g.splits = (int)s;
   g.part = part; g.part_ld = M; g.part_stride = M * N;
   return gemm_ws_op(g, opA, opB, st);

@@ -512,10 +512,9 @@ int trid_sbr_dbbr_mg(trid_comm_t comm, int64_t n, double* A, int64_t lda, int co
         ProfScope ps(PROF_ZY, st);
         double* U1 = w.U;
         double* U2 = w.U + ncols;
-        TRID_CUDA_TRY(gemm_ws_mm(OP_T, OP_N, ncols, kk, m, -1.0, w.Z + o, ld, w.W, ld, 0.0, U1, 2 * k, w.part,
-                                 w.part_elems, st));
-        TRID_CUDA_TRY(gemm_ws_mm(OP_T, OP_N, ncols, kk, m, -1.0, w.Y + o, ld, w.W, ld, 0.0, U2, 2 * k, w.part,
-                                 w.part_elems, st));
+        // U = -[Z_<^T W; Y_<^T W] in one launch over the stacked operands (U2 = U1 + ncols)
+        TRID_CUDA_TRY(gemm_ws_mm(OP_T, OP_N, 2 * ncols, kk, m, -1.0, w.Z + o, ld, w.W, ld, 0.0, U1, 2 * k, w.part,
+                                 w.part_elems, st, w.Y + o, ncols));
         // contiguous row slices starting at even rows (16-byte aligned operands for the engine's fast producer)
         const int64_t rlo = q == 0 ? 0 : (m * q / g) & ~(int64_t)1;
         const int64_t rhi = q == g - 1 ? m : (m * (q + 1) / g) & ~(int64_t)1;
