@@ -1018,63 +1018,81 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       // ---- 4. one fused pass per column (one warp per column): D -= v w^T + w v^T (lower); O -= tau y v^T, then
       //      O(:, j) -= taun vn (vn^T O(:, j)) for j >= 1, O(:, 0) = beta e1.  Window column 0 (rank 0, warp 0,
       //      first) is final right after its pass: stored and published at once (prog)
+      // Round 2: the step vectors are held in registers by absolute window row (lane + 32 k), and every column but
+      // column 0 goes from its fused pass straight to the band (no shared write-back, no separate store pass): the
+      // pass was bound by shared-memory traffic (5 accesses per element, then a 6th to store; trace: fused pass
+      // 7.4 us + store 4.1 us of a 25 us step at b = 128).  Same expressions in the same order (bitwise).
+      constexpr int KR = CS == 1 ? 4 : 8;   // rows per lane: L, L2 <= b <= 128 (CS = 1) or <= 256
+      double vD[KR], wD[KR], pO[KR], vnO[KR];
+#pragma unroll
+      for (int k = 0; k < KR; ++k) {
+        const int i = lane + 32 * k;
+        vD[k] = i < L ? v[i] : 0.0;
+        wD[k] = (tau != 0.0 && i < L) ? wv[i] : 0.0;
+        pO[k] = (tau != 0.0 && i < L2) ? pf[L + i] : 0.0;
+        vnO[k] = (L2 > 0 && i < L2) ? vn[i] : 0.0;
+      }
       for (int j = cbeg + warp; j < je; j += NW) {
         double* col = win + cofs[j];
+        if (j == 0 && L2 > 0) {
+          // window column 0: final in shared memory, stored and published at once (the chain's early hand-off)
+          if (tau != 0.0) {
+            const double vj = v[j], wj = wv[j];
+            for (int i = j + lane; i < L; i += 32) col[i] = fma(-wv[i], vj, fma(-v[i], wj, col[i]));
+          }
+#pragma unroll
+          for (int k = 0; k < KR; ++k) {
+            const int i = lane + 32 * k;
+            if (i < L2) col[L + i] = i == 0 ? scal[4] : 0.0;
+          }
+          __syncwarp();
+          double* dst0 = a.band + r0 * ldab;
+          for (int i = lane; i < H; i += 32) __stcg(dst0 + i, col[i]);
+          __syncwarp();   // the warp's stores of column 0 are ordered before lane 0's release
+          if (lane == 0) st_release_s32(a.prog + s, (int)(m + 1));
+          if (q == 0 && tid == 0) BCW_TRACE(s, m, 8);
+          continue;
+        }
+        double* dst = a.band + (r0 + j) * ldab - j;   // window element (i, j), i >= j, at dst[i]
         if (tau != 0.0) {
           const double vj = v[j], wj = wv[j];
-          for (int i = j + lane; i < L; i += 32) col[i] = fma(-wv[i], vj, fma(-v[i], wj, col[i]));
+#pragma unroll
+          for (int k = 0; k < KR; ++k) {
+            const int i = lane + 32 * k;
+            if (i >= j && i < L) __stcg(dst + i, fma(-wD[k], vj, fma(-vD[k], wj, col[i])));
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < KR; ++k) {
+            const int i = lane + 32 * k;
+            if (i >= j && i < L) __stcg(dst + i, col[i]);
+          }
         }
         if (L2 > 0) {
-          double* oc = col + L;
+          const double* oc = col + L;
           const double tvj = tau * v[j];
-          constexpr int KO = 8;   // L2 <= b <= 256 rows of O per column: <= 8 per lane
-          double o[KO];
+          double o[KR];
           double z = 0.0;
 #pragma unroll
-          for (int k = 0; k < KO; ++k) {
+          for (int k = 0; k < KR; ++k) {
             const int i = lane + 32 * k;
             o[k] = 0.0;
             if (i < L2) {
-              o[k] = tau != 0.0 ? fma(-pf[L + i], tvj, oc[i]) : oc[i];
-              z = fma(vn[i], o[k], z);
+              o[k] = tau != 0.0 ? fma(-pO[k], tvj, oc[i]) : oc[i];
+              z = fma(vnO[k], o[k], z);
             }
           }
-          if (j == 0) {
+          z = warp_sum(z);
+          const double tz = taun * z;
 #pragma unroll
-            for (int k = 0; k < KO; ++k) {
-              const int i = lane + 32 * k;
-              if (i < L2) oc[i] = i == 0 ? scal[4] : 0.0;
-            }
-            __syncwarp();
-            double* dst = a.band + r0 * ldab;
-            for (int i = lane; i < H; i += 32) __stcg(dst + i, col[i]);
-            __syncwarp();   // the warp's stores of column 0 are ordered before lane 0's release
-            if (lane == 0) st_release_s32(a.prog + s, (int)(m + 1));
-            if (q == 0 && tid == 0) BCW_TRACE(s, m, 8);
-          } else {
-            z = warp_sum(z);
-            const double tz = taun * z;
-#pragma unroll
-            for (int k = 0; k < KO; ++k) {
-              const int i = lane + 32 * k;
-              if (i < L2) oc[i] = taun != 0.0 ? fma(-tz, vn[i], o[k]) : o[k];
-            }
+          for (int k = 0; k < KR; ++k) {
+            const int i = lane + 32 * k;
+            if (i < L2) __stcg(dst + L + i, taun != 0.0 ? fma(-tz, vnO[k], o[k]) : o[k]);
           }
         }
       }
-      __syncthreads();
       if (a.opt & 256) bw_csync<CS>();
       if (q == 0 && tid == 0) BCW_TRACE(s, m, 5);
-      // ---- store my columns back (one warp per column), the reflector of this step, publish
-      for (int j = cbeg + warp; j < je; j += NW) {
-        if (j == 0 && L2 > 0) continue;   // column 0 went out early (step 4)
-        const int len = H - j, len2 = len >> 1;
-        const double* srcp = win + cofs[j] + j;
-        double* dst = a.band + (r0 + j) * ldab;
-        for (int i = lane; i < len2; i += 32)
-          __stcg(reinterpret_cast<double2*>(dst) + i, reinterpret_cast<const double2*>(srcp)[i]);
-        if ((len & 1) && lane == 0) __stcg(dst + len - 1, srcp[len - 1]);
-      }
       if (q == 0 && a.V2) {
         double* vd = a.V2 + (off + m) * a.vs;
         for (int i = tid; i < a.vs; i += BW_NT) vd[i] = i < L ? v[i] : 0.0;
