@@ -914,33 +914,63 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       // ---- 1. partial matvec [D; O] v over my BODY columns (all but the window's last, which sweep s-1 may still
       //      be producing), all H rows; the last column's terms are added once it arrives
       if (tau != 0.0) {
-        {
-          const int i = tid % H2, h = tid / H2;   // row i, half h (tpr == 2) of my columns
-          if (h < tpr) {
-            double acc = 0.0;
-            if (i < H) {
-              const int jlo = tpr == 2 ? (h ? jmid : cbeg) : cbeg;
-              int jhi = tpr == 2 ? (h ? je : (jmid < je ? jmid : je)) : je;
-              if (jhi > i + 1) jhi = i + 1;   // lower part of D (and all of O): columns j <= i
-              if (jhi > L - 1) jhi = L - 1;   // body only
-              for (int j = jlo; j < jhi; ++j) acc = fma(win[cofs[j] + i], v[j], acc);
+        if constexpr (CS == 1) {
+          // one CTA holds every column: thread (i, h) forms row i of [D; O] v over half h of the body columns in one
+          // pass, the upper part of D from its mirror in column i (D(j, i), j > i, incl. the last column's term,
+          // which column i holds), four accumulators (round 2: the former row pass + per-column warp dots took
+          // 7.2 us of a 19.5 us step at b = 128)
+          const int i = tid % H2, h = tid / H2;   // tpr == 2 (b <= 128, 512 threads)
+          double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
+          if (i < H) {
+            const int jend = i < L - 1 ? L : L - 1;
+            const int jlo = h ? jmid : 0;
+            const int jhi = h ? jend : (jmid < jend ? jmid : jend);
+            const int ci = i < L ? cofs[i] : 0;
+            auto el = [&](int j) { return win[j <= i ? cofs[j] + i : ci + j]; };
+            int j = jlo;
+            for (; j + 4 <= jhi; j += 4) {
+              const double e0 = el(j), e1 = el(j + 1), e2 = el(j + 2), e3 = el(j + 3);
+              a0 = fma(e0, v[j], a0);
+              a1 = fma(e1, v[j + 1], a1);
+              a2 = fma(e2, v[j + 2], a2);
+              a3 = fma(e3, v[j + 3], a3);
             }
-            prt[h * H2 + i] = acc;
+            for (; j < jhi; ++j) a0 = fma(el(j), v[j], a0);
+          }
+          if (h < 2) prt[h * H2 + i] = (a0 + a1) + (a2 + a3);
+          __syncthreads();
+          for (int r = tid; r < H2; r += BW_NT) prt[r] += prt[H2 + r];
+          // (the barrier after the last column's load orders these sums before their last-column terms)
+        } else {
+          {
+            const int i = tid % H2, h = tid / H2;   // row i, half h (tpr == 2) of my columns
+            if (h < tpr) {
+              double acc = 0.0;
+              if (i < H) {
+                const int jlo = tpr == 2 ? (h ? jmid : cbeg) : cbeg;
+                int jhi = tpr == 2 ? (h ? je : (jmid < je ? jmid : je)) : je;
+                if (jhi > i + 1) jhi = i + 1;   // lower part of D (and all of O): columns j <= i
+                if (jhi > L - 1) jhi = L - 1;   // body only
+                for (int j = jlo; j < jhi; ++j) acc = fma(win[cofs[j] + i], v[j], acc);
+              }
+              prt[h * H2 + i] = acc;
+            }
+          }
+          __syncthreads();
+          if (tpr == 2)
+            for (int i = tid; i < H2; i += BW_NT) prt[i] += prt[H2 + i];
+          __syncthreads();
+          // mirrored upper part of D for my columns c: sum_{j > c, j < L} D(j, c) v_j (a column dot, one warp)
+          for (int c = cbeg + warp; c < je; c += NW) {
+            const double* col = win + cofs[c];
+            double acc = 0.0;
+            for (int j = c + 1 + lane; j < L; j += 32) acc = fma(col[j], v[j], acc);
+            acc = warp_sum(acc);
+            if (lane == 0) prt[c] += acc;
           }
         }
-        __syncthreads();
-        if (tpr == 2)
-          for (int i = tid; i < H2; i += BW_NT) prt[i] += prt[H2 + i];
-        __syncthreads();
-        // mirrored upper part of D for my columns c: sum_{j > c, j < L} D(j, c) v_j (a column dot, one warp)
-        for (int c = cbeg + warp; c < je; c += NW) {
-          const double* col = win + cofs[c];
-          double acc = 0.0;
-          for (int j = c + 1 + lane; j < L; j += 32) acc = fma(col[j], v[j], acc);
-          acc = warp_sum(acc);
-          if (lane == 0) prt[c] += acc;
-        }
       }
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 9);   // (body matvec done in thread 0's warp)
       // ---- the last column = column 0 of sweep s-1's step m+1: wait for its early publication, load, add its terms
       //      D(L-1, L-1) v_{L-1} and O(:, L-1) v_{L-1} (fixed order: after the body and the mirror)
       if (s > 0 && need_c0 > need_full) {

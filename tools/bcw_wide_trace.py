@@ -2,7 +2,7 @@
 
 Slots (q == 0, tid 0): 0 body deps met (prog_full), 1 body loaded, 2 last-column deps met (prog), 3 partials complete
 (barrier 1), 4 next reflector everywhere (barrier 2), 5 fused pass done, 6 stores issued (barrier 3), 7 prog_full
-released, 8 column 0 published (prog).  Prints medians relative to slot 0 of the same step, the step-to-step advance
+released, 8 column 0 published (prog), 9 thread 0's warp done with the body matvec.  Prints medians relative to slot 0 of the same step, the step-to-step advance
 and the link (predecessor's prog release -> our step's deps)."""
 import json
 import os
@@ -35,7 +35,7 @@ tr = tr.astype(np.float64)
 steps = min((n - 3 - (sw + 1)) // b + 1, 1024)
 p, c = tr[0], tr[1]
 m = np.arange(2, steps - 3)
-rel = {str(k): round(float(np.median(c[m, k] - c[m, 0])), 1) for k in range(9)}
+rel = {str(k): round(float(np.median(c[m, k] - c[m, 0])), 1) for k in range(10)}
 adv = {"step_advance_ns (0: m -> m+1)": round(float(np.median(np.diff(c[m, 0]))), 1),
        "prog_full_link_ns (prod 7(m) -> cons 0(m))": round(float(np.median(c[m, 0] - p[m, 7])), 1),
        "col0_link_ns (prod 8(m+1) -> cons 2(m))": round(float(np.median(c[m, 2] - p[m + 1, 8])), 1),
