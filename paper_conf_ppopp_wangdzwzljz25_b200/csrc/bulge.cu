@@ -851,6 +851,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
     const int64_t off = bc_offset(n, b, s);
     const int64_t nprev = s > 0 ? bc_steps(n, b, s - 1) : 0;
     double tau = 0.0;
+    bool pref = false;   // this warp's body columns of the current step were requested during the previous one
     for (int64_t m = 0; m < nst; ++m) {
       double* v = vb + (m & 1) * b;
       double* vn = vb + ((m & 1) ^ 1) * b;
@@ -868,25 +869,34 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       // still being produced.
       const int need_full = (int)(a.serial ? nprev : m + 1);
       const int need_c0 = (int)((m + 2 < nprev && !a.serial) ? m + 2 : nprev);
-      if (s > 0) {
-        if (tid == 0) wait_geq(a.prog_full + (s - 1), need_full);
-        __syncthreads();
-      }
-      if (q == 0 && tid == 0) BCW_TRACE(s, m, 0);
-      if (a.opt & 64) bw_csync<CS>();   // debug (TRID_BC_OPT): extra cluster barriers
       // ---- load my window columns, one warp per column (rows j .. H-1: offsets 0 .. H-1-j); the last one after
-      // its producer published it
-      auto load_col = [&](int j) {
-        const int len = H - j, len2 = len >> 1;
+      // its producer published it.  A warp whose columns were prefetched at the end of the previous step (pref,
+      // below) skips this; otherwise its lane 0 waits for the dependency (each warp orders its own loads).
+      auto load_col_at = [&](int j, const double* gwx, int Hx) {
+        const int len = Hx - j, len2 = len >> 1;
         double* dst = win + cofs[j] + j;
-        const double* src = gw + (int64_t)j * ldab;
+        const double* src = gwx + (int64_t)j * ldab;
         for (int i = lane; i < len2; i += 32)
           asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(dst + 2 * i)), "l"(src + 2 * i)
                        : "memory");
-        if ((len & 1) && lane == 0) dst[len - 1] = __ldcg(src + len - 1);
+        // the odd tail element asynchronously too (round 2: a synchronous L2 load here stalled the warp once per
+        // odd-length column, about half of them)
+        if ((len & 1) && lane == 0)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(smem_u32(dst + len - 1)), "l"(src + len - 1)
+                       : "memory");
       };
-      for (int j = cbeg + warp; j < je && j < L - 1; j += NW) load_col(j);
+      auto load_col = [&](int j) { load_col_at(j, gw, H); };
+      if (!pref) {
+        if (s > 0) {
+          if (lane == 0) wait_geq(a.prog_full + (s - 1), need_full);
+          __syncwarp();
+        }
+        for (int j = cbeg + warp; j < je && j < L - 1; j += NW) load_col(j);
+      }
+      pref = false;
       asm volatile("cp.async.commit_group;\n" ::: "memory");
+      if (q == 0 && tid == 0) BCW_TRACE(s, m, 0);
+      if (a.opt & 64) bw_csync<CS>();   // debug (TRID_BC_OPT): extra cluster barriers
       const bool own_last = je == L && L - 1 >= cbeg;   // this CTA holds the window's last column
       // ---- step 0: the reflector annihilating column s below its first subdiagonal (every CTA, same bits)
       if (m == 0) {
@@ -1119,6 +1129,26 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
             const int i = lane + 32 * k;
             if (i < L2) __stcg(dst + L + i, taun != 0.0 ? fma(-tz, vnO[k], o[k]) : o[k]);
           }
+        }
+      }
+      // prefetch: this warp's columns are final in the band and its shared slots dead, so if the predecessor has
+      // already completed step m+1 (non-blocking check) the same columns of step m+1 are requested now and the
+      // load overlaps the rest of this step (round 2: the synchronous window load was 2.8 us of a 17 us step)
+      if (m + 1 < nst) {
+        const int need_n = (int)(a.serial ? nprev : m + 2);
+        int ready = 1;
+        if (s > 0 && lane == 0) ready = ld_acquire_s32(a.prog_full + (s - 1)) >= need_n;
+        ready = __shfl_sync(0xffffffffu, ready, 0);
+        if (ready) {
+          const int64_t r0n = r0 + b;
+          const int64_t r1n = (s + (m + 2) * b < n - 1) ? s + (m + 2) * b : n - 1;
+          const int Ln = (int)(r1n - r0n + 1);
+          const int64_t r2n = (r1n + b < n - 1) ? r1n + b : n - 1;
+          const int Hn = Ln + (int)(r2n - r1n);
+          const int jen = cend < Ln ? cend : Ln;
+          const double* gwn = a.band + r0n * ldab;
+          for (int j = cbeg + warp; j < jen && j < Ln - 1; j += NW) load_col_at(j, gwn, Hn);
+          pref = true;
         }
       }
       if (a.opt & 256) bw_csync<CS>();
