@@ -44,40 +44,54 @@ def per_launch(rows):
 
 
 def classify(launches):
-    """Assign each launch a stage class using the per-panel launch order (round 2, corrections folded into the
-    SYMM): panel, W = Y T, U1 = Z_<^T W (+ reduce), U2 = Y_<^T W (+ reduce), the SYMM with the correction K
-    segments (+ reduce), S = W^T X (gemm_kernel + reduce), Z, the next-panel update (ws_kernel<.., 1, 0>)."""
-    cls = []
-    ws_since_panel = 99
-    for d in launches:
+    """Assign each launch a stage class.  Per panel (the launches between two panel_* launches): the first
+    ws_kernel<128, 64, 4, 2, 0> is W = Y T, the longest one is the SYMM (with the folded corrections) and the
+    ws_reduce_kernel right after it belongs to it, ws_kernel<.., 1, 0> (B op T) is the next-panel update, the other
+    skinny launches (the stacked U, S, Z and their reductions) are the Z tail; ws_kernel<128, 128, ...> is the syr2k,
+    bc_* / band_* the chase."""
+    cls = [None] * len(launches)
+    group = []
+
+    def flush():
+        ws0 = [i for i in group if "ws_kernel<128, 64, 4, 2, 0" in launches[i]["name"]]
+        if not ws0:
+            return
+        w_i = ws0[0]
+        rest = ws0[1:]
+        s_i = max(rest, key=lambda i: launches[i].get("gpu__time_duration.sum", 0.0)) if rest else None
+        for i in group:
+            nm = launches[i]["name"]
+            if i == w_i:
+                cls[i] = "wy"
+            elif i == s_i:
+                cls[i] = "symm"
+            elif "ws_kernel<128, 64, 4, 2, 1" in nm:
+                cls[i] = "next_panel"
+            elif "ws_reduce_kernel" in nm and s_i is not None and i == s_i + 1:
+                cls[i] = "symm"
+            else:
+                cls[i] = "zy"
+
+    for i, d in enumerate(launches):
         nm = d["name"]
         if "panel_" in nm:
-            c = "panel_qr"
-            ws_since_panel = 0
+            flush()
+            group = []
+            cls[i] = "panel_qr"
         elif "ws_kernel<128, 128" in nm:
-            c = "syr2k"
-        elif "ws_kernel" in nm:
-            ws_since_panel += 1
-            if "ws_kernel<128, 64, 4, 2, 1" in nm:
-                c = "next_panel"
-            elif ws_since_panel == 1:
-                c = "wy"
-            elif ws_since_panel == 4:
-                c = "symm"
-            else:
-                c = "zy"
-        elif "ws_reduce_kernel" in nm:
-            c = "symm" if ws_since_panel == 4 else "zy"
-        elif "gemm_kernel" in nm or "reduce_partials" in nm:
-            c = "zy"
+            flush()
+            group = []
+            cls[i] = "syr2k"
         elif "bc_" in nm or "band_" in nm:
-            c = "bulge_chase"
-        elif "trid::" in nm or "ws_" in nm:
-            c = "other_trid"
+            cls[i] = "bulge_chase"
+        elif "ws_" in nm or "gemm_kernel" in nm or "reduce_partials" in nm:
+            group.append(i)
+        elif "trid::" in nm:
+            cls[i] = "other_trid"
         else:
-            c = "torch"
-        cls.append(c)
-    return cls
+            cls[i] = "torch"
+    flush()
+    return [c or "other_trid" for c in cls]
 
 
 def summarize_launches(path):
