@@ -1006,44 +1006,45 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           for (unsigned r = 0; r < CS; ++r) acc += bw_ld<CS>(prt + i, r);
           pf[i] = i < L ? tau * acc : acc;
         }
-        __syncthreads();
-        if (warp == 0) {
-          double pv = 0.0;
-          for (int i = lane; i < L; i += 32) pv = fma(pf[i], v[i], pv);
-          pv = warp_sum(pv);
-          if (lane == 0) scal[0] = pv;
+      }
+      __syncthreads();
+      // ---- p^T v (warp 0) and 3. the next reflector from x = O(:, 0) - tau y v_0 (O(:, 0) after the right update;
+      //      window column 0 belongs to rank 0; warp 1 at the same time), before any column is updated
+      //      (round 2: one barrier for both reductions instead of three)
+      if (tau != 0.0 && warp == 0) {
+        double pv = 0.0;
+        for (int i = lane; i < L; i += 32) pv = fma(pf[i], v[i], pv);
+        pv = warp_sum(pv);
+        if (lane == 0) scal[0] = pv;
+      }
+      const double* c0 = win + cofs[0] + L;
+      const double tv0 = tau * v[0];
+      auto xo = [&](int i) { return tau != 0.0 ? fma(-pf[L + i], tv0, c0[i]) : c0[i]; };
+      if (L2 > 0 && q == 0 && warp == 1) {
+        double sg = 0.0;
+        for (int i = 1 + lane; i < L2; i += 32) {
+          const double x = xo(i);
+          sg = fma(x, x, sg);
         }
-        __syncthreads();
-        if (a.opt & 512) bw_csync<CS>();
+        sg = warp_sum(sg);
+        if (lane == 0) {
+          const House h = make_house(xo(0), sg);
+          for (unsigned r = 0; r < CS; ++r) {
+            bw_st<CS>(scal + 4, r, h.beta);
+            bw_st<CS>(scal + 5, r, h.tau);
+            bw_st<CS>(scal + 6, r, h.scale);
+          }
+        }
+      }
+      __syncthreads();
+      if (a.opt & 512) bw_csync<CS>();
+      if (tau != 0.0) {
         const double hp = 0.5 * tau * scal[0];
         for (int i = tid; i < L; i += BW_NT) wv[i] = fma(-hp, v[i], pf[i]);
-        __syncthreads();
       }
-      // ---- 3. the next reflector from x = O(:, 0) - tau y v_0 (O(:, 0) after the right update; window column 0
-      //      belongs to rank 0), broadcast through DSMEM, before any column is updated
       double taun = 0.0;
       if (L2 > 0) {
         if (q == 0) {
-          const double* c0 = win + cofs[0] + L;
-          const double tv0 = tau * v[0];
-          auto xo = [&](int i) { return tau != 0.0 ? fma(-pf[L + i], tv0, c0[i]) : c0[i]; };
-          if (warp == 0) {
-            double sg = 0.0;
-            for (int i = 1 + lane; i < L2; i += 32) {
-              const double x = xo(i);
-              sg = fma(x, x, sg);
-            }
-            sg = warp_sum(sg);
-            if (lane == 0) {
-              const House h = make_house(xo(0), sg);
-              for (unsigned r = 0; r < CS; ++r) {
-                bw_st<CS>(scal + 4, r, h.beta);
-                bw_st<CS>(scal + 5, r, h.tau);
-                bw_st<CS>(scal + 6, r, h.scale);
-              }
-            }
-          }
-          __syncthreads();
           const double hs = scal[6];
           for (int i = tid; i < b; i += BW_NT) {
             const double x = i < L2 ? (i == 0 ? 1.0 : hs * xo(i)) : 0.0;
@@ -1051,9 +1052,11 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
             for (unsigned r = 0; r < CS; ++r) bw_st<CS>(vn + i, r, x);
           }
         }
-        bw_csync<CS>();   // (2) vn and its scalars everywhere
+        bw_csync<CS>();   // (2) w, vn and its scalars everywhere
         if (q == 0 && tid == 0) BCW_TRACE(s, m, 4);
         taun = scal[5];
+      } else {
+        __syncthreads();   // w
       }
       // ---- 4. one fused pass per column (one warp per column): D -= v w^T + w v^T (lower); O -= tau y v^T, then
       //      O(:, j) -= taun vn (vn^T O(:, j)) for j >= 1, O(:, 0) = beta e1.  Window column 0 (rank 0, warp 0,

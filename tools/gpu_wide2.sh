@@ -1,6 +1,6 @@
 #!/bin/bash
 # Wide chase with register-cached step vectors and direct column stores: parity, traces, config benches.
-O=gpurun_out/r02w5; mkdir -p $O
+O=gpurun_out/r02w7; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
 timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_parity_large.py -q -x -m gpu -k "bulge or two_stage" --timeout 300 > $O/pytest.log 2>&1
 echo "pytest rc=$?" >> $O/pytest.log
