@@ -888,7 +888,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       auto load_col = [&](int j) { load_col_at(j, gw, H); };
       if (!pref) {
         if (s > 0) {
-          if (lane == 0) wait_geq(a.prog_full + (s - 1), need_full);
+          if (lane == 0) wait_geq(a.prog_full + (s - 1) * a.fs, need_full);
           __syncwarp();
         }
         for (int j = cbeg + warp; j < je && j < L - 1; j += NW) load_col(j);
@@ -984,7 +984,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       // ---- the last column = column 0 of sweep s-1's step m+1: wait for its early publication, load, add its terms
       //      D(L-1, L-1) v_{L-1} and O(:, L-1) v_{L-1} (fixed order: after the body and the mirror)
       if (s > 0 && need_c0 > need_full) {
-        if (tid == 0) wait_geq(a.prog + (s - 1), need_c0);
+        if (tid == 0) wait_geq(a.prog + (s - 1) * a.fs, need_c0);
         __syncthreads();
       }
       if (q == 0 && tid == 0) BCW_TRACE(s, m, 2);
@@ -1092,7 +1092,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
           double* dst0 = a.band + r0 * ldab;
           for (int i = lane; i < H; i += 32) __stcg(dst0 + i, col[i]);
           __syncwarp();   // the warp's stores of column 0 are ordered before lane 0's release
-          if (lane == 0) st_release_s32(a.prog + s, (int)(m + 1));
+          if (lane == 0) st_release_s32(a.prog + s * a.fs, (int)(m + 1));
           if (q == 0 && tid == 0) BCW_TRACE(s, m, 8);
           continue;
         }
@@ -1140,7 +1140,7 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       if (m + 1 < nst) {
         const int need_n = (int)(a.serial ? nprev : m + 2);
         int ready = 1;
-        if (s > 0 && lane == 0) ready = ld_acquire_s32(a.prog_full + (s - 1)) >= need_n;
+        if (s > 0 && lane == 0) ready = ld_acquire_s32(a.prog_full + (s - 1) * a.fs) >= need_n;
         ready = __shfl_sync(0xffffffffu, ready, 0);
         if (ready) {
           const int64_t r0n = r0 + b;
@@ -1166,8 +1166,8 @@ __global__ void __launch_bounds__(BW_NT, 1) bc_wide_kernel(BcArgs a, BwPart part
       if (q == 0 && tid == 0) {
         // e_s (the rest of column s is dead): written only now, when every CTA of the cluster has read column s
         if (m == 0) __stcg(a.band + s * ldab + 1, scal[1]);
-        if (L2 == 0) st_release_s32(a.prog + s, (int)(m + 1));   // no early column-0 publication this step
-        st_release_s32(a.prog_full + s, (int)(m + 1));
+        if (L2 == 0) st_release_s32(a.prog + s * a.fs, (int)(m + 1));   // no early column-0 publication this step
+        st_release_s32(a.prog_full + s * a.fs, (int)(m + 1));
         BCW_TRACE(s, m, 7);
       }
       tau = taun;
@@ -1194,12 +1194,13 @@ cudaError_t bulge_chase_cs(int64_t n, int b, const double* X, int64_t cs, double
   const int ldab = bc_ldab(n, beff);
   double* band = (double*)work;
   const size_t band_bytes = ((sizeof(double) * (size_t)n * ldab + 255) / 256) * 256;
-  // per-sweep counters: one 32-byte sector apart for bc_v6 (no two sweeps' counters share a sector), packed
-  // (stride 1) for bc_kernel (b > 64); the region is sized for the widest layout (BC_FLAG_STRIDE)
+  // per-sweep counters: one 32-byte sector apart (no two sweeps' counters share a sector: packed, the producers'
+  // releases and the consumers' polls of neighbouring sweeps contended on the same lines); TRID_BC_FS = stride in
+  // ints (A/B); the region is sized for the widest layout (BC_FLAG_STRIDE)
   const char* fse = getenv("TRID_BC_FS");
   int fsv = fse ? atoi(fse) : 8;
   if (fsv < 1 || fsv > BC_FLAG_STRIDE) fsv = 8;
-  const int fs = beff <= 64 ? fsv : 1;
+  const int fs = fsv;   // round 2: the wide chase too (it used packed counters)
   int* prog = (int*)((char*)work + band_bytes);
   int* prog_full = prog + (n + 32) * fs;
   unsigned* ticket = (unsigned*)(prog_full + (n + 32) * fs);
