@@ -1,6 +1,7 @@
 """Parity at BASELINE.json's full sizes, in the launch configuration bench.py times (-m gpu).
 
-Q cannot be formed at n >= 8192, so:
+Q is formed on the GPU by the two back-transformation kernels only in test_exact_gates_timed_input_n32768 (the
+timed input, exact G1/G2); the other full-size cases check:
   * G3 on prescribed-spectrum inputs (trid_gen.clustered_symmetric: the 1-2-1 Toeplitz spectrum in closed
     form, or 32 tight clusters), eigenvalues of T sampled one by one with the oracle's Sturm count
     (bisection to full precision), against the known eigenvalues: within 1e-12 ||A||_2;
@@ -114,3 +115,35 @@ def test_probe_gates_detect_a_wrong_reflector(dev):
     tau2[len(tau2) // 2] *= -1.0
     g1b, g2b = probe_gates(A0, A, d, e, tau1, V2, tau2, b)
     assert g1b > 1e-10
+
+
+def test_exact_gates_timed_input_n32768(dev):
+    """The north_star gates G1/G2 EXACTLY (no probes) on the input bench.py times (BASELINE configs[2]: n = 32768
+    random symmetric, seed 3001, b = 64, nb = 16, k = 1024): Q = Q1 Q2 formed on the GPU by the two
+    back-transformation kernels, then ||A - Q T Q^T||_F / (n ||A||_F) and ||Q^T Q - I||_F / n
+    with cuBLAS DGEMMs (torch.matmul, test-side).  T is applied as a tridiagonal (column shifts), never formed."""
+    n, b, nb, k = 32768, 64, 16, 1024
+    A = trid_gen.random_symmetric(n, 3001, device="cuda:0")
+    A0 = A.clone()
+    d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=nb, k=k)
+    Qs = torch.eye(n, dtype=torch.float64, device="cuda:0")   # storage of the column-major identity
+    trid.bc_backtransform(V2, tau2, n, b, Qs)
+    del V2, tau2
+    trid.sbr_backtransform(A, tau1, b, Qs)
+    del A
+    Q = Qs.mT                                                  # logical Q (a view)
+    QT = Q * d                                                 # Q T: column j = d_j q_j + e_{j-1} q_{j-1} + e_j q_{j+1}
+    QT[:, 1:] += Q[:, :-1] * e
+    QT[:, :-1] += Q[:, 1:] * e
+    R = torch.matmul(QT, Q.T)
+    del QT
+    A0l = A0.mT                                                # logical A (symmetric: the same matrix)
+    nA = float(torch.linalg.norm(A0l))
+    R.sub_(A0l)
+    g1 = float(torch.linalg.norm(R)) / (n * nA)
+    del R, A0, A0l
+    G = torch.matmul(Q.T, Q)
+    G.diagonal().sub_(1.0)
+    g2 = float(torch.linalg.norm(G)) / n
+    assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
+    print(f"n=32768 seed 3001 exact G1={g1:.3e} G2={g2:.3e}")
