@@ -117,13 +117,19 @@ def test_probe_gates_detect_a_wrong_reflector(dev):
     assert g1b > 1e-10
 
 
-def test_exact_gates_timed_input_n32768(dev):
-    """The north_star gates G1/G2 EXACTLY (no probes) on the input bench.py times (BASELINE configs[2]: n = 32768
-    random symmetric, seed 3001, b = 64, nb = 16, k = 1024): Q = Q1 Q2 formed on the GPU by the two
-    back-transformation kernels, then ||A - Q T Q^T||_F / (n ||A||_F) and ||Q^T Q - I||_F / n
-    with cuBLAS DGEMMs (torch.matmul, test-side).  T is applied as a tridiagonal (column shifts), never formed."""
-    n, b, nb, k = 32768, 64, 16, 1024
-    A = trid_gen.random_symmetric(n, 3001, device="cuda:0")
+@pytest.mark.parametrize("n,b,seed,kind", [(32768, 64, 3001, "random"), (32768, 128, 3001, "random"),
+                                           (49152, 64, 4001, "clusters")])
+def test_exact_gates_timed_input_n32768(n, b, seed, kind, dev):
+    """The north_star gates G1/G2 EXACTLY (no probes) on the inputs bench.py times (BASELINE configs[2]: n = 32768
+    random symmetric, seed 3001, b = 64 and 128; configs[3]: n = 49152 clustered spectrum, seed 4001; nb = 16,
+    k = 1024): Q = Q1 Q2 formed on the GPU by the two back-transformation kernels, then
+    ||A - Q T Q^T||_F / (n ||A||_F) and ||Q^T Q - I||_F / n with cuBLAS DGEMMs (torch.matmul, test-side).  T is
+    applied as a tridiagonal (column shifts), never formed."""
+    nb, k = 16, 1024
+    if kind == "clusters":
+        A, _ = trid_gen.clustered_symmetric(n, seed, kind="clusters", device="cuda:0")
+    else:
+        A = trid_gen.random_symmetric(n, seed, device="cuda:0")
     A0 = A.clone()
     d, e, tau1, V2, tau2 = trid.sytrd_2stage(A, b, nb=nb, k=k)
     Qs = torch.eye(n, dtype=torch.float64, device="cuda:0")   # storage of the column-major identity
@@ -146,4 +152,4 @@ def test_exact_gates_timed_input_n32768(dev):
     G.diagonal().sub_(1.0)
     g2 = float(torch.linalg.norm(G)) / n
     assert g1 <= 1e-14 and g2 <= 1e-14, (g1, g2)
-    print(f"n=32768 seed 3001 exact G1={g1:.3e} G2={g2:.3e}")
+    print(f"n={n} b={b} seed {seed} {kind}: exact G1={g1:.3e} G2={g2:.3e}")
