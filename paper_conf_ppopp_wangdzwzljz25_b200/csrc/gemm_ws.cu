@@ -105,6 +105,11 @@ struct WsArgs {
   // ld): two stacked operands [op(A); op(A2)] sharing B in one launch (the Z builder's U = [Z_<^T W; Y_<^T W])
   const double* A2;
   int64_t msplit;
+  // symm_tma (SYMM, A op N K-tiles only): the m-inner A tiles of the row strip (A, dims {m, m}) and of the
+  // correction segments (CA[i], dims {m, ncorr}) are staged by one tensor copy each (box {BM + 4, BK}, lands as the
+  // padded [BK][BM + 4] stage); the transposed column strip, W and CB keep the cp.async producer
+  int symm_tma;
+  CUtensorMap tmSA, tmSC[2];
 };
 
 template <bool MG>
@@ -252,7 +257,7 @@ __device__ __forceinline__ bool corr_seg(const WsArgs& a, int z, int i, Seg& sg)
   const int64_t s0 = a.K[0] + i * a.ncorr, s1 = s0 + a.ncorr;
   const int64_t b0 = k0 > s0 ? k0 : s0, e0 = k1 < s1 ? k1 : s1;
   if (e0 <= b0) return false;
-  sg = Seg{a.CA[i], a.CB[i], a.ldca, a.ldcb, b0 - s0, e0 - s0, OP_N, 0, 0, 0};
+  sg = Seg{a.CA[i], a.CB[i], a.ldca, a.ldcb, b0 - s0, e0 - s0, OP_N, 0, 0, 0, 2 + i};
   return true;
 }
 
@@ -266,6 +271,9 @@ __device__ __forceinline__ void cp8(double* dst, const double* src, int bytes) {
 }
 __device__ __forceinline__ void cp_arrive_noinc(uint64_t* bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, unsigned bytes) {
+  asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
 // 2D tensor copy global -> shared (TMA), completing on an mbarrier; c0 = innermost (row) coordinate
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int c0, int c1, uint64_t* bar) {
@@ -329,7 +337,7 @@ __device__ __forceinline__ void load_kinner16(double* T, const double* base, int
 // Producer: one K-tile of A and B into stage buffers (NP threads).
 template <int BM, int BN, int NP, bool MG>
 __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t k0, int64_t m0, int64_t n0,
-                                          double* As, double* Bs, int pt) {
+                                          double* As, double* Bs, int pt, bool skip_a = false) {
   using C = Cfg<BM, BN>;
   const int64_t kend = s.ke;
   // the triangle masks only bite on K-tiles that overlap the diagonal block [m0, m0 + BM)
@@ -340,7 +348,9 @@ __device__ __forceinline__ void load_tile(const WsArgs& a, const Seg& s, int64_t
                         (s.mask == 2 && km(k0) > rm(m0 + BM - 1));
   const bool v16 = a.vec16 && unmasked;
   // ---- A
-  if (v16) {
+  if (skip_a) {
+    // staged by a tensor copy (the SYMM's row strip / correction operands, see ws_kernel)
+  } else if (v16) {
     if (s.opa == OP_N) load_minner16<BM, C::A_LD_N, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt);
     else if (s.seg == 0 && a.A2)
       load_kinner16<BM, C::A_LD_T, NP>(As, s.A, s.lda, m0, a.M, k0, kend, pt, a.A2, a.msplit);
@@ -523,7 +533,22 @@ __global__ void __launch_bounds__((CWM * CWN + NPW) * 32, 1) ws_kernel(const __g
           const uint32_t use = kt / STAGES;
           if (use > 0) mbar_wait(&empty[slot], (use - 1) & 1u);
           double* As = smem + (size_t)slot * C::STAGE;
-          load_tile<BM, BN, NPW * 32, MG>(a, sgm, k0, m0, n0, As, As + C::A_ELEMS, pt);
+          bool tma_a = false;
+          if constexpr (!MG && OPB == OP_N && BN <= 64) {
+            // SYMM: an m-inner A tile that is unmasked and not cut short inside its tensor goes by tensor copy;
+            // thread 0 registers its bytes (expect_tx, no arrival) before its own noinc arrival can complete the
+            // phase, so the slot cannot complete without the copy
+            if (a.symm_tma && sgm.opa == OP_N) {
+              const int64_t kext = sgm.seg >= 2 ? a.ncorr : a.K[0];
+              const bool unm = sgm.mask == 0 || (sgm.mask == 1 && k0 + BK - 1 <= m0);
+              tma_a = unm && (k0 + BK <= sgm.ke || sgm.ke == kext);
+              if (tma_a && pt == 0) {
+                mbar_expect_tx(&full[slot], (unsigned)((BM + 4) * BK * 8));
+                tma_load_2d(As, sgm.seg >= 2 ? &a.tmSC[sgm.seg - 2] : &a.tmSA, (int)m0, (int)k0, &full[slot]);
+              }
+            }
+          }
+          load_tile<BM, BN, NPW * 32, MG>(a, sgm, k0, m0, n0, As, As + C::A_ELEMS, pt, tma_a);
           cp_arrive_noinc(&full[slot]);
         }
       };
@@ -960,6 +985,13 @@ cudaError_t symm_ws(int64_t m, int64_t w, const double* A, int64_t lda, const do
   if (sp < 1) sp = 1;
   a.splits = (int)sp;
   a.part = part; a.part_ld = m; a.part_stride = m * w;
+  // tensor copies for the m-inner A tiles (TRID_WS_TMA: default 2 on; 0 / 1 keep cp.async for every tile)
+  const char* tenv = getenv("TRID_WS_TMA");
+  if ((!tenv || atoi(tenv) == 2) && a.vec16) {
+    bool ok = ws::encode_map(&a.tmSA, A, m, m, lda, 128 + 4, ws::BK);
+    for (int i = 0; i < 2 && ok && nc > 0; ++i) ok = ws::encode_map(&a.tmSC[i], a.CA[i], m, nc, ldca, 128 + 4, ws::BK);
+    a.symm_tma = ok ? 1 : 0;
+  }
   if (w <= 32 && ws::narrow_tiles()) return ws::launch<128, 32, 8, 1, OP_N>(a, st);
   return ws::launch<128, 64, 4, 2, OP_N>(a, st);
 }
