@@ -10,8 +10,12 @@
 //   * CWM x CWN consumer warps (2 per SMSP) wait only on full[slot]; there is no CTA-wide barrier;
 //   * the grid is persistent: each CTA walks work units (tile, split) with stride gridDim.x, so the
 //     producer prefetches the next unit while the consumers run the epilogue.
-//   * NT contractions on 128 x 128 tiles (the deferred syr2k): producer warp 0 alone stages every k-row of A and B
-//     with one bulk copy (TMA, cp.async.bulk ... mbarrier::complete_tx) into the padded, bank-conflict-free layout;
+//   * NT contractions on 128 x 128 tiles (the deferred syr2k): producer thread 0 alone stages each operand tile with
+//     ONE tensor copy (TMA, cp.async.bulk.tensor.2d from FP64 tensor maps, box {BM + 4, BK}) straight into the
+//     padded, bank-conflict-free layout (TRID_WS_TMA=1: one bulk copy per k-row; 0: cp.async);
+//   * the SYMM: its m-inner A tiles (row strip, correction operands) by tensor copies registered with expect_tx next
+//     to the cp.async producer's noinc arrivals on the same slot barrier (the k-inner operands stay on cp.async);
+//   * 128 x 128, 128 x 64 and (N <= 32) 128 x 32 tiles;
 //   * epilogue: a thread's Cin values are loaded in batches before any store (Cin may alias C);
 //   * triangular unit order grouped in bands of 8 tile rows (L2 reuse of the Y/Z strips: DRAM 65 -> 15 GB).
 // A unit's K range is a list of up to two segments; each segment has its own A/B pointers, leading
